@@ -1,0 +1,192 @@
+/*
+ * reduce.h -- C ABI of libreduce_b200.so, a B200-native (sm_100a) device-wide
+ * parallel reduction: one contiguous int32 / fp32 / fp64 array -> one scalar,
+ * with op = sum, min or max.
+ *
+ * What the operation is (PAPER.md = the CGO'19 paper "Automatic Generation of
+ * Warp-Level Primitives and Atomic Instructions for Fast and Portable Parallel
+ * Reduction on GPUs"; citations P:Lnnn are its line numbers):
+ *   - the spectrum `int sum(const Array<1,int> in)` returns one scalar, computed
+ *     by the sequential codelet `accum += in[i]` (Fig. 1(a), sec. II.B.1);
+ *   - the op set is the atomic Map API add / max / min (sec. III.A);
+ *     `atomicSub` is not a reduction (not associative) and is not offered;
+ *   - the host entry point takes the device input and leaves the result in
+ *     device memory (Listing 1/2 `Reduce_Grid`).
+ * How it is computed (steps S0-S7 of DESIGN.md): per-thread register
+ * accumulation over 32-byte vector loads of a block-tiled / thread-strided
+ * partition (Fig. 1(b)), a warp combine (shuffle / redux.sync,
+ * Listing 4), a block combine (shared `partial[32]` "Vs", shared
+ * atomics "VA1"/"VA2+S" Fig. 3, or a barrier'd shared tree "V"
+ * Fig. 1(c)), and a grid combine (global atomics "DT,A" Listing 2, a
+ * second kernel Listing 1, or a last-block pass).
+ *
+ * Conventions common to every entry point
+ *   - Pointers: `in`/`out` are DEVICE pointers on the current CUDA device and
+ *     are owned by the caller.  `out` receives exactly one element of the
+ *     input's dtype and must not overlap `in`.  `in` must be aligned to the
+ *     element size; any coarser misalignment is handled internally.
+ *   - Asynchrony: every call is stream-ordered on `stream` and returns without
+ *     host synchronisation (except reduce_host, see there).  The library owns
+ *     only a small per-(device, stream) workspace, allocated on first use or by
+ *     reduce_prepare(); calls are CUDA-graph capturable once prepared.
+ *   - Errors: functions return a reduce_status_t.  Invalid arguments are
+ *     rejected before any CUDA call is made.  Launch failures are reported as
+ *     REDUCE_ERR_CUDA; asynchronous faults surface at the caller's next
+ *     synchronisation, as in CUDA.  Nothing aborts, exits or throws across the
+ *     ABI.  reduce_last_error() gives a thread-local detail message.
+ *   - Semantics: int32 sum wraps modulo 2^32; fp sums
+ *     accumulate in the element type within a block (fp32 block partials are
+ *     combined across blocks in fp64); min/max are exact, NaN anywhere gives a
+ *     canonical quiet NaN and -0.0 < +0.0; n == 0 writes the identity
+ *     (0, INT32_MAX/+inf for min, INT32_MIN/-inf for max).
+ *   - Determinism: REDUCE_MODE_DETERMINISTIC uses no atomic instruction at all
+ *     (partials + a second kernel); its result bits depend only on
+ *     (dtype, op, n, in % 32, SM count).  REDUCE_MODE_FAST combines blocks with
+ *     global atomics: int32 and min/max results are still exact; fp sums may
+ *     differ run to run in the last bits.
+ */
+#ifndef REDUCE_B200_H
+#define REDUCE_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Same type as cudaStream_t (no CUDA header needed to use this ABI). NULL is
+ * the legacy default stream. */
+typedef struct CUstream_st* reduce_stream_t;
+
+typedef enum { REDUCE_INT32 = 0, REDUCE_FLOAT32 = 1, REDUCE_FLOAT64 = 2 } reduce_dtype_t;
+typedef enum { REDUCE_SUM = 0, REDUCE_MIN = 1, REDUCE_MAX = 2 } reduce_op_t;
+typedef enum { REDUCE_MODE_FAST = 0, REDUCE_MODE_DETERMINISTIC = 1 } reduce_mode_t;
+
+typedef enum {
+  REDUCE_OK = 0,
+  REDUCE_ERR_INVALID_ARG = 1,  /* bad dtype/op/option, NULL or misaligned pointer */
+  REDUCE_ERR_UNSUPPORTED = 2,  /* e.g. no sm_100 device, NCCL not loadable */
+  REDUCE_ERR_CUDA = 3,         /* a CUDA runtime call or launch failed */
+  REDUCE_ERR_NCCL = 4,         /* an NCCL call failed */
+  REDUCE_ERR_NO_MEMORY = 5,    /* workspace allocation failed */
+  REDUCE_ERR_NOT_PREPARED = 6  /* workspace missing/too small during graph capture */
+} reduce_status_t;
+
+/* Block combine (step S4), the paper's cooperative codelets:
+ *   SHFL        "Vs"   : warp shuffle/redux -> shared partial[32] -> warp 0
+ *                        (Fig. 1(c) after the shuffle pass, Listing 4)
+ *   SMEM_ATOMIC_WARP "VA2+S": warp shuffle, lane 0 atomically combines into one
+ *                        shared accumulator (Fig. 3(b), Listing 3)
+ *   SMEM_ATOMIC_ALL  "VA1"  : every thread atomically combines into one shared
+ *                        accumulator (Fig. 3(a))
+ *   SMEM_TREE   "V"    : shared-memory tree with a barrier per step
+ *                        (Fig. 1(c) lines 9-13) */
+typedef enum {
+  REDUCE_BC_SHFL = 0,
+  REDUCE_BC_SMEM_ATOMIC_WARP = 1,
+  REDUCE_BC_SMEM_ATOMIC_ALL = 2,
+  REDUCE_BC_SMEM_TREE = 3
+} reduce_block_combine_t;
+
+/* Grid combine (step S5):
+ *   DIRECT     : a single block writes the result (warp-only / single-block paths)
+ *   ATOMIC     : "DT,A" -- one global atomic per block into a self-resetting
+ *                accumulator, the last block (ticket) publishes it (Listing 2)
+ *   TWO_PASS   : per-block partials + a second single-block kernel, no atomics
+ *                (Listing 1 + second spectrum call)
+ *   LAST_BLOCK : per-block partials; the last block (integer ticket) reduces
+ *                them in a fixed order -- deterministic, one launch */
+typedef enum {
+  REDUCE_GC_DIRECT = 0,
+  REDUCE_GC_ATOMIC = 1,
+  REDUCE_GC_TWO_PASS = 2,
+  REDUCE_GC_LAST_BLOCK = 3
+} reduce_grid_combine_t;
+
+/* Options for reduce_ex & co.  Zero-initialise, then set fields; every field
+ * has an "auto" value (-1 or 0) that takes the dispatch table's choice. */
+typedef struct {
+  int mode;           /* -1 = process default (reduce_set_mode), else reduce_mode_t */
+  int grid_combine;   /* -1 = auto, else reduce_grid_combine_t */
+  int block_combine;  /* -1 = auto, else reduce_block_combine_t */
+  int block;          /* threads per block: 0 = auto, else 32..1024, multiple of 32
+                         (power of two for SMEM_TREE) */
+  int unroll;         /* 32-byte vectors per thread per tile: 0 = auto, else 1,2,4,8 */
+  int grid;           /* 0 = auto (one block per tile, capped), else max blocks */
+} reduce_opts_t;
+
+/* What a call will launch (filled by reduce_query_plan). */
+typedef struct {
+  int grid_combine, block_combine;
+  int grid, block, unroll;
+  int launches;        /* kernel launches per call: 1, or 2 for TWO_PASS */
+  int slots;           /* global accumulator slots used by ATOMIC */
+  int head, tail;      /* scalar elements before / after the 32-byte-aligned body */
+  long long tiles;     /* B*unroll-vector tiles in the body */
+  long long chain;     /* longest fp addition chain L (error bound (L+1)u*sum|x|) */
+} reduce_plan_t;
+
+/* Reduce in[0..n) with `op` into *out (device).  Uses the process-default mode. */
+int reduce(int dtype, int op, const void* in, size_t n, void* out, reduce_stream_t stream);
+
+/* As reduce(), with explicit mode / variant / launch overrides (opts may be NULL). */
+int reduce_ex(int dtype, int op, const void* in, size_t n, void* out, reduce_stream_t stream,
+              const reduce_opts_t* opts);
+
+/* Describe what reduce_ex(dtype, op, in, n, ..., opts) would launch on the
+ * current device.  `in` is only used for its address modulo 32 (may be any
+ * value when n == 0).  No CUDA work is issued. */
+int reduce_query_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* opts,
+                      reduce_plan_t* plan);
+
+/* Allocate (or grow) the workspace of (current device, stream) so that calls
+ * with up to `max_n` elements need no allocation -- call before graph capture.
+ * Also re-initialises the atomic accumulators and tickets (recovery after an
+ * aborted kernel). */
+int reduce_prepare(reduce_stream_t stream, size_t max_n);
+
+void reduce_set_mode(int mode);  /* process-wide default for reduce(); invalid values ignored */
+int reduce_get_mode(void);
+
+/* End-to-end entry with HOST buffers: copies host_in (n elements; pinned memory
+ * gives copy/compute overlap, pageable memory works but serialises) to the
+ * device in chunks on `stream`, reduces each chunk while the next is in flight,
+ * combines the chunk results on the device and copies the single result to
+ * host_out.  Synchronises `stream` before returning, so *host_out is valid on
+ * return.  Uses a library-owned device staging buffer (2 x chunk bytes). */
+int reduce_host(int dtype, int op, const void* host_in, size_t n, void* host_out,
+                reduce_stream_t stream, const reduce_opts_t* opts);
+
+/* ---- sharded mode over NCCL (one process per GPU) -------------------------
+ * reduce_multi: every rank of `comm` calls it with its own local shard
+ * (n_local may differ per rank, and may be 0); each rank's local result is
+ * combined with one in-place ncclAllReduce of a single element on `stream`
+ * (fp min/max are combined as order-preserving integer keys so NaN / signed
+ * zero semantics match the single-GPU path).  Every rank's *out receives the
+ * global result.  In REDUCE_MODE_DETERMINISTIC the per-rank results are
+ * all-gathered and combined in rank order by one warp instead (bitwise
+ * reproducible for a fixed rank count).  `comm` is an ncclComm_t created by
+ * reduce_comm_init (or borrowed from elsewhere; never destroyed here).
+ * NCCL is loaded at run time (dlopen "libnccl.so.2"); without it these calls
+ * return REDUCE_ERR_UNSUPPORTED. */
+int reduce_multi(int dtype, int op, const void* in_local, size_t n_local, void* out,
+                 reduce_stream_t stream, void* comm);
+int reduce_multi_ex(int dtype, int op, const void* in_local, size_t n_local, void* out,
+                    reduce_stream_t stream, void* comm, const reduce_opts_t* opts);
+
+int reduce_comm_unique_id_bytes(void);           /* 128 (sizeof ncclUniqueId) */
+int reduce_comm_get_unique_id(void* id_out);     /* rank 0; broadcast the bytes */
+int reduce_comm_init(void** comm_out, const void* id, int nranks, int rank); /* after cudaSetDevice */
+int reduce_comm_destroy(void* comm);
+
+/* ---- diagnostics ---------------------------------------------------------- */
+const char* reduce_status_string(int status);
+const char* reduce_last_error(void);   /* thread-local detail of the last failure */
+int reduce_version(void);              /* 10000*major + 100*minor + patch */
+void reduce_shutdown(void);            /* free all library-owned workspaces */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* REDUCE_B200_H */

@@ -1,0 +1,255 @@
+"""Python binding of libreduce_b200.so (include/reduce.h) — argument marshalling only.
+
+Every step of the reduction runs in the library's sm_100a kernels; this module
+only converts tensors / arrays to (pointer, count, dtype) and calls the C ABI
+with the same names.  There is no CPU fallback: if the shared library is
+missing, importing the binding raises.  (The CPU oracle under ``oracle/`` is
+test infrastructure and is never imported here.)
+
+PyTorch is used only for device memory, streams and process groups.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libreduce_b200.so")
+
+INT32, FLOAT32, FLOAT64 = 0, 1, 2
+SUM, MIN, MAX = 0, 1, 2
+MODE_FAST, MODE_DETERMINISTIC = 0, 1
+BC_SHFL, BC_SMEM_ATOMIC_WARP, BC_SMEM_ATOMIC_ALL, BC_SMEM_TREE = 0, 1, 2, 3
+GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK = 0, 1, 2, 3
+OK = 0
+
+OPS = {"sum": SUM, "min": MIN, "max": MAX}
+DTYPE_NAMES = {"int32": INT32, "float32": FLOAT32, "float64": FLOAT64}
+ELEM_BYTES = {INT32: 4, FLOAT32: 4, FLOAT64: 8}
+
+# every symbol include/reduce.h declares (checked by tests/test_abi.py)
+ABI_SYMBOLS = (
+    "reduce", "reduce_ex", "reduce_query_plan", "reduce_prepare", "reduce_set_mode",
+    "reduce_get_mode", "reduce_host", "reduce_multi", "reduce_multi_ex",
+    "reduce_comm_unique_id_bytes", "reduce_comm_get_unique_id", "reduce_comm_init",
+    "reduce_comm_destroy", "reduce_status_string", "reduce_last_error", "reduce_version",
+    "reduce_shutdown",
+)
+
+
+class ReduceError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        msg = f"{where}: {status_string(status)}: {last_error()}"
+        super().__init__(msg)
+
+
+class reduce_opts_t(ctypes.Structure):
+    _fields_ = [("mode", ctypes.c_int), ("grid_combine", ctypes.c_int), ("block_combine", ctypes.c_int),
+                ("block", ctypes.c_int), ("unroll", ctypes.c_int), ("grid", ctypes.c_int)]
+
+
+class reduce_plan_t(ctypes.Structure):
+    _fields_ = [("grid_combine", ctypes.c_int), ("block_combine", ctypes.c_int),
+                ("grid", ctypes.c_int), ("block", ctypes.c_int), ("unroll", ctypes.c_int),
+                ("launches", ctypes.c_int), ("slots", ctypes.c_int),
+                ("head", ctypes.c_int), ("tail", ctypes.c_int),
+                ("tiles", ctypes.c_longlong), ("chain", ctypes.c_longlong)]
+
+    def as_dict(self) -> dict:
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+def _load() -> ctypes.CDLL:
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(
+            f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; g.build()'` "
+            "(there is no CPU fallback)")
+    L = ctypes.CDLL(LIB_PATH, mode=ctypes.RTLD_GLOBAL)
+    vp, sz, i = ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int
+    opts_p, plan_p = ctypes.POINTER(reduce_opts_t), ctypes.POINTER(reduce_plan_t)
+    sigs = {
+        "reduce": (i, [i, i, vp, sz, vp, vp]),
+        "reduce_ex": (i, [i, i, vp, sz, vp, vp, opts_p]),
+        "reduce_query_plan": (i, [i, i, vp, sz, opts_p, plan_p]),
+        "reduce_prepare": (i, [vp, sz]),
+        "reduce_set_mode": (None, [i]),
+        "reduce_get_mode": (i, []),
+        "reduce_host": (i, [i, i, vp, sz, vp, vp, opts_p]),
+        "reduce_multi": (i, [i, i, vp, sz, vp, vp, vp]),
+        "reduce_multi_ex": (i, [i, i, vp, sz, vp, vp, vp, opts_p]),
+        "reduce_comm_unique_id_bytes": (i, []),
+        "reduce_comm_get_unique_id": (i, [vp]),
+        "reduce_comm_init": (i, [ctypes.POINTER(vp), vp, i, i]),
+        "reduce_comm_destroy": (i, [vp]),
+        "reduce_status_string": (ctypes.c_char_p, [i]),
+        "reduce_last_error": (ctypes.c_char_p, []),
+        "reduce_version": (i, []),
+        "reduce_shutdown": (None, []),
+    }
+    for name, (res, args) in sigs.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    return L
+
+
+lib = _load()
+
+
+def status_string(status: int) -> str:
+    return lib.reduce_status_string(status).decode()
+
+
+def last_error() -> str:
+    return lib.reduce_last_error().decode()
+
+
+def _check(status: int, where: str) -> None:
+    if status != OK:
+        raise ReduceError(status, where)
+
+
+def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=0, grid=0):
+    if isinstance(mode, str):
+        mode = {"fast": MODE_FAST, "deterministic": MODE_DETERMINISTIC}[mode]
+    return reduce_opts_t(-1 if mode is None else int(mode),
+                         -1 if grid_combine is None else int(grid_combine),
+                         -1 if block_combine is None else int(block_combine),
+                         int(block), int(unroll), int(grid))
+
+
+def _op(op) -> int:
+    return OPS[op] if isinstance(op, str) else int(op)
+
+
+def _torch_dtype_code(t) -> int:
+    import torch
+    m = {torch.int32: INT32, torch.float32: FLOAT32, torch.float64: FLOAT64}
+    if t.dtype not in m:
+        raise TypeError(f"unsupported dtype {t.dtype} (int32, float32, float64)")
+    return m[t.dtype]
+
+
+def _stream_handle(stream, device=None) -> int:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream(device)
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def reduce_ptr(dtype: int, op, in_ptr: int, n: int, out_ptr: int, stream: int = 0, opts=None) -> None:
+    """Raw-pointer form of reduce_ex (device pointers, stream handle)."""
+    st = lib.reduce_ex(int(dtype), _op(op), ctypes.c_void_p(in_ptr), n, ctypes.c_void_p(out_ptr),
+                       ctypes.c_void_p(stream), ctypes.byref(opts) if opts is not None else None)
+    _check(st, "reduce_ex")
+
+
+def reduce(x, op="sum", out=None, stream=None, **opt_kw):
+    """Reduce a contiguous CUDA tensor to a 1-element device tensor (async)."""
+    import torch
+    if not x.is_cuda:
+        raise ValueError("reduce() takes a CUDA tensor; use reduce_host() for host data")
+    if not x.is_contiguous():
+        raise ValueError("input must be contiguous")
+    dt = _torch_dtype_code(x)
+    if out is None:
+        out = torch.empty(1, dtype=x.dtype, device=x.device)
+    opts = make_opts(**opt_kw) if opt_kw else None
+    reduce_ptr(dt, op, x.data_ptr(), x.numel(), out.data_ptr(), _stream_handle(stream, x.device), opts)
+    return out
+
+
+def query_plan(dtype, op, n: int, in_ptr: int = 0, **opt_kw) -> dict:
+    dt = DTYPE_NAMES[dtype] if isinstance(dtype, str) else int(dtype)
+    plan = reduce_plan_t()
+    opts = make_opts(**opt_kw) if opt_kw else None
+    st = lib.reduce_query_plan(dt, _op(op), ctypes.c_void_p(in_ptr or None), n,
+                               ctypes.byref(opts) if opts is not None else None, ctypes.byref(plan))
+    _check(st, "reduce_query_plan")
+    return plan.as_dict()
+
+
+def prepare(stream=None, max_n: int = 0) -> None:
+    _check(lib.reduce_prepare(ctypes.c_void_p(_stream_handle(stream)), max_n), "reduce_prepare")
+
+
+def set_mode(mode) -> None:
+    if isinstance(mode, str):
+        mode = {"fast": MODE_FAST, "deterministic": MODE_DETERMINISTIC}[mode]
+    lib.reduce_set_mode(int(mode))
+
+
+def get_mode() -> int:
+    return lib.reduce_get_mode()
+
+
+def reduce_host(x, op="sum", stream=None, **opt_kw):
+    """End-to-end: host array/tensor in, Python scalar out (copies inside the call)."""
+    import numpy as np
+    if hasattr(x, "numpy") and not isinstance(x, np.ndarray):
+        if x.is_cuda:
+            raise ValueError("reduce_host() takes host memory")
+        dt = _torch_dtype_code(x)
+        ptr, n = x.data_ptr(), x.numel()
+        npdt = {INT32: np.int32, FLOAT32: np.float32, FLOAT64: np.float64}[dt]
+    else:
+        x = np.ascontiguousarray(x)
+        npdt = x.dtype.type
+        dt = {np.dtype(np.int32): INT32, np.dtype(np.float32): FLOAT32, np.dtype(np.float64): FLOAT64}[x.dtype]
+        ptr, n = x.ctypes.data, x.size
+    res = np.zeros(1, dtype=npdt)
+    opts = make_opts(**opt_kw) if opt_kw else None
+    st = lib.reduce_host(dt, _op(op), ctypes.c_void_p(ptr or None), n, ctypes.c_void_p(res.ctypes.data),
+                         ctypes.c_void_p(_stream_handle(stream)), ctypes.byref(opts) if opts is not None else None)
+    _check(st, "reduce_host")
+    return res[0]
+
+
+# ------------------------------------------------------------- sharded mode
+class Comm:
+    """An NCCL communicator owned by the library (reduce_comm_init), bootstrapped
+    over a torch.distributed process group (the unique id travels through it)."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        nbytes = lib.reduce_comm_unique_id_bytes()
+        uid = (ctypes.c_char * nbytes)()
+        if rank == 0:
+            _check(lib.reduce_comm_get_unique_id(ctypes.cast(uid, ctypes.c_void_p)), "reduce_comm_get_unique_id")
+        obj = [bytes(uid) if rank == 0 else None]
+        src = dist.get_global_rank(group, 0) if group is not None else 0
+        dist.broadcast_object_list(obj, src=src, group=group)
+        uid = (ctypes.c_char * nbytes).from_buffer_copy(obj[0])
+        handle = ctypes.c_void_p()
+        _check(lib.reduce_comm_init(ctypes.byref(handle), ctypes.cast(uid, ctypes.c_void_p), world, rank),
+               "reduce_comm_init")
+        self.handle = handle.value
+        self.rank, self.world = rank, world
+
+    def destroy(self) -> None:
+        if self.handle:
+            _check(lib.reduce_comm_destroy(ctypes.c_void_p(self.handle)), "reduce_comm_destroy")
+            self.handle = None
+
+
+def reduce_multi(x, op, comm: Comm, out=None, stream=None, **opt_kw):
+    """Every rank passes its local CUDA shard; every rank gets the global result."""
+    import torch
+    dt = _torch_dtype_code(x)
+    if out is None:
+        out = torch.empty(1, dtype=x.dtype, device=x.device)
+    opts = make_opts(**opt_kw) if opt_kw else None
+    st = lib.reduce_multi_ex(dt, _op(op), ctypes.c_void_p(x.data_ptr() or None), x.numel(),
+                             ctypes.c_void_p(out.data_ptr()), ctypes.c_void_p(_stream_handle(stream, x.device)),
+                             ctypes.c_void_p(comm.handle), ctypes.byref(opts) if opts is not None else None)
+    _check(st, "reduce_multi_ex")
+    return out
+
+
+def shard_range(n: int, world: int, rank: int) -> tuple[int, int]:
+    """Contiguous shard [lo, hi) of rank r: floor(r*n/k) .. floor((r+1)*n/k)."""
+    return (rank * n) // world, ((rank + 1) * n) // world

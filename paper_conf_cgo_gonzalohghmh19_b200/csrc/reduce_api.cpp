@@ -1,0 +1,349 @@
+// reduce_api.cpp -- the C ABI of include/reduce.h: argument validation, the
+// dispatch step (S0), the per-(device, stream) workspace, and error reporting.
+// Every step of the reduction itself runs in the CUDA kernels; there is no
+// host or CPU fallback anywhere in this library.
+#include <atomic>
+#include <cmath>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <string>
+#include <utility>
+
+#include "reduce_runtime.h"
+
+namespace rb {
+
+struct DispatchEntry {
+  int dtype, op, mode, max_log2_bytes, block, unroll, grid_kind, bc;
+};
+#include "dispatch_table.inc"
+
+static thread_local std::string g_err;
+static std::atomic<int> g_mode{REDUCE_MODE_FAST};
+static std::mutex g_ws_mu;
+static std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
+
+void set_error(const std::string& msg) { g_err = msg; }
+int fail(int status, const std::string& msg) {
+  g_err = msg;
+  return status;
+}
+int cuda_fail(cudaError_t e, const char* what) {
+  g_err = std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")";
+  return REDUCE_ERR_CUDA;
+}
+int default_mode() { return g_mode.load(); }
+
+int num_sms() {
+  int dev = 0, sms = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 148;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms <= 0) return 148;
+  return sms;
+}
+
+static int elem_bytes(int dtype) { return dtype == REDUCE_FLOAT64 ? 8 : 4; }
+static int ilog2_ceil(unsigned long long v) {
+  int l = 0;
+  while ((1ull << l) < v && l < 63) ++l;
+  return l;
+}
+
+int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* opts, int raw_out, Plan* P) {
+  if (dtype < 0 || dtype > 2) return fail(REDUCE_ERR_INVALID_ARG, "dtype must be REDUCE_INT32/FLOAT32/FLOAT64");
+  if (op < 0 || op > 2) return fail(REDUCE_ERR_INVALID_ARG, "op must be REDUCE_SUM/MIN/MAX");
+  const int s = elem_bytes(dtype);
+  if (n > 0 && in == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "in is NULL with n > 0");
+  if (n > 0 && ((uintptr_t)in % (uintptr_t)s) != 0)
+    return fail(REDUCE_ERR_INVALID_ARG, "in is not aligned to the element size");
+  if (n > (size_t)1 << 46) return fail(REDUCE_ERR_INVALID_ARG, "n too large");
+
+  reduce_opts_t o;
+  o.mode = -1; o.grid_combine = -1; o.block_combine = -1; o.block = 0; o.unroll = 0; o.grid = 0;
+  if (opts) o = *opts;
+  int mode = o.mode < 0 ? g_mode.load() : o.mode;
+  if (mode != REDUCE_MODE_FAST && mode != REDUCE_MODE_DETERMINISTIC)
+    return fail(REDUCE_ERR_INVALID_ARG, "mode must be -1, REDUCE_MODE_FAST or REDUCE_MODE_DETERMINISTIC");
+  if (o.grid_combine < -1 || o.grid_combine > 3) return fail(REDUCE_ERR_INVALID_ARG, "bad grid_combine");
+  if (o.block_combine < -1 || o.block_combine > 3) return fail(REDUCE_ERR_INVALID_ARG, "bad block_combine");
+  if (o.unroll != 0 && o.unroll != 1 && o.unroll != 2 && o.unroll != 4 && o.unroll != 8)
+    return fail(REDUCE_ERR_INVALID_ARG, "unroll must be 0, 1, 2, 4 or 8");
+  if (o.block != 0 && (o.block < 32 || o.block > 1024 || o.block % 32 != 0))
+    return fail(REDUCE_ERR_INVALID_ARG, "block must be 0 or a multiple of 32 in [32, 1024]");
+  if (o.grid < 0) return fail(REDUCE_ERR_INVALID_ARG, "grid must be >= 0");
+  if (mode == REDUCE_MODE_DETERMINISTIC) {
+    if (o.grid_combine == REDUCE_GC_ATOMIC)
+      return fail(REDUCE_ERR_INVALID_ARG, "deterministic mode forbids the ATOMIC grid combine");
+    if (o.block_combine == REDUCE_BC_SMEM_ATOMIC_WARP || o.block_combine == REDUCE_BC_SMEM_ATOMIC_ALL)
+      return fail(REDUCE_ERR_INVALID_ARG, "deterministic mode forbids shared-atomic block combines");
+  }
+
+  // ---- S0: table lookup by ceil(log2(bytes))
+  const unsigned long long bytes = (unsigned long long)n * (unsigned long long)s;
+  const int lb = ilog2_ceil(bytes ? bytes : 1);
+  const DispatchEntry* e = nullptr;
+  for (const DispatchEntry& r : kDispatch) {
+    if ((r.dtype < 0 || r.dtype == dtype) && (r.op < 0 || r.op == op) && (r.mode < 0 || r.mode == mode) &&
+        lb <= r.max_log2_bytes) {
+      e = &r;
+      break;
+    }
+  }
+  if (!e) e = &kDispatch[sizeof(kDispatch) / sizeof(kDispatch[0]) - 1];
+
+  int block = o.block ? o.block : e->block;
+  int unroll = o.unroll ? o.unroll : e->unroll;
+  int bc = o.block_combine >= 0 ? o.block_combine : e->bc;
+  int gc;
+  if (o.grid_combine >= 0) gc = o.grid_combine;
+  else if (e->grid_kind == 0) gc = REDUCE_GC_DIRECT;
+  else gc = mode == REDUCE_MODE_DETERMINISTIC ? REDUCE_GC_TWO_PASS : REDUCE_GC_ATOMIC;
+  if (block > max_block_threads(dtype, op, unroll))
+    return fail(REDUCE_ERR_INVALID_ARG, "block too large for this (dtype, op, unroll): max " +
+                                            std::to_string(max_block_threads(dtype, op, unroll)));
+  if (bc == REDUCE_BC_SMEM_TREE && (block & (block - 1)) != 0)
+    return fail(REDUCE_ERR_INVALID_ARG, "SMEM_TREE needs a power-of-two block");
+
+  // ---- partition: head | 32-byte-aligned body of vectors | tail
+  const int ve = 32 / s;
+  size_t head = 0;
+  if (n > 0) {
+    const uintptr_t mis = (uintptr_t)in % 32u;
+    head = mis ? (32u - mis) / (uintptr_t)s : 0;
+    if (head > n) head = n;
+  }
+  const size_t rest = n - head;
+  const unsigned long long body_vecs = rest / ve;
+  const int tail = (int)(rest % ve);
+  const long long tile_vecs = (long long)block * unroll;
+  const long long tiles = (long long)((body_vecs + tile_vecs - 1) / tile_vecs);
+
+  long long grid;
+  if (gc == REDUCE_GC_DIRECT) {
+    grid = 1;
+  } else {
+    grid = tiles > 0 ? tiles : 1;
+    if (o.grid > 0 && o.grid < grid) grid = o.grid;
+    if ((gc == REDUCE_GC_TWO_PASS || gc == REDUCE_GC_LAST_BLOCK) && grid > kMaxPartialBlocks) grid = kMaxPartialBlocks;
+    if (grid > 0x7FFFFFFFll) grid = 0x7FFFFFFFll;
+  }
+  const int nslots = gc == REDUCE_GC_ATOMIC ? (int)(grid < 32 ? grid : 32) : 0;
+
+  // ---- longest fp addition chain L of this variant (for the G2 gate)
+  long long chain = 0;
+  if (op == REDUCE_SUM && dtype != REDUCE_INT32) {
+    const int na = dtype == REDUCE_FLOAT64 ? 4 : 8;
+    const long long tpb = (tiles + grid - 1) / grid;
+    const int nw = block / 32;
+    chain = (long long)unroll * tpb + 1 + ilog2_ceil(na);  // per-thread lanes (+head/tail) + lane tree
+    switch (bc) {
+      case REDUCE_BC_SHFL: chain += 5 + (nw > 1 ? 5 : 0); break;
+      case REDUCE_BC_SMEM_ATOMIC_WARP: chain += 5 + nw; break;
+      case REDUCE_BC_SMEM_ATOMIC_ALL: chain += block; break;
+      case REDUCE_BC_SMEM_TREE: chain += ilog2_ceil(block); break;
+    }
+    if (dtype == REDUCE_FLOAT32) {
+      // blocks combine in fp64: the cross-block error is < grid * 2^-53 relative,
+      // far below one fp32 ulp; the single fp64 -> fp32 rounding adds 1.
+      chain += gc == REDUCE_GC_DIRECT ? 0 : 1;
+    } else {
+      switch (gc) {
+        case REDUCE_GC_ATOMIC: chain += (grid + nslots - 1) / nslots + 5; break;
+        case REDUCE_GC_TWO_PASS: chain += (grid + 1023) / 1024 + 10; break;
+        case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + ilog2_ceil(block); break;
+        default: break;
+      }
+    }
+  }
+
+  P->dtype = dtype; P->op = op; P->mode = mode; P->n = n; P->elem = s;
+  LaunchDesc& d = P->d;
+  std::memset(&d, 0, sizeof(d));
+  d.dtype = dtype; d.op = op; d.in = in;
+  d.body = (const char*)in + head * s;
+  d.body_vecs = body_vecs; d.tiles = tiles;
+  d.head = (int)head; d.tail = tail;
+  d.grid = (int)grid; d.block = block; d.unroll = unroll; d.bc = bc; d.gc = gc;
+  d.raw_out = raw_out; d.nslots = nslots;
+
+  reduce_plan_t& p = P->pub;
+  p.grid_combine = gc; p.block_combine = bc;
+  p.grid = (int)grid; p.block = block; p.unroll = unroll;
+  p.launches = gc == REDUCE_GC_TWO_PASS ? 2 : 1;
+  p.slots = nslots; p.head = (int)head; p.tail = tail;
+  p.tiles = tiles; p.chain = chain;
+  return REDUCE_OK;
+}
+
+static void free_workspace(Workspace* w) {
+  int prev = 0;
+  cudaGetDevice(&prev);
+  cudaSetDevice(w->device);
+  if (w->base) cudaFree(w->base);
+  if (w->partials) cudaFree(w->partials);
+  if (w->staging) cudaFree(w->staging);
+  for (int i = 0; i < 2; ++i) {
+    if (w->ev_copied[i]) cudaEventDestroy(w->ev_copied[i]);
+    if (w->ev_done[i]) cudaEventDestroy(w->ev_done[i]);
+  }
+  if (w->copy_stream) cudaStreamDestroy(w->copy_stream);
+  cudaSetDevice(prev);
+  delete w;
+}
+
+int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+  std::lock_guard<std::mutex> lk(g_ws_mu);
+  Workspace*& w = g_ws[std::make_pair(dev, stream)];
+  const bool need_base = (w == nullptr);
+  const bool need_partials = (w == nullptr || w->partials_bytes < partials_bytes);
+  if (need_base || need_partials) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
+      if (need_base) g_ws.erase(std::make_pair(dev, stream));
+      return fail(REDUCE_ERR_NOT_PREPARED, "workspace missing or too small during stream capture: call reduce_prepare first");
+    }
+  }
+  if (need_base) {
+    Workspace* nw = new Workspace();
+    nw->device = dev;
+    nw->stream = stream;
+    const size_t base_bytes = kCombos * kSlotRegionBytes + kCombos * (size_t)kSlotBytes + kNumScalars * kScalarBytes;
+    e = cudaMalloc(&nw->base, base_bytes);
+    if (e != cudaSuccess) {
+      delete nw;
+      g_ws.erase(std::make_pair(dev, stream));
+      cudaGetLastError();
+      return fail(REDUCE_ERR_NO_MEMORY, "cudaMalloc(workspace) failed");
+    }
+    nw->slots = nw->base;
+    nw->tickets = nw->base + kCombos * kSlotRegionBytes;
+    nw->scalars = nw->tickets + kCombos * (size_t)kSlotBytes;
+    e = launch_init_workspace(nw->slots, nw->tickets, stream);
+    if (e != cudaSuccess) {
+      cudaFree(nw->base);
+      delete nw;
+      g_ws.erase(std::make_pair(dev, stream));
+      return cuda_fail(e, "workspace init kernel");
+    }
+    w = nw;
+  }
+  if (w->partials_bytes < partials_bytes) {
+    size_t want = partials_bytes < (64u << 10) ? (64u << 10) : partials_bytes;
+    char* p = nullptr;
+    // stream-ordered: the old buffer may still be read by queued kernels
+    e = cudaMallocAsync((void**)&p, want, stream);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(REDUCE_ERR_NO_MEMORY, "cudaMallocAsync(partials) failed");
+    }
+    if (w->partials) cudaFreeAsync(w->partials, stream);
+    w->partials = p;
+    w->partials_bytes = want;
+  }
+  *out = w;
+  return REDUCE_OK;
+}
+
+int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream) {
+  LaunchDesc& d = P->d;
+  const int combo = d.dtype * 3 + d.op;
+  d.out = out;
+  d.slots = ws->slots + combo * kSlotRegionBytes;
+  d.ticket = (unsigned*)(ws->tickets + combo * (size_t)kSlotBytes);
+  d.partials = ws->partials;
+  cudaError_t e = launch_reduce(d, stream);
+  if (e != cudaSuccess) return cuda_fail(e, "reduction kernel launch");
+  return REDUCE_OK;
+}
+
+static size_t partials_needed(const Plan& P) {
+  if (P.d.gc == REDUCE_GC_TWO_PASS || P.d.gc == REDUCE_GC_LAST_BLOCK)
+    return (size_t)P.d.grid * (size_t)grid_value_bytes(P.dtype, P.op);
+  return 0;
+}
+
+}  // namespace rb
+
+using namespace rb;
+
+extern "C" {
+
+int reduce_ex(int dtype, int op, const void* in, size_t n, void* out, reduce_stream_t stream,
+              const reduce_opts_t* opts) {
+  if (out == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "out is NULL");
+  const int s = (dtype == REDUCE_FLOAT64) ? 8 : 4;
+  if (((uintptr_t)out % (uintptr_t)s) != 0) return fail(REDUCE_ERR_INVALID_ARG, "out is not aligned to the element size");
+  Plan P;
+  int st = make_plan(dtype, op, in, n, opts, 0, &P);
+  if (st != REDUCE_OK) return st;
+  Workspace* ws = nullptr;
+  st = get_workspace((cudaStream_t)stream, partials_needed(P), &ws);
+  if (st != REDUCE_OK) return st;
+  return launch_plan(&P, ws, out, (cudaStream_t)stream);
+}
+
+int reduce(int dtype, int op, const void* in, size_t n, void* out, reduce_stream_t stream) {
+  return reduce_ex(dtype, op, in, n, out, stream, nullptr);
+}
+
+int reduce_query_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* opts, reduce_plan_t* plan) {
+  if (plan == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "plan is NULL");
+  Plan P;
+  // `in` is only used for alignment here; allow NULL by treating it as aligned
+  const void* probe = in ? in : (const void*)(uintptr_t)256;
+  int st = make_plan(dtype, op, probe, n, opts, 0, &P);
+  if (st != REDUCE_OK) return st;
+  *plan = P.pub;
+  return REDUCE_OK;
+}
+
+int reduce_prepare(reduce_stream_t stream, size_t max_n) {
+  // partials for the largest possible partials-based grid at max_n
+  const unsigned long long tiles_min_tile = (max_n + 255) / 256;  // smallest tile is 32 threads x 1 vector
+  long long g = (long long)(tiles_min_tile < (unsigned long long)kMaxPartialBlocks ? tiles_min_tile : kMaxPartialBlocks);
+  if (g < 1024) g = 1024;
+  Workspace* ws = nullptr;
+  int st = get_workspace((cudaStream_t)stream, (size_t)g * 8, &ws);
+  if (st != REDUCE_OK) return st;
+  cudaError_t e = launch_init_workspace(ws->slots, ws->tickets, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "workspace init kernel");
+  return REDUCE_OK;
+}
+
+void reduce_set_mode(int mode) {
+  if (mode == REDUCE_MODE_FAST || mode == REDUCE_MODE_DETERMINISTIC) g_mode.store(mode);
+}
+int reduce_get_mode(void) { return g_mode.load(); }
+
+const char* reduce_status_string(int status) {
+  switch (status) {
+    case REDUCE_OK: return "REDUCE_OK";
+    case REDUCE_ERR_INVALID_ARG: return "REDUCE_ERR_INVALID_ARG";
+    case REDUCE_ERR_UNSUPPORTED: return "REDUCE_ERR_UNSUPPORTED";
+    case REDUCE_ERR_CUDA: return "REDUCE_ERR_CUDA";
+    case REDUCE_ERR_NCCL: return "REDUCE_ERR_NCCL";
+    case REDUCE_ERR_NO_MEMORY: return "REDUCE_ERR_NO_MEMORY";
+    case REDUCE_ERR_NOT_PREPARED: return "REDUCE_ERR_NOT_PREPARED";
+  }
+  return "REDUCE_ERR_UNKNOWN";
+}
+
+const char* reduce_last_error(void) { return g_err.c_str(); }
+
+int reduce_version(void) { return 10000 * 0 + 100 * 1 + 0; }
+
+void reduce_shutdown(void) {
+  std::lock_guard<std::mutex> lk(g_ws_mu);
+  for (auto& kv : g_ws) {
+    if (kv.second) {
+      cudaStreamSynchronize(kv.second->stream);
+      free_workspace(kv.second);
+    }
+  }
+  g_ws.clear();
+}
+
+}  // extern "C"

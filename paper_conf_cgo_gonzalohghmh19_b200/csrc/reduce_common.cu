@@ -1,0 +1,48 @@
+// reduce_common.cu -- dtype switch for the per-dtype kernel translation units.
+#include "reduce_internal.h"
+
+namespace rb {
+
+cudaError_t launch_reduce_i32(const LaunchDesc&, cudaStream_t);
+cudaError_t launch_reduce_f32(const LaunchDesc&, cudaStream_t);
+cudaError_t launch_reduce_f64(const LaunchDesc&, cudaStream_t);
+cudaError_t combine_i32(int, const void*, long long, void*, int, int, cudaStream_t);
+cudaError_t combine_f32(int, const void*, long long, void*, int, int, cudaStream_t);
+cudaError_t combine_f64(int, const void*, long long, void*, int, int, cudaStream_t);
+cudaError_t init_i32(char*, char*, cudaStream_t);
+cudaError_t init_f32(char*, char*, cudaStream_t);
+cudaError_t init_f64(char*, char*, cudaStream_t);
+
+int grid_value_bytes(int dtype, int op) {
+  if (dtype == 0) return 4;            // int32: uint32 / int32
+  if (dtype == 1) return op == 0 ? 8 : 4;  // fp32: double sum / uint32 key
+  return 8;                            // fp64: double / uint64 key
+}
+
+cudaError_t launch_reduce(const LaunchDesc& d, cudaStream_t s) {
+  switch (d.dtype) {
+    case 0: return launch_reduce_i32(d, s);
+    case 1: return launch_reduce_f32(d, s);
+    case 2: return launch_reduce_f64(d, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_combine(int dtype, int op, const void* vals, long long count, void* out, int raw_out,
+                           int block, cudaStream_t s) {
+  switch (dtype) {
+    case 0: return combine_i32(op, vals, count, out, raw_out, block, s);
+    case 1: return combine_f32(op, vals, count, out, raw_out, block, s);
+    case 2: return combine_f64(op, vals, count, out, raw_out, block, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_init_workspace(void* slots_base, void* tickets_base, cudaStream_t s) {
+  cudaError_t e;
+  if ((e = init_i32((char*)slots_base, (char*)tickets_base, s)) != cudaSuccess) return e;
+  if ((e = init_f32((char*)slots_base, (char*)tickets_base, s)) != cudaSuccess) return e;
+  return init_f64((char*)slots_base, (char*)tickets_base, s);
+}
+
+}  // namespace rb

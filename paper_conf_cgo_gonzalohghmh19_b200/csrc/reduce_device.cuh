@@ -1,0 +1,346 @@
+// reduce_device.cuh -- device-side building blocks of the B200 reduction path.
+//
+// Element / accumulator traits per (dtype, op), the 32-byte streaming load, the
+// warp combine (step S3), the four block combines (step S4) and the grid
+// combines (step S5).  Citations P:Lnnn are PAPER.md lines (the CGO'19 paper);
+// section numbers are DESIGN.md's.
+//
+// Hardware facts this file relies on (measured on the B200, see
+// profiles/r01_probe_sm100.txt):
+//   * FMNMX / DSETP.MAX order -0.0 < +0.0, and `max.NaN.f32` / `min.NaN.f32`
+//     return the canonical NaN 0x7FFFFFFF whenever an input is NaN;
+//   * `redux.sync.{min,max}.NaN.f32` (CREDUX.*.F32.NAN) has the same semantics;
+//   * `ld.global.nc.L1::no_allocate.v8` is a single 256-bit LDG (sm_100 only).
+#pragma once
+#include <cstdint>
+#include <type_traits>
+#include <cuda_runtime.h>
+#include "reduce_internal.h"
+
+namespace rb {
+
+constexpr int DT_I32 = 0, DT_F32 = 1, DT_F64 = 2;
+constexpr int OP_SUM = 0, OP_MIN = 1, OP_MAX = 2;
+constexpr int BC_SHFL = 0, BC_ATOMIC_WARP = 1, BC_ATOMIC_ALL = 2, BC_TREE = 3;
+constexpr int GC_DIRECT = 0, GC_ATOMIC = 1, GC_TWO_PASS = 2, GC_LAST_BLOCK = 3;
+constexpr int kVecBytes = 32;    // one 256-bit load per thread per vector
+
+// ------------------------------------------------------------------ loads ---
+// Streaming 32-byte read-only load; never allocates in L1 (each byte is read
+// once).  Not `volatile`: the compiler may hoist/batch these (they read memory
+// no thread writes during the kernel).
+__device__ __forceinline__ void ld_v8(const void* p, uint32_t (&r)[8]) {
+  asm("ld.global.nc.L1::no_allocate.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
+      : "l"(p));
+}
+
+// ------------------------------------------------------- fp primitives ---
+__device__ __forceinline__ float fmax_nan(float a, float b) {
+  float r; asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r;
+}
+__device__ __forceinline__ float fmin_nan(float a, float b) {
+  float r; asm("min.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r;
+}
+__device__ __forceinline__ float redux_max_nan(float a) {
+  float r; asm("redux.sync.max.NaN.f32 %0, %1, 0xffffffff;" : "=f"(r) : "f"(a)); return r;
+}
+__device__ __forceinline__ float redux_min_nan(float a) {
+  float r; asm("redux.sync.min.NaN.f32 %0, %1, 0xffffffff;" : "=f"(r) : "f"(a)); return r;
+}
+// fp64 min/max: max.f64 is sign-aware but drops NaN; NaN is tracked separately
+// in the streaming loop and re-applied here for the combine trees.
+__device__ __forceinline__ double dmax_sel(double a, double b) {
+  double r; asm("max.f64 %0, %1, %2;" : "=d"(r) : "d"(a), "d"(b)); return r;
+}
+__device__ __forceinline__ double dmin_sel(double a, double b) {
+  double r; asm("min.f64 %0, %1, %2;" : "=d"(r) : "d"(a), "d"(b)); return r;
+}
+__device__ __forceinline__ double nan64() { return __longlong_as_double(0x7FF8000000000000ll); }
+
+// Order-preserving keys (reading R3): unsigned order of key(x) == the order
+// -inf < ... < -0.0 < +0.0 < ... < +inf, and NaN maps to the extreme that wins
+// for the op (0 for min, all-ones for max), so integer min/max atomics give the
+// exact fp min/max with NaN propagation.  Decoding the winning sentinel yields
+// the canonical quiet NaN.
+template <bool kMax>
+__device__ __forceinline__ uint32_t key32(float x) {
+  uint32_t b = __float_as_uint(x);
+  if (x != x) return kMax ? 0xFFFFFFFFu : 0u;
+  return (b & 0x80000000u) ? ~b : (b | 0x80000000u);
+}
+template <bool kMax>
+__device__ __forceinline__ uint32_t unkey32(uint32_t k) {
+  if (kMax ? (k == 0xFFFFFFFFu) : (k == 0u)) return 0x7FC00000u;
+  return (k & 0x80000000u) ? (k & 0x7FFFFFFFu) : ~k;
+}
+template <bool kMax>
+__device__ __forceinline__ unsigned long long key64(double x) {
+  unsigned long long b = (unsigned long long)__double_as_longlong(x);
+  if (x != x) return kMax ? ~0ull : 0ull;
+  return (b >> 63) ? ~b : (b | 0x8000000000000000ull);
+}
+template <bool kMax>
+__device__ __forceinline__ unsigned long long unkey64(unsigned long long k) {
+  if (kMax ? (k == ~0ull) : (k == 0ull)) return 0x7FF8000000000000ull;
+  return (k >> 63) ? (k & 0x7FFFFFFFFFFFFFFFull) : ~k;
+}
+
+// Generic butterfly for any 4/8-byte type with a combine functor; result in all lanes.
+template <class V, class F>
+__device__ __forceinline__ V warp_butterfly(V v, F f) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = f(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+// ------------------------------------------------------------- traits ---
+// Acc  : per-thread / warp / block value;  NA independent accumulators per thread.
+// Grid : type of the cross-block combine (atomics, partials, raw output).
+// fold(a, aux, x): a (+)= x for one element; aux carries fp64 NaN flags.
+template <int DT, int OP> struct Tr;
+
+template <int OP> struct TrI32 {
+  using Elem = int32_t;
+  using Acc = typename std::conditional<OP == OP_SUM, uint32_t, int32_t>::type;
+  using Grid = Acc;
+  static constexpr int VE = 8, NA = 8, kLaneWords = 1;
+  __device__ static Acc ident() {
+    return OP == OP_SUM ? Acc(0) : (OP == OP_MIN ? Acc(0x7FFFFFFF) : Acc(0x80000000));
+  }
+  __device__ static Acc comb(Acc a, Acc b) {
+    return OP == OP_SUM ? Acc(a + b) : (OP == OP_MIN ? (a < b ? a : b) : (a > b ? a : b));
+  }
+  __device__ static void fold(Acc& a, uint32_t&, uint32_t w) { a = comb(a, Acc(w)); }
+  __device__ static Acc warp(Acc v) {  // REDUX / CREDUX, one instruction
+    if (OP == OP_SUM) return __reduce_add_sync(0xffffffffu, (unsigned)v);
+    if (OP == OP_MIN) return __reduce_min_sync(0xffffffffu, (int)v);
+    return __reduce_max_sync(0xffffffffu, (int)v);
+  }
+  __device__ static Acc finish(Acc a, uint32_t) { return a; }
+  __device__ static Grid to_grid(Acc a) { return a; }
+  __device__ static Grid gident() { return ident(); }
+  __device__ static Grid gcomb(Grid a, Grid b) { return comb(a, b); }
+  __device__ static Grid gwarp(Grid v) { return warp(v); }
+  __device__ static void gred(Grid* p, Grid v) {  // global or shared (generic address)
+    if (OP == OP_SUM) atomicAdd((unsigned*)p, (unsigned)v);
+    else if (OP == OP_MIN) atomicMin((int*)p, (int)v);
+    else atomicMax((int*)p, (int)v);
+  }
+  __device__ static Grid gexch(Grid* p, Grid v) { return (Grid)atomicExch((unsigned*)p, (unsigned)v); }
+  __device__ static void finalize(Grid g, void* out) { *(int32_t*)out = (int32_t)g; }
+};
+
+template <int OP> struct TrF32 {
+  using Elem = float;
+  using Acc = float;
+  using Grid = typename std::conditional<OP == OP_SUM, double, uint32_t>::type;
+  static constexpr int VE = 8, NA = 8, kLaneWords = 1;
+  static constexpr bool kMax = OP == OP_MAX;
+  __device__ static Acc ident() {
+    return OP == OP_SUM ? 0.0f : (OP == OP_MIN ? __int_as_float(0x7F800000) : __int_as_float(0xFF800000));
+  }
+  __device__ static Acc comb(Acc a, Acc b) {
+    return OP == OP_SUM ? a + b : (OP == OP_MIN ? fmin_nan(a, b) : fmax_nan(a, b));
+  }
+  __device__ static void fold(Acc& a, uint32_t&, uint32_t w) { a = comb(a, __uint_as_float(w)); }
+  __device__ static Acc warp(Acc v) {
+    if (OP == OP_MIN) return redux_min_nan(v);
+    if (OP == OP_MAX) return redux_max_nan(v);
+    return warp_butterfly(v, [](float x, float y) { return x + y; });
+  }
+  __device__ static Acc finish(Acc a, uint32_t) { return a; }
+  // fp32 sums cross blocks in fp64 (accuracy at no bandwidth cost).
+  __device__ static Grid to_grid(Acc a) {
+    if constexpr (OP == OP_SUM) return (double)a; else return key32<kMax>(a);
+  }
+  __device__ static Grid gident() {
+    if constexpr (OP == OP_SUM) return 0.0; else return key32<kMax>(ident());
+  }
+  __device__ static Grid gcomb(Grid a, Grid b) {
+    if constexpr (OP == OP_SUM) return a + b; else return kMax ? (a > b ? a : b) : (a < b ? a : b);
+  }
+  __device__ static Grid gwarp(Grid v) {
+    if constexpr (OP == OP_SUM) return warp_butterfly(v, [](double x, double y) { return x + y; });
+    else return kMax ? __reduce_max_sync(0xffffffffu, v) : __reduce_min_sync(0xffffffffu, v);
+  }
+  __device__ static void gred(Grid* p, Grid v) {
+    if constexpr (OP == OP_SUM) atomicAdd(p, v);
+    else if constexpr (kMax) atomicMax(p, v);
+    else atomicMin(p, v);
+  }
+  __device__ static Grid gexch(Grid* p, Grid v) {
+    if constexpr (OP == OP_SUM)
+      return __longlong_as_double((long long)atomicExch((unsigned long long*)p, (unsigned long long)__double_as_longlong(v)));
+    else return atomicExch(p, v);
+  }
+  __device__ static void finalize(Grid g, void* out) {
+    if constexpr (OP == OP_SUM) {
+      float f = (float)g;
+      *(uint32_t*)out = (f != f) ? 0x7FC00000u : __float_as_uint(f);
+    } else {
+      *(uint32_t*)out = unkey32<kMax>(g);
+    }
+  }
+};
+
+template <int OP> struct TrF64 {
+  using Elem = double;
+  using Acc = double;
+  using Grid = typename std::conditional<OP == OP_SUM, double, unsigned long long>::type;
+  static constexpr int VE = 4, NA = 4, kLaneWords = 2;
+  static constexpr bool kMax = OP == OP_MAX;
+  __device__ static Acc ident() {
+    return OP == OP_SUM ? 0.0 : __longlong_as_double(OP == OP_MIN ? 0x7FF0000000000000ll : (long long)0xFFF0000000000000ull);
+  }
+  // NaN-propagating combine (trees): sign-aware select, then NaN override.
+  __device__ static Acc comb(Acc a, Acc b) {
+    if (OP == OP_SUM) return a + b;
+    double m = OP == OP_MIN ? dmin_sel(a, b) : dmax_sel(a, b);
+    return (a != a || b != b) ? nan64() : m;
+  }
+  // Streaming fold: select + a sticky NaN flag (cheaper than the full comb).
+  __device__ static void fold(Acc& a, uint32_t& aux, double x) {
+    if (OP == OP_SUM) { a += x; return; }
+    a = OP == OP_MIN ? dmin_sel(a, x) : dmax_sel(a, x);
+    aux |= (x != x) ? 1u : 0u;
+  }
+  __device__ static Acc warp(Acc v) { return warp_butterfly(v, [](double x, double y) { return comb(x, y); }); }
+  __device__ static Acc finish(Acc a, uint32_t aux) {
+    if (OP == OP_SUM) return a;
+    return aux ? nan64() : a;
+  }
+  __device__ static Grid to_grid(Acc a) {
+    if constexpr (OP == OP_SUM) return a; else return key64<kMax>(a);
+  }
+  __device__ static Grid gident() {
+    if constexpr (OP == OP_SUM) return 0.0; else return key64<kMax>(ident());
+  }
+  __device__ static Grid gcomb(Grid a, Grid b) {
+    if constexpr (OP == OP_SUM) return a + b; else return kMax ? (a > b ? a : b) : (a < b ? a : b);
+  }
+  __device__ static Grid gwarp(Grid v) { return warp_butterfly(v, [](Grid x, Grid y) { return gcomb(x, y); }); }
+  __device__ static void gred(Grid* p, Grid v) {
+    if constexpr (OP == OP_SUM) atomicAdd(p, v);
+    else if constexpr (kMax) atomicMax(p, v);
+    else atomicMin(p, v);
+  }
+  __device__ static Grid gexch(Grid* p, Grid v) {
+    if constexpr (OP == OP_SUM)
+      return __longlong_as_double((long long)atomicExch((unsigned long long*)p, (unsigned long long)__double_as_longlong(v)));
+    else return atomicExch(p, v);
+  }
+  __device__ static void finalize(Grid g, void* out) {
+    if constexpr (OP == OP_SUM) {
+      *(unsigned long long*)out = (g != g) ? 0x7FF8000000000000ull : (unsigned long long)__double_as_longlong(g);
+    } else {
+      *(unsigned long long*)out = unkey64<kMax>(g);
+    }
+  }
+};
+
+template <int OP> struct Tr<DT_I32, OP> : TrI32<OP> {};
+template <int OP> struct Tr<DT_F32, OP> : TrF32<OP> {};
+template <int OP> struct Tr<DT_F64, OP> : TrF64<OP> {};
+
+// Fold one 32-byte vector into the NA per-thread accumulators (lane k of the
+// vector goes to accumulator k: NA independent chains).
+template <class T>
+__device__ __forceinline__ void fold_vec(typename T::Acc (&a)[T::NA], uint32_t& aux, const uint32_t (&r)[8]) {
+  if constexpr (T::kLaneWords == 1) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) T::fold(a[k], aux, r[k]);
+  } else {
+#pragma unroll
+    for (int k = 0; k < 4; ++k) T::fold(a[k], aux, __hiloint2double((int)r[2 * k + 1], (int)r[2 * k]));
+  }
+}
+
+template <class T>
+__device__ __forceinline__ void fold_elem(typename T::Acc& a, uint32_t& aux, typename T::Elem e) {
+  if constexpr (T::kLaneWords == 1) T::fold(a, aux, *reinterpret_cast<const uint32_t*>(&e));
+  else T::fold(a, aux, e);
+}
+
+// Pairwise tree over the NA accumulators (depth log2 NA).
+template <class T>
+__device__ __forceinline__ typename T::Acc thread_result(typename T::Acc (&a)[T::NA], uint32_t aux) {
+#pragma unroll
+  for (int w = T::NA / 2; w > 0; w >>= 1)
+#pragma unroll
+    for (int k = 0; k < w; ++k) a[k] = T::comb(a[k], a[k + w]);
+  return T::finish(a[0], aux);
+}
+
+// ------------------------------------------------------ block combine (S4) --
+// Returns the block's value as T::Grid, valid in thread 0.
+template <class T, int BC>
+__device__ __forceinline__ typename T::Grid block_combine(typename T::Acc v) {
+  using Acc = typename T::Acc;
+  using Grid = typename T::Grid;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  if constexpr (BC == BC_SHFL) {
+    // "Vs": warp shuffle/redux, partial[32] in shared memory, warp 0 again
+    // (Listing 4 lines 14-29), padding with the op identity.
+    __shared__ Acc part[32];
+    Acc w = T::warp(v);
+    if (nw == 1) return T::to_grid(w);
+    if (lane == 0) part[wid] = w;
+    __syncthreads();
+    Grid g = T::gident();
+    if (wid == 0) {
+      Acc x = lane < nw ? part[lane] : T::ident();
+      g = T::to_grid(T::warp(x));
+    }
+    return g;
+  } else if constexpr (BC == BC_ATOMIC_WARP || BC == BC_ATOMIC_ALL) {
+    // "VA2+S" (Fig. 3(b) with the shuffle pass) or "VA1"
+    // (Fig. 3(a)): one shared accumulator updated atomically by lane 0
+    // of every warp, or by every thread.
+    __shared__ Grid acc;
+    if (threadIdx.x == 0) acc = T::gident();
+    __syncthreads();
+    if constexpr (BC == BC_ATOMIC_WARP) {
+      Acc w = T::warp(v);
+      if (lane == 0) T::gred(&acc, T::to_grid(w));
+    } else {
+      T::gred(&acc, T::to_grid(v));
+    }
+    __syncthreads();
+    return acc;
+  } else {
+    // "V": shared tree, one barrier per step (Fig. 1(c) lines 9-13 with the
+    // barrier Volta+ needs -- DESIGN.md reading R6).  blockDim.x must be a power of two.
+    __shared__ Acc tmp[1024];
+    tmp[threadIdx.x] = v;
+    __syncthreads();
+    for (int s = blockDim.x >> 1; s > 0; s >>= 1) {
+      if ((int)threadIdx.x < s) tmp[threadIdx.x] = T::comb(tmp[threadIdx.x], tmp[threadIdx.x + s]);
+      __syncthreads();
+    }
+    return T::to_grid(tmp[0]);
+  }
+}
+
+// Fixed-order reduction of `count` Grid values by the whole block: thread t
+// folds t, t+B, t+2B, ... then a shared tree over the B thread values.  Reads
+// with ld.global.cg (L2) since the values were written by other SMs.
+template <class T>
+__device__ __forceinline__ typename T::Grid reduce_grid_values(const typename T::Grid* vals, long long count) {
+  using Grid = typename T::Grid;
+  __shared__ Grid gtmp[1024];
+  Grid x = T::gident();
+  for (long long i = threadIdx.x; i < count; i += blockDim.x) x = T::gcomb(x, __ldcg(vals + i));
+  gtmp[threadIdx.x] = x;
+  __syncthreads();
+  int p2 = 1;
+  while (p2 < (int)blockDim.x) p2 <<= 1;
+  for (int s = p2 >> 1; s > 0; s >>= 1) {
+    if ((int)threadIdx.x < s && (int)threadIdx.x + s < (int)blockDim.x)
+      gtmp[threadIdx.x] = T::gcomb(gtmp[threadIdx.x], gtmp[threadIdx.x + s]);
+    __syncthreads();
+  }
+  return gtmp[0];
+}
+
+}  // namespace rb

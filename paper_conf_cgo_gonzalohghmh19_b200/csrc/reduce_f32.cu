@@ -1,0 +1,11 @@
+// reduce_f32.cu -- instantiates the reduction kernels for one dtype (split per
+// dtype so the 48 kernel instantiations per dtype compile in parallel).
+#include "reduce_kernels.cuh"
+
+namespace rb {
+cudaError_t launch_reduce_f32(const LaunchDesc& d, cudaStream_t s) { return launch_dt<DT_F32>(d, s); }
+cudaError_t combine_f32(int op, const void* v, long long c, void* out, int raw, int block, cudaStream_t s) {
+  return combine_dt<DT_F32>(op, v, c, out, raw, block, s);
+}
+cudaError_t init_f32(char* slots, char* tickets, cudaStream_t s) { return init_dt<DT_F32>(slots, tickets, s); }
+}  // namespace rb

@@ -1,0 +1,56 @@
+// reduce_internal.h -- interface between the host runtime (reduce_api.cpp,
+// reduce_multi.cpp) and the kernel translation units.  Not part of the ABI.
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace rb {
+
+constexpr int kSlotBytes = 256;  // stride between global accumulator slots (separate L2 lines)
+constexpr int kMaxSlots = 32;
+
+// Largest block the (dtype, op, unroll) instantiation is compiled for: the
+// register budget of 64/thread at 1024 threads is too small for 8 in-flight
+// 32-byte loads, and for the fp64 min/max select+NaN-flag fold at unroll >= 2.
+constexpr int max_block_threads(int dtype, int op, int unroll) {
+  return (unroll >= 8 || (dtype == 2 && op != 0 && unroll >= 2)) ? 512 : 1024;
+}
+
+// One launch of the main reduction kernel (steps S2-S5), fully resolved by the
+// host dispatcher (step S0).
+struct LaunchDesc {
+  int dtype, op;
+  const void* in;                // original input pointer (element-aligned)
+  const void* body;              // first 32-byte-aligned element of the body
+  unsigned long long body_vecs;  // 32-byte vectors in the body
+  long long tiles;               // ceil(body_vecs / (block*unroll))
+  int head, tail;                // scalar elements before / after the body
+  int grid, block, unroll, bc, gc;
+  void* out;                     // device scalar (T, or the raw Grid type)
+  int raw_out;                   // 1: write the un-finalised Grid value
+  void* slots;                   // this (dtype, op)'s accumulator slots (GC_ATOMIC)
+  int nslots;
+  unsigned* ticket;              // this (dtype, op)'s ticket (GC_ATOMIC / GC_LAST_BLOCK)
+  void* partials;                // Grid[grid] (GC_TWO_PASS / GC_LAST_BLOCK)
+};
+
+// Size in bytes of the Grid (cross-block) type of (dtype, op).
+int grid_value_bytes(int dtype, int op);
+
+cudaError_t launch_reduce(const LaunchDesc& d, cudaStream_t s);
+
+// Reduce `count` Grid-typed values in a fixed order with one block of
+// `block` threads and write the finalised (or raw) result to `out`.
+cudaError_t launch_combine(int dtype, int op, const void* vals, long long count, void* out,
+                           int raw_out, int block, cudaStream_t s);
+
+// Write the identity into every accumulator slot of every (dtype, op) and zero
+// the tickets.  slots_base: 9 regions of kMaxSlots*kSlotBytes; tickets: 9 words
+// spaced kSlotBytes apart.
+cudaError_t launch_init_workspace(void* slots_base, void* tickets_base, cudaStream_t s);
+
+constexpr int kCombos = 9;  // 3 dtypes x 3 ops
+constexpr size_t kSlotRegionBytes = (size_t)kMaxSlots * kSlotBytes;
+
+}  // namespace rb

@@ -1,0 +1,246 @@
+// reduce_kernels.cuh -- the reduction kernels (steps S2-S6 of DESIGN.md) as
+// templates, instantiated per dtype in reduce_{i32,f32,f64}.cu.
+//
+// k_reduce<DT, OP, U, BC>: one kernel covers the paper's warp-only, single-block
+// and grid-level versions (Fig. 6):
+//   * partition (S2): the 32-byte-aligned body is cut into tiles of
+//     blockDim.x * U vectors; tiles go to blocks ("Global Atomic Tile
+//     Distribute", DT at grid level) and, inside a tile, vectors go to threads
+//     with stride blockDim.x ("Stride Distribute", DS at thread level) -- the
+//     large-array winners (b), (e) of P:L687 -- so each warp load instruction
+//     covers 1 KB contiguous.  Each thread issues its U 256-bit loads before
+//     consuming any (memory-level parallelism), folding into NA independent
+//     register accumulators (Fig. 1(a)'s `accum += in[i]`).
+//     With grid == tiles (the default) every block does exactly one tile and
+//     the hardware block scheduler balances the tail across the 148 SMs; with
+//     a smaller grid, blocks loop over tiles (persistent, Catanzaro-style
+//     two-stage); grid == 1 is the single-block / warp-only path.
+//   * head (< 32 B before the aligned body) and tail (< 32 B after it) are
+//     folded by the last block's threads 0..7 and 8..15.
+//   * warp / block combine (S3, S4): block_combine<BC>.
+//   * grid combine (S5) and finalise (S6): by desc.gc, see grid_combine().
+#pragma once
+#include <type_traits>
+#include "reduce_device.cuh"
+#include "reduce_internal.h"
+
+namespace rb {
+
+struct KParams {
+  const char* in;
+  const char* body;
+  unsigned long long body_vecs;
+  long long tiles;
+  int head, tail;
+  void* out;
+  int raw_out;
+  int gc;
+  void* slots;
+  int nslots;
+  unsigned* ticket;
+  void* partials;
+};
+
+template <class T>
+__device__ __forceinline__ void store_out(typename T::Grid g, const KParams& p) {
+  if (p.raw_out) *(typename T::Grid*)p.out = g;
+  else T::finalize(g, p.out);
+}
+
+template <class T>
+__device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& p) {
+  using Grid = typename T::Grid;
+  __shared__ int s_last;
+  if (p.gc == GC_DIRECT) {
+    if (threadIdx.x == 0) store_out<T>(g, p);
+    return;
+  }
+  if (p.gc == GC_TWO_PASS) {  // Listing 1: Return[blockIdx.x] = ...; second launch reduces
+    if (threadIdx.x == 0) ((Grid*)p.partials)[blockIdx.x] = g;
+    return;
+  }
+  if (p.gc == GC_ATOMIC) {
+    // Listing 2's `atomicAdd(Return, ...)` per block, spread over
+    // nslots accumulators on separate L2 lines; the ticket's last holder
+    // collects the slots (atomicExch resets them to the identity, so no memset
+    // is ever needed) and publishes the result.
+    if (threadIdx.x == 0) {
+      Grid* slot = (Grid*)((char*)p.slots + (size_t)(blockIdx.x % p.nslots) * kSlotBytes);
+      T::gred(slot, g);
+      __threadfence();
+      unsigned tk = atomicAdd(p.ticket, 1u);
+      s_last = (tk == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (s_last && threadIdx.x < 32) {
+      __threadfence();
+      const int lane = threadIdx.x;
+      Grid x = T::gident();
+      if (lane < p.nslots) x = T::gexch((Grid*)((char*)p.slots + (size_t)lane * kSlotBytes), T::gident());
+      x = T::gwarp(x);
+      if (lane == 0) {
+        store_out<T>(x, p);
+        atomicExch(p.ticket, 0u);
+      }
+    }
+    return;
+  }
+  // GC_LAST_BLOCK: partials + ticket; the last block reduces them in a fixed
+  // order (deterministic; the only atomic touches the integer ticket).
+  if (threadIdx.x == 0) {
+    ((Grid*)p.partials)[blockIdx.x] = g;
+    __threadfence();
+    unsigned tk = atomicAdd(p.ticket, 1u);
+    s_last = (tk == gridDim.x - 1);
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    Grid x = reduce_grid_values<T>((const Grid*)p.partials, gridDim.x);
+    if (threadIdx.x == 0) {
+      store_out<T>(x, p);
+      atomicExch(p.ticket, 0u);
+    }
+  }
+}
+
+template <int DT, int OP, int U, int BC>
+__global__ void __launch_bounds__(max_block_threads(DT, OP, U)) k_reduce(const KParams p) {
+  using T = Tr<DT, OP>;
+  using Acc = typename T::Acc;
+  Acc a[T::NA];
+#pragma unroll
+  for (int k = 0; k < T::NA; ++k) a[k] = T::ident();
+  uint32_t aux = 0;
+
+  const long long B = blockDim.x;
+  const long long tile_vecs = B * U;
+  for (long long tile = blockIdx.x; tile < p.tiles; tile += gridDim.x) {
+    const unsigned long long v0 = (unsigned long long)(tile * tile_vecs) + threadIdx.x;
+    const char* ptr = p.body + v0 * kVecBytes;
+    if ((unsigned long long)((tile + 1) * tile_vecs) <= p.body_vecs) {
+      uint32_t r[U][8];
+#pragma unroll
+      for (int u = 0; u < U; ++u) ld_v8(ptr + (size_t)u * B * kVecBytes, r[u]);
+#pragma unroll
+      for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, r[u]);
+    } else {  // the ragged last tile
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (v0 + (unsigned long long)(u * B) < p.body_vecs) {
+          uint32_t r[8];
+          ld_v8(ptr + (size_t)u * B * kVecBytes, r);
+          fold_vec<T>(a, aux, r);
+        }
+      }
+    }
+  }
+  if (blockIdx.x == gridDim.x - 1) {
+    using Elem = typename T::Elem;
+    const int t = threadIdx.x;
+    if (t < p.head) fold_elem<T>(a[0], aux, __ldg((const Elem*)p.in + t));
+    else if (t >= 8 && t - 8 < p.tail)
+      fold_elem<T>(a[0], aux, __ldg((const Elem*)(p.body + p.body_vecs * kVecBytes) + (t - 8)));
+  }
+  const Acc v = thread_result<T>(a, aux);
+  const typename T::Grid g = block_combine<T, BC>(v);
+  grid_combine<T>(g, p);
+}
+
+// Second pass of GC_TWO_PASS and the cross-chunk / cross-rank combine.
+template <int DT, int OP>
+__global__ void __launch_bounds__(1024) k_combine(const void* vals, long long count, void* out, int raw_out) {
+  using T = Tr<DT, OP>;
+  typename T::Grid x = reduce_grid_values<T>((const typename T::Grid*)vals, count);
+  if (threadIdx.x == 0) {
+    if (raw_out) *(typename T::Grid*)out = x;
+    else T::finalize(x, out);
+  }
+}
+
+template <int DT, int OP>
+__global__ void k_init_slots(void* slots, unsigned* ticket) {
+  using T = Tr<DT, OP>;
+  if (threadIdx.x < kMaxSlots) *(typename T::Grid*)((char*)slots + threadIdx.x * kSlotBytes) = T::gident();
+  if (threadIdx.x == 0) *ticket = 0u;
+}
+
+inline KParams make_params(const LaunchDesc& d) {
+  KParams p;
+  p.in = (const char*)d.in;
+  p.body = (const char*)d.body;
+  p.body_vecs = d.body_vecs;
+  p.tiles = d.tiles;
+  p.head = d.head;
+  p.tail = d.tail;
+  p.out = d.out;
+  p.raw_out = d.raw_out;
+  p.gc = d.gc;
+  p.slots = d.slots;
+  p.nslots = d.nslots < 1 ? 1 : d.nslots;
+  p.ticket = d.ticket;
+  p.partials = d.partials;
+  return p;
+}
+
+template <int DT, int OP, int U>
+cudaError_t launch_u(const LaunchDesc& d, const KParams& p, cudaStream_t s) {
+  switch (d.bc) {
+    case BC_SHFL: k_reduce<DT, OP, U, BC_SHFL><<<d.grid, d.block, 0, s>>>(p); break;
+    case BC_ATOMIC_WARP: k_reduce<DT, OP, U, BC_ATOMIC_WARP><<<d.grid, d.block, 0, s>>>(p); break;
+    case BC_ATOMIC_ALL: k_reduce<DT, OP, U, BC_ATOMIC_ALL><<<d.grid, d.block, 0, s>>>(p); break;
+    case BC_TREE: k_reduce<DT, OP, U, BC_TREE><<<d.grid, d.block, 0, s>>>(p); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaPeekAtLastError();
+}
+
+template <int DT, int OP>
+cudaError_t launch_op(const LaunchDesc& d, cudaStream_t s) {
+  const KParams p = make_params(d);
+  cudaError_t e;
+  switch (d.unroll) {
+    case 1: e = launch_u<DT, OP, 1>(d, p, s); break;
+    case 2: e = launch_u<DT, OP, 2>(d, p, s); break;
+    case 4: e = launch_u<DT, OP, 4>(d, p, s); break;
+    case 8: e = launch_u<DT, OP, 8>(d, p, s); break;
+    default: return cudaErrorInvalidValue;
+  }
+  if (e != cudaSuccess || d.gc != GC_TWO_PASS) return e;
+  k_combine<DT, OP><<<1, 1024, 0, s>>>(d.partials, (long long)d.grid, d.out, d.raw_out);
+  return cudaPeekAtLastError();
+}
+
+template <int DT>
+cudaError_t launch_dt(const LaunchDesc& d, cudaStream_t s) {
+  switch (d.op) {
+    case OP_SUM: return launch_op<DT, OP_SUM>(d, s);
+    case OP_MIN: return launch_op<DT, OP_MIN>(d, s);
+    case OP_MAX: return launch_op<DT, OP_MAX>(d, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+template <int DT>
+cudaError_t combine_dt(int op, const void* vals, long long count, void* out, int raw_out, int block, cudaStream_t s) {
+  switch (op) {
+    case OP_SUM: k_combine<DT, OP_SUM><<<1, block, 0, s>>>(vals, count, out, raw_out); break;
+    case OP_MIN: k_combine<DT, OP_MIN><<<1, block, 0, s>>>(vals, count, out, raw_out); break;
+    case OP_MAX: k_combine<DT, OP_MAX><<<1, block, 0, s>>>(vals, count, out, raw_out); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaPeekAtLastError();
+}
+
+template <int DT>
+cudaError_t init_dt(char* slots_base, char* tickets_base, cudaStream_t s) {
+  k_init_slots<DT, OP_SUM><<<1, 32, 0, s>>>(slots_base + (DT * 3 + OP_SUM) * kSlotRegionBytes,
+                                             (unsigned*)(tickets_base + (DT * 3 + OP_SUM) * kSlotBytes));
+  k_init_slots<DT, OP_MIN><<<1, 32, 0, s>>>(slots_base + (DT * 3 + OP_MIN) * kSlotRegionBytes,
+                                             (unsigned*)(tickets_base + (DT * 3 + OP_MIN) * kSlotBytes));
+  k_init_slots<DT, OP_MAX><<<1, 32, 0, s>>>(slots_base + (DT * 3 + OP_MAX) * kSlotRegionBytes,
+                                             (unsigned*)(tickets_base + (DT * 3 + OP_MAX) * kSlotBytes));
+  return cudaPeekAtLastError();
+}
+
+}  // namespace rb

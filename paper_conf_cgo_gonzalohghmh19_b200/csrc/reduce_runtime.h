@@ -1,0 +1,65 @@
+// reduce_runtime.h -- host runtime internals shared by reduce_api.cpp,
+// reduce_host.cpp and reduce_multi.cpp (not part of the ABI).
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <string>
+#include <cuda_runtime.h>
+#include "../../include/reduce.h"
+#include "reduce_internal.h"
+
+namespace rb {
+
+// Per-(device, stream) workspace.  Everything is allocated once (or grown
+// outside graph capture) and reused; the atomic slots reset themselves.
+struct Workspace {
+  int device = -1;
+  cudaStream_t stream = nullptr;
+  char* base = nullptr;        // slots | tickets | scalars
+  char* slots = nullptr;       // kCombos regions of kSlotRegionBytes
+  char* tickets = nullptr;     // kCombos words, kSlotBytes apart
+  char* scalars = nullptr;     // 64 x 64-byte scratch scalars (raw results, gathers)
+  char* partials = nullptr;    // per-block / per-chunk Grid values
+  size_t partials_bytes = 0;
+  // reduce_host staging (lazily created)
+  char* staging = nullptr;     // 2 x staging_bytes
+  size_t staging_bytes = 0;
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_copied[2] = {nullptr, nullptr};
+  cudaEvent_t ev_done[2] = {nullptr, nullptr};
+};
+
+constexpr size_t kScalarBytes = 64;
+constexpr int kNumScalars = 64;
+constexpr long long kMaxPartialBlocks = 1 << 16;  // grid cap for partials-based combines
+
+// Resolved plan of one reduction call (step S0).
+struct Plan {
+  int dtype, op, mode;
+  size_t n;
+  int elem;  // bytes per element
+  LaunchDesc d;
+  reduce_plan_t pub;
+};
+
+void set_error(const std::string& msg);
+int fail(int status, const std::string& msg);
+int cuda_fail(cudaError_t e, const char* what);
+
+// Validate arguments (no CUDA calls) and resolve the launch.  `raw_out`
+// selects the un-finalised Grid value as output.
+int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* opts, int raw_out,
+              Plan* plan);
+
+// Find or create the workspace for (current device, stream) with at least
+// `partials_bytes` of partials.  Returns REDUCE_ERR_NOT_PREPARED when an
+// allocation would be needed during stream capture.
+int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** ws);
+
+// Fill the workspace pointers of plan->d and launch it.
+int launch_plan(Plan* plan, Workspace* ws, void* out, cudaStream_t stream);
+
+int num_sms();
+int default_mode();
+
+}  // namespace rb

@@ -1,0 +1,137 @@
+"""Boundary tests that need no GPU: the C-ABI library loads, exports every
+function include/reduce.h declares, rejects bad arguments before touching
+CUDA, and plans launches (step S0) as DESIGN.md describes."""
+import ctypes
+import os
+import re
+
+import pytest
+
+import paper_conf_cgo_gonzalohghmh19_b200 as rb
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "reduce.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"^\s*(?:const\s+)?(?:int|void|char)\s*\*?\s*(reduce_\w+|reduce)\s*\(", src, flags=re.M)))
+
+
+def test_header_symbols_exported():
+    names = header_functions()
+    assert len(names) >= 17, names
+    assert set(names) == set(rb.ABI_SYMBOLS)
+    L = ctypes.CDLL(rb.LIB_PATH)
+    for name in names:
+        assert hasattr(L, name), name
+
+
+def test_library_is_sm100a_only():
+    out = os.popen(f"cuobjdump --list-elf {rb.LIB_PATH} 2>&1").read()
+    assert "sm_100a" in out
+    assert "sm_90" not in out and "sm_80" not in out
+
+
+def test_status_strings_and_version():
+    assert rb.status_string(0) == "REDUCE_OK"
+    assert rb.status_string(6) == "REDUCE_ERR_NOT_PREPARED"
+    assert rb.status_string(99) == "REDUCE_ERR_UNKNOWN"
+    assert rb.lib.reduce_version() >= 100
+    assert rb.lib.reduce_comm_unique_id_bytes() == 128
+
+
+def _ex(dtype, op, inp, n, out, opts=None):
+    return rb.lib.reduce_ex(dtype, op, ctypes.c_void_p(inp), n, ctypes.c_void_p(out), None,
+                            ctypes.byref(opts) if opts is not None else None)
+
+
+@pytest.mark.parametrize("args,why", [
+    ((3, 0, 4096, 10, 8192), "bad dtype"),
+    ((-1, 0, 4096, 10, 8192), "bad dtype"),
+    ((0, 3, 4096, 10, 8192), "bad op"),
+    ((0, 0, None, 10, 8192), "NULL in with n > 0"),
+    ((0, 0, 4096, 10, None), "NULL out"),
+    ((0, 0, 4098, 10, 8192), "misaligned int32 in"),
+    ((2, 0, 4100, 10, 8192), "misaligned fp64 in"),
+    ((2, 0, 4096, 10, 8196), "misaligned fp64 out"),
+])
+def test_invalid_arguments_rejected_without_cuda(args, why):
+    st = _ex(*args)
+    assert st == 1, (why, st, rb.last_error())
+    assert rb.last_error()
+
+
+@pytest.mark.parametrize("kw", [
+    dict(mode=7), dict(grid_combine=9), dict(block_combine=5), dict(unroll=3),
+    dict(block=48), dict(block=2048), dict(block=1024, unroll=8), dict(grid=-2),
+    dict(mode="deterministic", grid_combine=rb.GC_ATOMIC),
+    dict(mode="deterministic", block_combine=rb.BC_SMEM_ATOMIC_ALL),
+    dict(block=96, block_combine=rb.BC_SMEM_TREE),
+])
+def test_invalid_options_rejected(kw):
+    o = rb.make_opts(**kw)
+    assert _ex(1, 0, 4096, 1000, 8192, o) == 1, rb.last_error()
+
+
+def test_query_plan_partition_and_head_tail():
+    # fp32, pointer 4 bytes past a 32-byte boundary: 7 head elements
+    p = rb.query_plan("float32", "sum", 1000, in_ptr=0x10004)
+    assert p["head"] == 7 and p["tail"] == (1000 - 7) % 8
+    p = rb.query_plan("float64", "sum", 1000, in_ptr=0x10008)
+    assert p["head"] == 3 and p["tail"] == (1000 - 3) % 4
+    p = rb.query_plan("int32", "max", 5, in_ptr=0x10004)
+    assert p["head"] == 5 and p["tail"] == 0
+    p = rb.query_plan("int32", "sum", 0)
+    assert p["grid"] == 1 and p["grid_combine"] == rb.GC_DIRECT
+
+
+def test_query_plan_modes():
+    n = 1 << 28
+    fast = rb.query_plan("float32", "sum", n, mode="fast")
+    det = rb.query_plan("float32", "sum", n, mode="deterministic")
+    assert fast["grid_combine"] == rb.GC_ATOMIC and fast["launches"] == 1
+    assert det["grid_combine"] == rb.GC_TWO_PASS and det["launches"] == 2
+    assert det["grid"] <= 1 << 16
+    # one block per 32 KiB tile at the headline size
+    tile = fast["block"] * fast["unroll"] * 32
+    assert fast["tiles"] == (n * 4) // tile and fast["grid"] == fast["tiles"]
+    small = rb.query_plan("float32", "sum", 1000)
+    assert small["grid"] == 1 and small["grid_combine"] == rb.GC_DIRECT
+
+
+def test_query_plan_chain_bounds():
+    # chain L: per-thread + lane tree + warp + block + grid terms (S5)
+    p = rb.query_plan("float32", "sum", 1 << 28)
+    assert 0 < p["chain"] < 64
+    p = rb.query_plan("float64", "sum", 1 << 26, mode="deterministic")
+    assert p["chain"] < 200
+    assert rb.query_plan("int32", "sum", 1 << 20)["chain"] == 0
+    assert rb.query_plan("float32", "max", 1 << 20)["chain"] == 0
+    va1 = rb.query_plan("float32", "sum", 1 << 20, block_combine=rb.BC_SMEM_ATOMIC_ALL, block=256)
+    assert va1["chain"] >= 256
+
+
+def test_forced_overrides_respected():
+    p = rb.query_plan("float32", "sum", 1 << 24, block=128, unroll=8, grid=300,
+                      grid_combine=rb.GC_LAST_BLOCK, block_combine=rb.BC_SMEM_TREE)
+    assert (p["block"], p["unroll"], p["grid"], p["grid_combine"], p["block_combine"]) == (128, 8, 300, 3, 3)
+    assert p["tiles"] == ((1 << 24) // 8 + 128 * 8 - 1) // (128 * 8)
+
+
+def test_mode_default_roundtrip():
+    old = rb.get_mode()
+    rb.set_mode("deterministic")
+    assert rb.get_mode() == 1
+    rb.set_mode(42)  # ignored
+    assert rb.get_mode() == 1
+    rb.set_mode(old)
+
+
+def test_shard_range_partitions_exactly():
+    for n in (0, 1, 7, 1000, 2 ** 31):
+        for k in (1, 2, 3, 8):
+            ranges = [rb.shard_range(n, k, r) for r in range(k)]
+            assert ranges[0][0] == 0 and ranges[-1][1] == n
+            assert all(a[1] == b[0] for a, b in zip(ranges, ranges[1:]))
+            assert max(h - l for l, h in ranges) - min(h - l for l, h in ranges) <= 1

@@ -1,0 +1,348 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element
+by element on the same seeded inputs.  Integer and min/max results must be
+bit-exact; fp sums must pass gate G1 (north star) and the tight gate G2
+(chain-length bound of the variant that ran).  Pins P1-P11 of DESIGN.md."""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from tests._util import check, gpu_reduce_many, to_device, NP
+
+pytestmark = pytest.mark.gpu
+
+DTYPES = ["int32", "float32", "float64"]
+OPS = ["sum", "min", "max"]
+
+
+def _rb():
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    return rb
+
+
+def _dist(dtype):
+    return "int_full" if dtype == "int32" else "uniform_pm1"
+
+
+# ------------------------------------------------------------- P6 / P7 paper examples
+@pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("variant", [dict(), dict(block=32, grid_combine=0), dict(block=256, unroll=1, grid_combine=1),
+                                     dict(block=32, unroll=1, grid_combine=2), dict(block=64, grid_combine=3)])
+def test_p6_fig1c_example_and_p7_fig2(dtype, variant):
+    for xs, want in ((list(range(16)), 120), (list(range(1, 35)), 595)):
+        x = np.array(xs, NP[dtype])
+        for off in range(4):
+            t = to_device(x, off)
+            (got,), (plan,) = gpu_reduce_many([(t, "sum")], **variant)
+            assert got[0] == want
+            (mn,), _ = gpu_reduce_many([(t, "min")], **variant)
+            (mx,), _ = gpu_reduce_many([(t, "max")], **variant)
+            assert mn[0] == xs[0] and mx[0] == xs[-1]
+
+
+# ------------------------------------------------------------- P8 brute force, small n
+SMALL_N = sorted(set(list(range(0, 130)) + [255, 256, 257, 511, 512, 513, 1023, 1024, 1025, 2047, 2048, 2049,
+                                             4095, 4096, 4097, 8191, 8193, 16385, 65535, 65536, 65537]))
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("mode", ["fast", "deterministic"])
+def test_p8_small_sizes_all_offsets(dtype, mode):
+    cases, xs = [], []
+    for k, n in enumerate(SMALL_N):
+        x = synth.make(dtype, n, _dist(dtype), 1000 + k)
+        for off in range(8 if dtype != "float64" else 4):
+            t = to_device(x, off)
+            for op in OPS:
+                cases.append((t, op))
+                xs.append((x, op))
+    got, plans = gpu_reduce_many(cases, mode=mode)
+    for (x, op), g, p in zip(xs, got, plans):
+        check(x, op, g, p)
+
+
+# ------------------------------------------------------------- P1 / P2 / P3 closed forms on the GPU
+@pytest.mark.parametrize("n", [1000, 4097, (1 << 20) + 3, (1 << 24)])
+def test_p1_ones_and_p2_iota(n):
+    rb = _rb()
+    import torch
+    for dtype in DTYPES:
+        t = torch.ones(n, dtype=getattr(torch, dtype), device="cuda")
+        assert rb.reduce(t, "sum").item() == n
+        it = torch.arange(n, dtype=torch.int64, device="cuda").to(getattr(torch, dtype))
+        r = rb.reduce(it, "sum").item()
+        exact = n * (n - 1) // 2
+        if dtype == "int32":
+            exact = ((exact + 2 ** 31) % 2 ** 32) - 2 ** 31
+            assert r == exact
+        elif dtype == "float64":
+            assert r == exact  # exact for n <= 2^27
+        assert rb.reduce(it, "min").item() == 0 and rb.reduce(it, "max").item() == n - 1
+
+
+@pytest.mark.parametrize("dtype,bound,n", [("float32", 1 << 7, (1 << 17) - 3), ("float64", 1 << 20, (1 << 22) + 5)])
+def test_p3_integer_valued_sums_bit_exact(dtype, bound, n):
+    x = synth.make(dtype, n, "intvalued", 77, bound=bound)
+    exact = int(x.astype(np.int64).sum())
+    for mode in ("fast", "deterministic"):
+        (g,), _ = gpu_reduce_many([(to_device(x, 1), "sum")], mode=mode)
+        assert float(g[0]) == exact
+
+
+# ------------------------------------------------------------- sweep 2^k-1, 2^k, 2^k+1
+@pytest.mark.parametrize("dtype", DTYPES)
+def test_size_sweep(dtype):
+    cases, xs = [], []
+    for k in range(10, 25, 2):
+        for d in (-1, 0, 1):
+            n = (1 << k) + d
+            x = synth.make(dtype, n, "uniform01" if dtype != "int32" else "int_full", 50 + k)
+            t = to_device(x, (k + d) % 3)
+            for op in OPS:
+                cases.append((t, op))
+                xs.append((x, op))
+    for mode in ("fast", "deterministic"):
+        got, plans = gpu_reduce_many(cases, mode=mode)
+        for (x, op), g, p in zip(xs, got, plans):
+            check(x, op, g, p)
+
+
+# ------------------------------------------------------------- every variant on the same inputs
+VARIANTS = []
+for bc in range(4):
+    for gc in range(4):
+        for blk, u in ((32, 1), (128, 2), (256, 4), (512, 8), (1024, 1)):
+            VARIANTS.append(dict(block_combine=bc, grid_combine=gc, block=blk, unroll=u))
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+def test_every_variant(dtype):
+    n = (1 << 18) + 13
+    x = synth.make(dtype, n, _dist(dtype), 4242)
+    x[[0, n // 2, n - 1]] = x[[n - 1, 0, n // 2]]
+    t = to_device(x, 3)
+    for v in VARIANTS:
+        if dtype == "float64" and v["block"] > 512 and v["unroll"] >= 2:
+            continue
+        got, plans = gpu_reduce_many([(t, op) for op in OPS], **v)
+        for op, g, p in zip(OPS, got, plans):
+            check(x, op, g, p)
+
+
+@pytest.mark.parametrize("grid", [1, 7, 148, 1000])
+def test_persistent_grids(grid):
+    """Blocks looping over tiles (grid < tiles): the Catanzaro-style persistent
+    partition must cover every tile exactly once."""
+    for dtype in DTYPES:
+        x = synth.make(dtype, (1 << 20) + 5, _dist(dtype), grid)
+        t = to_device(x, 1)
+        for gc in (1, 2, 3):
+            got, plans = gpu_reduce_many([(t, op) for op in OPS], grid=grid, grid_combine=gc)
+            for op, g, p in zip(OPS, got, plans):
+                check(x, op, g, p)
+
+
+# ------------------------------------------------------------- P5 permutations: extremes everywhere
+@pytest.mark.parametrize("dtype", DTYPES)
+def test_p5_permutation_extremes_in_head_tail_and_boundaries(dtype):
+    rb = _rb()
+    n = 100003
+    base = synth.make(dtype, n, "perm", 9)
+    plan = rb.query_plan(dtype, "min", n, in_ptr=0x1004)
+    tile = plan["block"] * plan["unroll"] * (8 if dtype != "float64" else 4)
+    positions = [0, 1, 2, n - 1, n - 2, tile - 1, tile, tile + 1, n // 2]
+    for pos in positions:
+        x = base.copy()
+        i0, i1 = int(np.where(x == 0)[0][0]), int(np.where(x == n - 1)[0][0])
+        x[[i0, pos]] = x[[pos, i0]]
+        got, plans = gpu_reduce_many([(to_device(x, 1), "min"), (to_device(x, 1), "max")])
+        assert got[0][0] == 0 and got[1][0] == n - 1
+
+
+# ------------------------------------------------------------- P11 special values
+@pytest.mark.parametrize("dtype", ["float32", "float64"])
+@pytest.mark.parametrize("variant", [dict(), dict(mode="deterministic"), dict(block=32, grid_combine=0),
+                                     dict(block_combine=1), dict(block_combine=2), dict(block_combine=3),
+                                     dict(grid_combine=3)])
+def test_p11_special_values(dtype, variant):
+    dt = NP[dtype]
+    n = 50000
+    sp = lambda k: synth.special_f(dtype, k)
+    cases = []
+    for where in (0, 7, 24999, n - 1):
+        for kind in ("nan", "neg_nan", "inf", "ninf"):
+            x = synth.make(dtype, n, "uniform_pm1", 5)
+            x[where] = sp(kind)
+            cases.append(x)
+        x = synth.make(dtype, n, "uniform_pm1", 6)
+        x[where] = sp("inf"); x[(where + 11) % n] = sp("ninf")
+        cases.append(x)
+    # signed zeros
+    z = np.zeros(n, dt); z[::3] = -0.0
+    cases.append(z)
+    cases.append(np.full(n, -0.0, dt))
+    cases.append(np.full(n, sp("nan"), dt))
+    cases.append(np.array([-0.0, 0.0] * 20, dt))
+    for x in cases:
+        t = to_device(x, 2)
+        got, plans = gpu_reduce_many([(t, op) for op in OPS], **variant)
+        for op, g, p in zip(OPS, got, plans):
+            check(x, op, g, p)
+
+
+def test_p11_empty_and_single():
+    rb = _rb()
+    import torch
+    for dtype in DTYPES:
+        e = torch.empty(0, dtype=getattr(torch, dtype), device="cuda")
+        for op in OPS:
+            got = rb.reduce(e, op).cpu().numpy()
+            check(np.zeros(0, NP[dtype]), op, got)
+        one = torch.tensor([-3], dtype=getattr(torch, dtype), device="cuda")
+        for op in OPS:
+            assert rb.reduce(one, op).item() == -3
+
+
+# ------------------------------------------------------------- P9 determinism / invariants
+@pytest.mark.parametrize("dtype", ["float32", "float64"])
+@pytest.mark.parametrize("gc", [2, 3])
+def test_p9_deterministic_mode_bitwise_repeatable(dtype, gc):
+    import torch
+    rb = _rb()
+    x = synth.make(dtype, (1 << 22) + 77, "uniform_pm1", 31)
+    t = to_device(x, 1)
+    outs = torch.empty(100, dtype=t.dtype, device="cuda")
+    for i in range(100):
+        rb.reduce(t, "sum", out=outs[i:i + 1], mode="deterministic", grid_combine=gc)
+    o = outs.cpu().numpy()
+    assert len(set(o.view(np.uint32 if dtype == "float32" else np.uint64).tolist())) == 1
+    check(x, "sum", o[:1], rb.query_plan(dtype, "sum", x.size, in_ptr=t.data_ptr(), mode="deterministic", grid_combine=gc))
+
+
+def test_p9_int_results_permutation_invariant():
+    rb = _rb()
+    x = synth.make("int32", (1 << 20) + 9, "int_full", 8)
+    rng = np.random.Generator(np.random.PCG64(1))
+    y = rng.permutation(x)
+    got, _ = gpu_reduce_many([(to_device(x), op) for op in OPS] + [(to_device(y, 5), op) for op in OPS])
+    assert [int(g[0]) for g in got[:3]] == [int(g[0]) for g in got[3:]]
+
+
+# ------------------------------------------------------------- full sizes (bench launch config)
+def test_full_size_fp32_sum_2p28_bench_config():
+    """BASELINE configs[1] at its largest point (2^28 fp32) in the exact launch
+    configuration bench.py times (default dispatch, fast mode), whole-array
+    oracle comparison with G1 and G2; plus deterministic mode."""
+    rb = _rb()
+    n = 1 << 28
+    x = synth.make("float32", n, "uniform01", synth.seed_for(1, n))
+    t = to_device(x)
+    for mode in ("fast", "deterministic"):
+        (g,), (p,) = gpu_reduce_many([(t, "sum")], mode=mode)
+        check(x, "sum", g, p)
+    xm = synth.make("float32", n, "uniform_pm1", synth.seed_for(1, n) + 1)
+    tm = to_device(xm)
+    got, plans = gpu_reduce_many([(tm, op) for op in OPS])
+    for op, g, p in zip(OPS, got, plans):
+        check(xm, op, g, p)
+
+
+def test_full_size_int32_and_fp64_2p26_config3():
+    """BASELINE configs[2]: int32 / fp64 sum, min, max at 64M elements, atomic
+    vs deterministic-tree variants; int32 full range with INT32_MIN/MAX planted
+    (one in the tail), fp64 integer-valued (exact, P3) with +-2.0 planted."""
+    n = 1 << 26
+    xi = synth.make("int32", n, "int_full", synth.seed_for(2, n))
+    synth.plant(xi, [np.iinfo(np.int32).min, np.iinfo(np.int32).max], seed=3, positions=[12345, n - 3])
+    xd = synth.make("float64", n, "intvalued", synth.seed_for(2, n) + 1, bound=1 << 20)
+    synth.plant(xd, [2.0 ** 21, -(2.0 ** 21)], seed=4, positions=[n - 1, 777])
+    for x in (xi, xd):
+        t = to_device(x, 1)
+        for mode in ("fast", "deterministic"):
+            got, plans = gpu_reduce_many([(t, op) for op in OPS], mode=mode)
+            for op, g, p in zip(OPS, got, plans):
+                check(x, op, g, p)
+            if x.dtype == np.float64:
+                assert float(got[0][0]) == float(int(x.astype(np.int64).sum()))  # P3 bit-exact
+
+
+def test_full_size_2p31_elements_64bit_indexing():
+    """BASELINE configs[4] at k=1: 2^31 fp32 (8 GiB) on one GPU.  Property pins
+    at full size: sum of ones is exactly 2^31 (every 8192-element tile sum is
+    exact in fp32 and blocks combine exactly in fp64), int32 ones wrap to
+    INT32_MIN, and a planted extreme at the very end is found."""
+    import torch
+    rb = _rb()
+    n = 1 << 31
+    t = torch.ones(n, dtype=torch.float32, device="cuda")
+    assert rb.reduce(t, "sum").item() == float(n)
+    assert rb.reduce(t, "sum", mode="deterministic").item() == float(n)
+    t[n - 1] = 5.0
+    t[3] = -7.0
+    assert rb.reduce(t, "max").item() == 5.0 and rb.reduce(t, "min").item() == -7.0
+    del t
+    torch.cuda.empty_cache()
+    ti = torch.ones(n, dtype=torch.int32, device="cuda")
+    assert rb.reduce(ti, "sum").item() == -(2 ** 31)
+    del ti
+    torch.cuda.empty_cache()
+
+
+# ------------------------------------------------------------- workspace / graphs / streams
+def test_graph_capture_after_prepare():
+    import torch
+    rb = _rb()
+    x = synth.make("float32", (1 << 22) + 3, "uniform01", 2)
+    t = to_device(x, 1)
+    s = torch.cuda.Stream()
+    out = torch.empty(1, dtype=torch.float32, device="cuda")
+    with torch.cuda.stream(s):
+        # not prepared: capture must fail cleanly with NOT_PREPARED
+        g = torch.cuda.CUDAGraph()
+        with pytest.raises(Exception):
+            with torch.cuda.graph(g, stream=s):
+                rb.reduce(t, "sum", out=out, mode="deterministic")
+    s2 = torch.cuda.Stream()
+    rb.prepare(s2, t.numel())
+    g2 = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g2, stream=s2):
+        rb.reduce(t, "sum", out=out, stream=s2)
+    for _ in range(3):
+        out.zero_()
+        g2.replay()
+        torch.cuda.synchronize()
+        check(x, "sum", out.cpu().numpy(), rb.query_plan("float32", "sum", t.numel(), in_ptr=t.data_ptr()))
+
+
+def test_concurrent_streams_private_workspaces():
+    import torch
+    rb = _rb()
+    xs = [synth.make("float64", (1 << 20) + i, "uniform01", i) for i in range(4)]
+    ts = [to_device(x, i) for i, x in enumerate(xs)]
+    streams = [torch.cuda.Stream() for _ in xs]
+    outs = [torch.empty(1, dtype=torch.float64, device="cuda") for _ in xs]
+    for _ in range(20):
+        for t, s, o in zip(ts, streams, outs):
+            rb.reduce(t, "sum", out=o, stream=s)
+    torch.cuda.synchronize()
+    for x, o, t in zip(xs, outs, ts):
+        check(x, "sum", o.cpu().numpy(), rb.query_plan("float64", "sum", t.numel(), in_ptr=t.data_ptr()))
+
+
+# ------------------------------------------------------------- end-to-end host entry
+@pytest.mark.parametrize("dtype", DTYPES)
+def test_reduce_host_chunks(dtype):
+    import torch
+    rb = _rb()
+    n = (1 << 24) + 1001  # several 32 MiB chunks for fp64, 2+ for 4-byte types
+    x = synth.make(dtype, n, _dist(dtype), 12)
+    pinned = torch.from_numpy(x).pin_memory()
+    for op in OPS:
+        for src in (pinned, x):
+            g = rb.reduce_host(src, op)
+            check(x, op, np.array([g], NP[dtype]), None, gates=("g1",))
+    for op in OPS:
+        g = rb.reduce_host(x[:0], op)
+        check(x[:0], op, np.array([g], NP[dtype]))
