@@ -1,0 +1,387 @@
+#!/usr/bin/env python
+"""Bench harness: device-wide reduction throughput on B200 (BASELINE.json metric
+"reduction GB/s & fraction of HBM peak vs array size, 1/2/4/8 B200").
+
+One step = one pass of the whole hot path (steps S0-S6, plus S7 for N>1) over
+one batch of synthetic input already resident in HBM:
+  N = 1 : reduce(fp32, sum) of n = 2^28 elements (1 GiB) -- the largest point
+          of BASELINE configs[1] ("fp32 sum size sweep 1K-256M"), the headline.
+  N > 1 : reduce_multi(fp32, sum): every rank reduces its own 2^28-element
+          shard and the per-rank scalars are combined by one NCCL all-reduce
+          (configs[4]: at N = 8 this is the 8 GiB array).  Weak scaling.
+The 1 GiB per-GPU input is larger than the 126 MB L2, so consecutive steps
+read from HBM without an explicit flush.
+
+Extra keys: roofline (dominant kernel vs the measured HBM peak), cpu_baseline
+(the oracle on the host cores), e2e (the same metric through the C-ABI host
+entry with H2D/D2H copies in the timed region), clocks (NVML, sampled during
+the timed region), gpu_launches, and `sweep` (fp32 sum GB/s vs size, each
+call after an L2 flush).
+
+`--impl reference` times the CPU oracle (this tier's reference arm) on the
+same config.  Launch: python bench.py --gpus N --steps K --warmup W
+(N > 1 under torch.distributed.run, one rank per GPU).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+N_PER_GPU = 1 << 28
+METRIC = "reduction GB/s & fraction of HBM peak vs array size, 1/2/4/8 B200"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=N_PER_GPU, help="elements per GPU")
+    ap.add_argument("--mode", default="fast", choices=["fast", "deterministic"])
+    ap.add_argument("--no-sweep", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic():
+    """dram bytes per launch of the dominant kernel from the committed ncu capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_summary.json")) as f:
+            s = json.load(f)
+        return s.get("dram_bytes_per_launch"), s
+    except Exception:
+        return None, None
+
+
+class ClockSampler:
+    """NVML clocks + throttle reasons sampled in a thread during the timed region."""
+    REASONS = {
+        "sw_power_cap": 0x4, "hw_slowdown": 0x8, "sync_boost": 0x10, "sw_thermal_slowdown": 0x20,
+        "hw_thermal_slowdown": 0x40, "hw_power_brake_slowdown": 0x80, "applications_clocks_setting": 0x2,
+    }
+
+    def __init__(self, index: int):
+        self.samples, self.reasons, self.ok = [], set(), False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # no NVML: report it, do not fake
+            self.err = repr(e)
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for k, bit in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.ok:
+            self._stop.set()
+            self.t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "error": getattr(self, "err", "")}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def host_info():
+    model = ""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return model, len(os.sched_getaffinity(0))
+
+
+# --------------------------------------------------------------- reference arm
+def run_reference(args, rank, world):
+    """This tier's reference arm: the CPU oracle, as it stands, on the host cores."""
+    if rank != 0:
+        return
+    import numpy as np
+    import oracle
+    import synth
+    n = args.n
+    # bounded sample of the workload so (W + K) steps finish in about a minute
+    probe = synth.make("float32", 1 << 22, "uniform01", 1)
+    t0 = time.perf_counter(); oracle.reduce(probe, "sum"); t1 = time.perf_counter()
+    rate = (1 << 22) / max(t1 - t0, 1e-6)
+    budget_s = 60.0
+    sample_n = int(min(n, max(1 << 20, rate * budget_s / max(1, args.steps + args.warmup))))
+    sample_n -= sample_n % 8
+    x = synth.make("float32", sample_n, "uniform01", synth.seed_for(1, n))
+    for _ in range(args.warmup):
+        oracle.reduce(x, "sum")
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.reduce(x, "sum")
+    dt = (time.perf_counter() - t0) / args.steps
+    gbs = sample_n * 4 / dt / 1e9
+    model, cores = host_info()
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(gbs, 4), "unit": "GB/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 4),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic", "config": workload_config(args, world, None),
+        "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                         "sample": f"first {sample_n} elements of the seeded 2^28 fp32 U[0,1) workload per step "
+                                   f"(Neumaier sum in double, oracle/oracle.c), host {model}"},
+        "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def workload_config(args, world, plan):
+    cfg = {"workload": f"fp32 sum of {args.n} (2^{args.n.bit_length() - 1}) elements per GPU"
+                       + (" -- BASELINE configs[1] largest point" if world == 1 else
+                          f" -- BASELINE configs[4] sharded sum, {world} GPUs, NCCL all-reduce of partials"),
+           "n_per_gpu": args.n, "total_bytes": args.n * 4 * world, "op": "sum", "mode": args.mode,
+           "parallelism": f"shard{world}" if world > 1 else "single-gpu",
+           "l2": "inputs (4 B x n per GPU) larger than the 126 MB L2 between steps; no flush needed",
+           "distribution": "U[0,1) fp32, numpy PCG64 seed 2019+1000*1+log2(n)+rank"}
+    if plan is not None:
+        cfg["variant"] = plan
+    return cfg
+
+
+# --------------------------------------------------------------- our arm
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import synth
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    n = args.n
+    x_host = synth.make("float32", n, "uniform01", synth.seed_for(1, n, rank))
+    x = torch.from_numpy(x_host).to(dev)
+    out = torch.empty(1, dtype=torch.float32, device=dev)
+    stream = torch.cuda.Stream(dev)
+    comm = rb.Comm() if world > 1 else None
+    plan = rb.query_plan("float32", "sum", n, in_ptr=x.data_ptr(), mode=args.mode)
+    rb.prepare(stream, n)
+
+    def step():
+        if comm is None:
+            rb.reduce(x, "sum", out=out, stream=stream, mode=args.mode)
+        else:
+            rb.reduce_multi(x, "sum", comm, out=out, stream=stream, mode=args.mode)
+
+    def sync_all():
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+
+    with torch.cuda.stream(stream):
+        for _ in range(max(3, args.warmup)):
+            step()
+    sync_all()
+    # ---- timed region: K steps between two events on the launch stream
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clocks = ClockSampler(local)
+    with clocks:
+        e0.record(stream)
+        with torch.cuda.stream(stream):
+            for _ in range(args.steps):
+                step()
+        e1.record(stream)
+        e1.synchronize()
+    sync_all()
+    ms = e0.elapsed_time(e1) / args.steps
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = world * n * 4 / (ms * 1e-3) / 1e9
+
+    # ---- dominant kernel alone: per-launch events on its stream
+    kern_ms = []
+    with torch.cuda.stream(stream):
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(50)]
+        for a, b in evs:
+            a.record(stream)
+            rb.reduce(x, "sum", out=out, stream=stream, mode=args.mode)
+            b.record(stream)
+    torch.cuda.synchronize(dev)
+    kern_ms = [a.elapsed_time(b) for a, b in evs]
+    kavg = statistics.mean(kern_ms)
+    peak, peak_src = measured_peaks()
+    achieved = n * 4 / (kavg * 1e-3) / 1e9
+    traffic, ncu_s = ncu_traffic()
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "kernel": "rb::k_reduce<f32,sum,U,Vs> (+ grid combine epilogue)",
+                "algorithmic_bytes_per_launch": n * 4, "avg_launch_ms": round(kavg, 5),
+                "peak_source": peak_src, "frac_of_nominal_8TBps": round(achieved / 8000.0, 4)}
+    # kernel share of the step (compare with the committed ncu launch list)
+    roofline["kernel_share_of_step"] = round(min(1.0, kavg / ms), 4)
+
+    # ---- e2e through the C-ABI host entry (H2D + reduce + D2H in the timed region)
+    e2e = None
+    if not args.no_e2e:
+        pinned = torch.from_numpy(x_host).pin_memory()
+        k_e2e = max(3, min(args.steps, 20))
+        if comm is None:
+            rb.reduce_host(pinned, "sum", stream=stream, mode=args.mode)
+            sync_all()
+            t0 = time.perf_counter()
+            for _ in range(k_e2e):
+                rb.reduce_host(pinned, "sum", stream=stream, mode=args.mode)
+            dt = (time.perf_counter() - t0) / k_e2e
+        else:
+            xd = torch.empty_like(x)
+            sync_all()
+            t0 = time.perf_counter()
+            with torch.cuda.stream(stream):
+                for _ in range(k_e2e):
+                    xd.copy_(pinned, non_blocking=True)
+                    rb.reduce_multi(xd, "sum", comm, out=out, stream=stream, mode=args.mode)
+                    out.item()
+            dt = (time.perf_counter() - t0) / k_e2e
+            t = torch.tensor([dt], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dt = float(t.item())
+        e2e = {"value": round(world * n * 4 / dt / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": n * 4,
+               "d2h_bytes_per_step": 4, "ms_per_step": round(dt * 1e3, 3),
+               "path": "reduce_host (C ABI, pinned host buffer, chunked H2D overlapped with the chunk reductions)"
+               if comm is None else "pinned H2D copy + reduce_multi + D2H of the result"}
+
+    # ---- size sweep (rank 0 only, N = 1): each call after an L2 flush
+    sweep = None
+    if not args.no_sweep and world == 1:
+        sweep = []
+        flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)  # 256 MB > L2
+        xs = x  # sizes are prefixes of the resident 1 GiB input
+        for k in range(10, 29, 2):
+            m = 1 << k
+            sub = xs[:m]
+            p = rb.query_plan("float32", "sum", m, in_ptr=sub.data_ptr(), mode=args.mode)
+            times = []
+            with torch.cuda.stream(stream):
+                for _ in range(3):
+                    rb.reduce(sub, "sum", out=out, stream=stream, mode=args.mode)
+                for _ in range(15):
+                    flush.fill_(1.0)
+                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record(stream)
+                    rb.reduce(sub, "sum", out=out, stream=stream, mode=args.mode)
+                    b.record(stream)
+                    times.append((a, b))
+                torch.cuda.synchronize(dev)
+                cold = statistics.median([a.elapsed_time(b) for a, b in times])
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                for _ in range(50):
+                    rb.reduce(sub, "sum", out=out, stream=stream, mode=args.mode)
+                b.record(stream)
+                torch.cuda.synchronize(dev)
+                warm = a.elapsed_time(b) / 50
+            sweep.append({"n": m, "cold_us": round(cold * 1e3, 2), "cold_GBps": round(m * 4 / (cold * 1e-3) / 1e9, 1),
+                          "cold_frac_of_peak": round(m * 4 / (cold * 1e-3) / 1e9 / peak, 4),
+                          "warm_b2b_us": round(warm * 1e3, 2),
+                          "warm_GBps": round(m * 4 / (warm * 1e-3) / 1e9, 1),
+                          "variant": f"g{p['grid']}x{p['block']}u{p['unroll']} gc{p['grid_combine']}"})
+        del flush
+
+    # ---- CPU baseline: the oracle on the host cores (rank 0, N = 1)
+    cpu = None
+    if not args.no_cpu and world == 1 and rank == 0:
+        import oracle
+        model, ncores = host_info()
+        reps = 2
+        oracle.reduce(x_host[: 1 << 20], "sum")
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            oracle.reduce(x_host, "sum")
+        dt = (time.perf_counter() - t0) / reps
+        cpu = {"value": round(n * 4 / dt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+               "sample": f"the full 2^28-element fp32 workload, {reps} repetitions (Neumaier in double, "
+                         f"single thread) on {model} ({ncores} usable cores)"}
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            oracle.omp_sum_f32(x_host)
+        dto = (time.perf_counter() - t0) / reps
+        cpu_omp = {"value": round(n * 4 / dto / 1e9, 3), "unit": "GB/s", "cores": oracle.omp_threads(),
+                   "kind": "paper-style OpenMP reduce pragma (P:L469), context only"}
+
+    if rank == 0:
+        launches_per_step = plan["launches"] + (0 if comm is None else 1)
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic", "config": workload_config(args, world, plan),
+            "elements_per_s": round(world * n / (ms * 1e-3), 1),
+            "frac_of_hbm_peak": round(value / world / peak, 4),
+            "roofline": roofline, "e2e": e2e, "clocks": clocks.summary(),
+            "gpu_launches": args.steps * launches_per_step,
+        }
+        if cpu is not None:
+            line["cpu_baseline"] = cpu
+            line["cpu_openmp"] = cpu_omp
+        if sweep is not None:
+            line["sweep"] = sweep
+        if ncu_s is not None:
+            line["ncu"] = {k: ncu_s[k] for k in ("source", "dram_pct_of_peak", "duration_us") if k in ncu_s}
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        torch.cuda.synchronize(dev)
+        comm.destroy()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -150,7 +150,7 @@ def test_p5_permutation_extremes_in_head_tail_and_boundaries(dtype):
     rb = _rb()
     n = 100003
     base = synth.make(dtype, n, "perm", 9)
-    plan = rb.query_plan(dtype, "min", n, in_ptr=0x1004)
+    plan = rb.query_plan(dtype, "min", n, in_ptr=0x1008)
     tile = plan["block"] * plan["unroll"] * (8 if dtype != "float64" else 4)
     positions = [0, 1, 2, n - 1, n - 2, tile - 1, tile, tile + 1, n // 2]
     for pos in positions:
