@@ -209,21 +209,34 @@ def reduce_host(x, op="sum", stream=None, **opt_kw):
 
 
 # ------------------------------------------------------------- sharded mode
+def broadcast_unique_id(group=None) -> bytes:
+    """Rank 0 of `group` creates an NCCL unique id (reduce_comm_get_unique_id);
+    it is broadcast to every rank through the torch process group (any backend)."""
+    import torch.distributed as dist
+    rank = dist.get_rank(group)
+    nbytes = lib.reduce_comm_unique_id_bytes()
+    obj = [None]
+    if rank == 0:
+        uid = (ctypes.c_char * nbytes)()
+        _check(lib.reduce_comm_get_unique_id(ctypes.cast(uid, ctypes.c_void_p)), "reduce_comm_get_unique_id")
+        obj = [bytes(uid)]
+    src = dist.get_global_rank(group, 0) if group is not None else 0
+    dist.broadcast_object_list(obj, src=src, group=group)
+    if not isinstance(obj[0], bytes) or len(obj[0]) != nbytes:
+        raise RuntimeError("bad NCCL unique id received")
+    return obj[0]
+
+
 class Comm:
     """An NCCL communicator owned by the library (reduce_comm_init), bootstrapped
-    over a torch.distributed process group (the unique id travels through it)."""
+    over a torch.distributed process group (the unique id travels through it).
+    Call after torch.cuda.set_device(local_rank)."""
 
     def __init__(self, group=None):
         import torch.distributed as dist
         rank, world = dist.get_rank(group), dist.get_world_size(group)
-        nbytes = lib.reduce_comm_unique_id_bytes()
-        uid = (ctypes.c_char * nbytes)()
-        if rank == 0:
-            _check(lib.reduce_comm_get_unique_id(ctypes.cast(uid, ctypes.c_void_p)), "reduce_comm_get_unique_id")
-        obj = [bytes(uid) if rank == 0 else None]
-        src = dist.get_global_rank(group, 0) if group is not None else 0
-        dist.broadcast_object_list(obj, src=src, group=group)
-        uid = (ctypes.c_char * nbytes).from_buffer_copy(obj[0])
+        uid_bytes = broadcast_unique_id(group)
+        uid = (ctypes.c_char * len(uid_bytes)).from_buffer_copy(uid_bytes)
         handle = ctypes.c_void_p()
         _check(lib.reduce_comm_init(ctypes.byref(handle), ctypes.cast(uid, ctypes.c_void_p), world, rank),
                "reduce_comm_init")

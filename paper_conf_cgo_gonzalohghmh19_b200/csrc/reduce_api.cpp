@@ -15,7 +15,7 @@
 namespace rb {
 
 struct DispatchEntry {
-  int dtype, op, mode, max_log2_bytes, block, unroll, grid_kind, bc;
+  int dtype, op, mode, max_log2_bytes, block, unroll, gc, bc, grid_cap;
 };
 #include "dispatch_table.inc"
 
@@ -96,8 +96,13 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   int bc = o.block_combine >= 0 ? o.block_combine : e->bc;
   int gc;
   if (o.grid_combine >= 0) gc = o.grid_combine;
-  else if (e->grid_kind == 0) gc = REDUCE_GC_DIRECT;
+  else if (e->gc >= 0) gc = e->gc;
   else gc = mode == REDUCE_MODE_DETERMINISTIC ? REDUCE_GC_TWO_PASS : REDUCE_GC_ATOMIC;
+  if (o.grid_combine < 0 && mode == REDUCE_MODE_DETERMINISTIC && gc == REDUCE_GC_ATOMIC) gc = REDUCE_GC_TWO_PASS;
+  if (o.block_combine < 0 && mode == REDUCE_MODE_DETERMINISTIC &&
+      (bc == REDUCE_BC_SMEM_ATOMIC_WARP || bc == REDUCE_BC_SMEM_ATOMIC_ALL))
+    bc = REDUCE_BC_SHFL;
+  const int grid_cap = o.grid > 0 ? o.grid : e->grid_cap;
   if (block > max_block_threads(dtype, op, unroll))
     return fail(REDUCE_ERR_INVALID_ARG, "block too large for this (dtype, op, unroll): max " +
                                             std::to_string(max_block_threads(dtype, op, unroll)));
@@ -123,7 +128,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
     grid = 1;
   } else {
     grid = tiles > 0 ? tiles : 1;
-    if (o.grid > 0 && o.grid < grid) grid = o.grid;
+    if (grid_cap > 0 && grid_cap < grid) grid = grid_cap;
     if ((gc == REDUCE_GC_TWO_PASS || gc == REDUCE_GC_LAST_BLOCK) && grid > kMaxPartialBlocks) grid = kMaxPartialBlocks;
     if (grid > 0x7FFFFFFFll) grid = 0x7FFFFFFFll;
   }

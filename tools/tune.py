@@ -1,0 +1,173 @@
+#!/usr/bin/env python
+"""Autotuner -> csrc/dispatch_table.inc (step S0's table).
+
+The paper tunes every version with every tunable at the largest size with "a
+simple script" and observes that the best version changes with array
+size and GPU.  This does the same on the B200, per size: every
+candidate (block combine x grid combine x block x unroll x grid cap) is timed
+as device time per call (CUDA graph of R calls over cold input regions, see
+tools/cudatiming.py), and the fastest candidate per (dtype, op, mode, log2
+bytes) becomes a table row.  Results are also written as JSON for the record.
+
+Usage (on the GPU box):
+  python tools/tune.py --dtypes float32 --ops sum --modes fast --out gpurun_out/tune.json
+  python tools/tune.py --emit gpurun_out/tune.json [more.json ...]  # write dispatch_table.inc
+"""
+from __future__ import annotations
+
+import argparse
+import itertools
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tools"))
+
+ELEM = {"int32": 4, "float32": 4, "float64": 8}
+DT = {"int32": 0, "float32": 1, "float64": 2}
+OPC = {"sum": 0, "min": 1, "max": 2}
+MODE = {"fast": 0, "deterministic": 1}
+MAXBLK = lambda dt, op, u: 512 if (u >= 8 or (dt == "float64" and op != "sum" and u >= 2)) else 1024
+
+
+def candidates(dtype, op, mode, lb):
+    gcs = [1, 2, 3] if mode == "fast" else [2, 3]
+    out = []
+    if lb <= 18:
+        for blk, u in itertools.product((32, 128, 256, 512, 1024), (1, 2, 4)):
+            out.append(dict(block=blk, unroll=u, grid_combine=0, block_combine=0, grid=0))
+    if lb >= 12:
+        for blk, u, gc in itertools.product((128, 256, 512), (1, 2, 4, 8), gcs):
+            out.append(dict(block=blk, unroll=u, grid_combine=gc, block_combine=0, grid=0))
+        for bc in (1, 2, 3):
+            if mode == "deterministic" and bc in (1, 2):
+                continue
+            out.append(dict(block=256, unroll=2, grid_combine=gcs[0], block_combine=bc, grid=0))
+    if lb >= 24:
+        for blk, g in itertools.product((256, 512), (148 * 2, 148 * 4, 148 * 8)):
+            out.append(dict(block=blk, unroll=4, grid_combine=gcs[0], block_combine=0, grid=g))
+    return [c for c in out if c["block"] <= MAXBLK(dtype, op, c["unroll"])]
+
+
+def run(args):
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    from cudatiming import time_calls, disjoint_regions
+
+    dev = torch.device("cuda", 0)
+    stream = torch.cuda.Stream(dev)
+    pool_bytes = 2 << 30
+    pools = {}
+    results = []
+    t_start = time.time()
+    for dtype in args.dtypes:
+        tdt = getattr(torch, dtype)
+        if dtype not in pools:
+            p = torch.empty(pool_bytes // ELEM[dtype], dtype=tdt, device=dev)
+            if dtype == "int32":
+                p.random_(-1000, 1000)
+            else:
+                p.uniform_(-1, 1)
+            pools[dtype] = p
+        pool = pools[dtype]
+        rb.prepare(stream, pool.numel())
+        out = torch.empty(4096, dtype=tdt, device=dev)
+        for op, mode in itertools.product(args.ops, args.modes):
+            for lb in range(args.min_lb, args.max_lb + 1):
+                nbytes = 1 << lb
+                n = nbytes // ELEM[dtype]
+                R = max(5, min(100, (400 << 20) // nbytes))
+                warm, timed = disjoint_regions(pool, R, n)
+                best = None
+                for c in candidates(dtype, op, mode, lb):
+                    opts = rb.make_opts(mode=mode, **c)
+                    k = [0]
+
+                    def launch(t, opts=opts):
+                        i = k[0] = (k[0] + 1) % 4096
+                        rb.reduce_ptr(DT[dtype], op, t.data_ptr(), t.numel(), out[i:i + 1].data_ptr(),
+                                      stream.cuda_stream, opts)
+                    try:
+                        s = time_calls(launch, warm, timed, stream, repeats=2)
+                    except Exception as e:  # an invalid combination: record and skip
+                        results.append(dict(dtype=dtype, op=op, mode=mode, lb=lb, cfg=c, error=str(e)[:200]))
+                        torch.cuda.synchronize()
+                        continue
+                    results.append(dict(dtype=dtype, op=op, mode=mode, lb=lb, cfg=c, us=s * 1e6,
+                                        gbps=nbytes / s / 1e9))
+                    if best is None or s < best[0]:
+                        best = (s, c)
+                print(f"[{time.time() - t_start:7.1f}s] {dtype} {op} {mode} 2^{lb}B: best {best[0] * 1e6:8.2f} us "
+                      f"{nbytes / best[0] / 1e9:8.1f} GB/s {best[1]}", flush=True)
+                with open(args.out, "w") as f:
+                    json.dump(results, f)
+    return results
+
+
+def emit(paths, dst):
+    res = []
+    for p in paths:
+        res += [r for r in json.load(open(p)) if "us" in r]
+    best = {}
+    for r in res:
+        key = (r["dtype"], r["op"], r["mode"], r["lb"])
+        if key not in best or r["us"] < best[key]["us"]:
+            best[key] = r
+    rows = []
+    groups = sorted(set(k[:3] for k in best))
+    for dtype, op, mode in groups:
+        lbs = sorted(k[3] for k in best if k[:3] == (dtype, op, mode))
+        prev = None
+        for i, lb in enumerate(lbs):
+            c = best[(dtype, op, mode, lb)]["cfg"]
+            sig = (c["block"], c["unroll"], c["grid_combine"], c["block_combine"], c["grid"])
+            last = i == len(lbs) - 1
+            nxt = None if last else best[(dtype, op, mode, lbs[i + 1])]["cfg"]
+            nsig = None if last else (nxt["block"], nxt["unroll"], nxt["grid_combine"], nxt["block_combine"], nxt["grid"])
+            if sig != nsig:
+                rows.append((DT[dtype], OPC[op], MODE[mode], 63 if last else lb) + sig +
+                            (round(best[(dtype, op, mode, lb)]["gbps"], 1),))
+        # min mirrors max when only max was tuned
+        if op == "max" and (dtype, "min", mode) not in groups:
+            for r in [r for r in rows if r[:3] == (DT[dtype], OPC["max"], MODE[mode])]:
+                rows.append((r[0], OPC["min"]) + r[2:])
+    lines = [
+        "// dispatch_table.inc -- variant / launch choice per (dtype, op, mode, size).",
+        "// Step S0 of DESIGN.md: the paper picks a code version per size and",
+        "// architecture by tuning (P:L483); the winners change with size",
+        "// (P:L681-L687, P:L691-L735, P:L739-L781).  GENERATED by tools/tune.py from",
+        "// B200 measurements (device time per call, cold inputs); first match wins.",
+        "//",
+        "// fields: dtype, op, mode, max_log2_bytes, block, unroll, grid_combine, block_combine, grid_cap",
+        "//   (grid_cap 0 = one block per tile)      // measured GB/s at the bucket that ended the row",
+        "static const DispatchEntry kDispatch[] = {",
+    ]
+    for r in rows:
+        lines.append("    {%d, %d, %d, %d, %d, %d, %d, %d, %d},  // %.1f GB/s" % r)
+    lines += ["    {-1, -1, -1, 63, 256, 4, -1, 0, 0},  // fallback", "};", ""]
+    open(dst, "w").write("\n".join(lines))
+    print(f"wrote {len(rows)} rows to {dst}")
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--dtypes", nargs="+", default=["int32", "float32", "float64"])
+    ap.add_argument("--ops", nargs="+", default=["sum", "max"])
+    ap.add_argument("--modes", nargs="+", default=["fast", "deterministic"])
+    ap.add_argument("--min-lb", type=int, default=7)
+    ap.add_argument("--max-lb", type=int, default=30)
+    ap.add_argument("--out", default="gpurun_out/tune.json")
+    ap.add_argument("--emit", nargs="*")
+    ap.add_argument("--dst", default=os.path.join(ROOT, "paper_conf_cgo_gonzalohghmh19_b200", "csrc",
+                                                  "dispatch_table.inc"))
+    args = ap.parse_args()
+    if args.emit:
+        return emit(args.emit, args.dst)
+    run(args)
+
+
+if __name__ == "__main__":
+    main()
