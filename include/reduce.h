@@ -96,12 +96,19 @@ typedef enum {
  *   TWO_PASS   : per-block partials + a second single-block kernel, no atomics
  *                (Listing 1 + second spectrum call)
  *   LAST_BLOCK : per-block partials; the last block (integer ticket) reduces
- *                them in a fixed order -- deterministic, one launch */
+ *                them in a fixed order -- deterministic, one launch
+ *   CLUSTER    : one thread-block cluster of `grid` CTAs (<= 16, on 16 SMs of
+ *                one GPC) loops over all tiles; CTA partials meet in CTA 0's
+ *                shared memory through distributed shared memory (DSMEM) and a
+ *                cluster barrier -- no atomics, deterministic, one launch; the
+ *                sm_90+/sm_100 form of the paper's two-stage per-SM partition
+ *                 for medium arrays */
 typedef enum {
   REDUCE_GC_DIRECT = 0,
   REDUCE_GC_ATOMIC = 1,
   REDUCE_GC_TWO_PASS = 2,
-  REDUCE_GC_LAST_BLOCK = 3
+  REDUCE_GC_LAST_BLOCK = 3,
+  REDUCE_GC_CLUSTER = 4
 } reduce_grid_combine_t;
 
 /* Options for reduce_ex & co.  Zero-initialise, then set fields; every field
@@ -113,7 +120,8 @@ typedef struct {
   int block;          /* threads per block: 0 = auto, else 32..1024, multiple of 32
                          (power of two for SMEM_TREE) */
   int unroll;         /* 32-byte vectors per thread per tile: 0 = auto, else 1,2,4,8 */
-  int grid;           /* 0 = auto (one block per tile, capped), else max blocks */
+  int grid;           /* 0 = auto (one block per tile, capped), else max blocks;
+                         for REDUCE_GC_CLUSTER: the cluster size, 1..16 (0 = 16) */
 } reduce_opts_t;
 
 /* What a call will launch (filled by reduce_query_plan). */

@@ -20,7 +20,7 @@ INT32, FLOAT32, FLOAT64 = 0, 1, 2
 SUM, MIN, MAX = 0, 1, 2
 MODE_FAST, MODE_DETERMINISTIC = 0, 1
 BC_SHFL, BC_SMEM_ATOMIC_WARP, BC_SMEM_ATOMIC_ALL, BC_SMEM_TREE = 0, 1, 2, 3
-GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK = 0, 1, 2, 3
+GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER = 0, 1, 2, 3, 4
 OK = 0
 
 OPS = {"sum": SUM, "min": MIN, "max": MAX}

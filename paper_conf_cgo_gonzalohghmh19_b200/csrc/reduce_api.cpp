@@ -64,7 +64,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   int mode = o.mode < 0 ? g_mode.load() : o.mode;
   if (mode != REDUCE_MODE_FAST && mode != REDUCE_MODE_DETERMINISTIC)
     return fail(REDUCE_ERR_INVALID_ARG, "mode must be -1, REDUCE_MODE_FAST or REDUCE_MODE_DETERMINISTIC");
-  if (o.grid_combine < -1 || o.grid_combine > 3) return fail(REDUCE_ERR_INVALID_ARG, "bad grid_combine");
+  if (o.grid_combine < -1 || o.grid_combine > 4) return fail(REDUCE_ERR_INVALID_ARG, "bad grid_combine");
   if (o.block_combine < -1 || o.block_combine > 3) return fail(REDUCE_ERR_INVALID_ARG, "bad block_combine");
   if (o.unroll != 0 && o.unroll != 1 && o.unroll != 2 && o.unroll != 4 && o.unroll != 8)
     return fail(REDUCE_ERR_INVALID_ARG, "unroll must be 0, 1, 2, 4 or 8");
@@ -126,6 +126,10 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   long long grid;
   if (gc == REDUCE_GC_DIRECT) {
     grid = 1;
+  } else if (gc == REDUCE_GC_CLUSTER) {
+    grid = grid_cap > 0 ? grid_cap : 16;
+    if (grid > 16) return fail(REDUCE_ERR_INVALID_ARG, "cluster size must be <= 16");
+    if (tiles > 0 && grid > tiles) grid = tiles;
   } else {
     grid = tiles > 0 ? tiles : 1;
     if (grid_cap > 0 && grid_cap < grid) grid = grid_cap;
@@ -156,6 +160,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
         case REDUCE_GC_ATOMIC: chain += (grid + nslots - 1) / nslots + 5; break;
         case REDUCE_GC_TWO_PASS: chain += (grid + 1023) / 1024 + 10; break;
         case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + ilog2_ceil(block); break;
+        case REDUCE_GC_CLUSTER: chain += 5; break;
         default: break;
       }
     }

@@ -22,7 +22,7 @@ namespace rb {
 constexpr int DT_I32 = 0, DT_F32 = 1, DT_F64 = 2;
 constexpr int OP_SUM = 0, OP_MIN = 1, OP_MAX = 2;
 constexpr int BC_SHFL = 0, BC_ATOMIC_WARP = 1, BC_ATOMIC_ALL = 2, BC_TREE = 3;
-constexpr int GC_DIRECT = 0, GC_ATOMIC = 1, GC_TWO_PASS = 2, GC_LAST_BLOCK = 3;
+constexpr int GC_DIRECT = 0, GC_ATOMIC = 1, GC_TWO_PASS = 2, GC_LAST_BLOCK = 3, GC_CLUSTER = 4;
 constexpr int kVecBytes = 32;    // one 256-bit load per thread per vector
 
 // ------------------------------------------------------------------ loads ---

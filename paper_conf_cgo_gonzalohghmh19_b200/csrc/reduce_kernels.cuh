@@ -20,7 +20,10 @@
 //   * warp / block combine (S3, S4): block_combine<BC>.
 //   * grid combine (S5) and finalise (S6): by desc.gc, see grid_combine().
 #pragma once
+#include <cooperative_groups.h>
+#include <mutex>
 #include <type_traits>
+#include <unordered_set>
 #include "reduce_device.cuh"
 #include "reduce_internal.h"
 
@@ -53,6 +56,23 @@ __device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& 
   __shared__ int s_last;
   if (p.gc == GC_DIRECT) {
     if (threadIdx.x == 0) store_out<T>(g, p);
+    return;
+  }
+  if (p.gc == GC_CLUSTER) {
+    // CTA partials meet in CTA 0's shared memory over DSMEM; one cluster
+    // barrier (release/acquire) orders the remote stores before CTA 0 reads.
+    namespace cg = cooperative_groups;
+    __shared__ Grid cl_vals[16];
+    cg::cluster_group cluster = cg::this_cluster();
+    const unsigned r = cluster.block_rank();
+    if (threadIdx.x == 0) cluster.map_shared_rank(&cl_vals[0], 0)[r] = g;
+    cluster.sync();
+    if (r == 0 && threadIdx.x < 32) {
+      const unsigned C = cluster.num_blocks();
+      Grid x = threadIdx.x < C ? cl_vals[threadIdx.x] : T::gident();
+      x = T::gwarp(x);
+      if (threadIdx.x == 0) store_out<T>(x, p);
+    }
     return;
   }
   if (p.gc == GC_TWO_PASS) {  // Listing 1: Return[blockIdx.x] = ...; second launch reduces
@@ -183,16 +203,47 @@ inline KParams make_params(const LaunchDesc& d) {
   return p;
 }
 
+// Launch one k_reduce instantiation; GC_CLUSTER launches exactly one cluster
+// of d.grid CTAs (sizes above the portable 8 need the non-portable opt-in).
+inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& d, const KParams& p, cudaStream_t s) {
+  if (d.gc != GC_CLUSTER) {
+    kern<<<d.grid, d.block, 0, s>>>(p);
+    return cudaPeekAtLastError();
+  }
+  if (d.grid > 8) {
+    static std::mutex mu;
+    static std::unordered_set<const void*> opted;
+    std::lock_guard<std::mutex> lk(mu);
+    if (!opted.count((const void*)kern)) {
+      cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+      if (e != cudaSuccess) return e;
+      opted.insert((const void*)kern);
+    }
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(d.grid, 1, 1);
+  cfg.blockDim = dim3(d.block, 1, 1);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = d.grid;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, p);
+}
+
 template <int DT, int OP, int U>
 cudaError_t launch_u(const LaunchDesc& d, const KParams& p, cudaStream_t s) {
   switch (d.bc) {
-    case BC_SHFL: k_reduce<DT, OP, U, BC_SHFL><<<d.grid, d.block, 0, s>>>(p); break;
-    case BC_ATOMIC_WARP: k_reduce<DT, OP, U, BC_ATOMIC_WARP><<<d.grid, d.block, 0, s>>>(p); break;
-    case BC_ATOMIC_ALL: k_reduce<DT, OP, U, BC_ATOMIC_ALL><<<d.grid, d.block, 0, s>>>(p); break;
-    case BC_TREE: k_reduce<DT, OP, U, BC_TREE><<<d.grid, d.block, 0, s>>>(p); break;
-    default: return cudaErrorInvalidValue;
+    case BC_SHFL: return launch_kernel(k_reduce<DT, OP, U, BC_SHFL>, d, p, s);
+    case BC_ATOMIC_WARP: return launch_kernel(k_reduce<DT, OP, U, BC_ATOMIC_WARP>, d, p, s);
+    case BC_ATOMIC_ALL: return launch_kernel(k_reduce<DT, OP, U, BC_ATOMIC_ALL>, d, p, s);
+    case BC_TREE: return launch_kernel(k_reduce<DT, OP, U, BC_TREE>, d, p, s);
   }
-  return cudaPeekAtLastError();
+  return cudaErrorInvalidValue;
 }
 
 template <int DT, int OP>

@@ -112,7 +112,7 @@ def test_size_sweep(dtype):
 # ------------------------------------------------------------- every variant on the same inputs
 VARIANTS = []
 for bc in range(4):
-    for gc in range(4):
+    for gc in range(5):
         for blk, u in ((32, 1), (128, 2), (256, 4), (512, 8), (1024, 1)):
             VARIANTS.append(dict(block_combine=bc, grid_combine=gc, block=blk, unroll=u))
 
@@ -129,6 +129,22 @@ def test_every_variant(dtype):
         got, plans = gpu_reduce_many([(t, op) for op in OPS], **v)
         for op, g, p in zip(OPS, got, plans):
             check(x, op, g, p)
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+def test_cluster_dsmem_combine_all_sizes(dtype):
+    """GC_CLUSTER: one cluster of C CTAs (C = 1..16) combining through DSMEM;
+    deterministic (no atomics) and exact for int32 / min / max."""
+    cases, xs, plans_kw = [], [], []
+    for k, n in enumerate([1, 33, 4097, 65537, (1 << 20) + 3]):
+        x = synth.make(dtype, n, _dist(dtype), 300 + k)
+        t = to_device(x, k % 4)
+        for C in (1, 2, 3, 8, 13, 16):
+            for blk in (128, 512):
+                got, plans = gpu_reduce_many([(t, op) for op in OPS], grid_combine=4, grid=C, block=blk)
+                for op, g, p in zip(OPS, got, plans):
+                    check(x, op, g, p)
+                    assert p["grid_combine"] == 4 and p["grid"] <= C
 
 
 @pytest.mark.parametrize("grid", [1, 7, 148, 1000])

@@ -46,6 +46,9 @@ def candidates(dtype, op, mode, lb):
             if mode == "deterministic" and bc in (1, 2):
                 continue
             out.append(dict(block=256, unroll=2, grid_combine=gcs[0], block_combine=bc, grid=0))
+    if 10 <= lb <= 26:
+        for blk, u, c in itertools.product((256, 512, 1024), (1, 2, 4), (4, 8, 16)):
+            out.append(dict(block=blk, unroll=u, grid_combine=4, block_combine=0, grid=c))
     if lb >= 24:
         for blk, g in itertools.product((256, 512), (148 * 2, 148 * 4, 148 * 8)):
             out.append(dict(block=blk, unroll=4, grid_combine=gcs[0], block_combine=0, grid=g))
@@ -107,29 +110,37 @@ def run(args):
     return results
 
 
-def emit(paths, dst):
+def emit(paths, dst, tol=0.01):
+    """Pick, per (dtype, op, mode, log2 bytes), the fastest candidate -- but among
+    candidates within `tol` of the fastest (timer noise) keep the previous size
+    bucket's choice when it qualifies, so the table only changes where the
+    measurements say it must."""
     res = []
     for p in paths:
         res += [r for r in json.load(open(p)) if "us" in r]
-    best = {}
+    by = {}
     for r in res:
-        key = (r["dtype"], r["op"], r["mode"], r["lb"])
-        if key not in best or r["us"] < best[key]["us"]:
-            best[key] = r
+        by.setdefault((r["dtype"], r["op"], r["mode"], r["lb"]), []).append(r)
+    sig = lambda c: (c["block"], c["unroll"], c["grid_combine"], c["block_combine"], c["grid"])
     rows = []
-    groups = sorted(set(k[:3] for k in best))
+    groups = sorted(set(k[:3] for k in by))
     for dtype, op, mode in groups:
-        lbs = sorted(k[3] for k in best if k[:3] == (dtype, op, mode))
+        lbs = sorted(k[3] for k in by if k[:3] == (dtype, op, mode))
+        chosen = []
         prev = None
-        for i, lb in enumerate(lbs):
-            c = best[(dtype, op, mode, lb)]["cfg"]
-            sig = (c["block"], c["unroll"], c["grid_combine"], c["block_combine"], c["grid"])
-            last = i == len(lbs) - 1
-            nxt = None if last else best[(dtype, op, mode, lbs[i + 1])]["cfg"]
-            nsig = None if last else (nxt["block"], nxt["unroll"], nxt["grid_combine"], nxt["block_combine"], nxt["grid"])
-            if sig != nsig:
-                rows.append((DT[dtype], OPC[op], MODE[mode], 63 if last else lb) + sig +
-                            (round(best[(dtype, op, mode, lb)]["gbps"], 1),))
+        for lb in lbs:
+            cands = by[(dtype, op, mode, lb)]
+            fastest = min(r["us"] for r in cands)
+            ok = [r for r in cands if r["us"] <= fastest * (1 + tol)]
+            keep = [r for r in ok if prev is not None and sig(r["cfg"]) == prev]
+            pick = keep[0] if keep else min(ok, key=lambda r: r["us"])
+            prev = sig(pick["cfg"])
+            chosen.append((lb, pick))
+        for i, (lb, pick) in enumerate(chosen):
+            last = i == len(chosen) - 1
+            if last or sig(chosen[i + 1][1]["cfg"]) != sig(pick["cfg"]):
+                rows.append((DT[dtype], OPC[op], MODE[mode], 63 if last else lb) + sig(pick["cfg"]) +
+                            (round(pick["gbps"], 1),))
         # min mirrors max when only max was tuned
         if op == "max" and (dtype, "min", mode) not in groups:
             for r in [r for r in rows if r[:3] == (DT[dtype], OPC["max"], MODE[mode])]:
