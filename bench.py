@@ -299,42 +299,59 @@ def main():
                "path": "reduce_host (C ABI, pinned host buffer, chunked H2D overlapped with the chunk reductions)"
                if comm is None else "pinned H2D copy + reduce_multi + D2H of the result"}
 
-    # ---- size sweep (rank 0 only, N = 1): each call after an L2 flush
-    sweep = None
+    # ---- size sweep (N = 1): device time per call from a CUDA graph of R calls
+    # over disjoint, never-recently-touched regions of the resident 1 GiB input
+    # (cold: every call reads HBM), plus the small-array latency regime
+    # (BASELINE configs[3]) measured three ways.
+    sweep = latency = None
     if not args.no_sweep and world == 1:
+        sys.path.insert(0, os.path.join(ROOT, "tools"))
+        from cudatiming import time_calls, disjoint_regions
+        outs = torch.empty(4096, dtype=torch.float32, device=dev)
         sweep = []
-        flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)  # 256 MB > L2
-        xs = x  # sizes are prefixes of the resident 1 GiB input
-        for k in range(10, 29, 2):
+        for k in range(6, 29, 2):
             m = 1 << k
-            sub = xs[:m]
-            p = rb.query_plan("float32", "sum", m, in_ptr=sub.data_ptr(), mode=args.mode)
-            times = []
-            with torch.cuda.stream(stream):
-                for _ in range(3):
-                    rb.reduce(sub, "sum", out=out, stream=stream, mode=args.mode)
-                for _ in range(15):
-                    flush.fill_(1.0)
-                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                    a.record(stream)
-                    rb.reduce(sub, "sum", out=out, stream=stream, mode=args.mode)
-                    b.record(stream)
-                    times.append((a, b))
-                torch.cuda.synchronize(dev)
-                cold = statistics.median([a.elapsed_time(b) for a, b in times])
+            R = max(3, min(100, (256 << 20) // (4 * m)))
+            warm, timed = disjoint_regions(x, R, m)
+            p = rb.query_plan("float32", "sum", m, in_ptr=timed[0].data_ptr(), mode=args.mode)
+            ctr = [0]
+
+            def launch(t):
+                ctr[0] = (ctr[0] + 1) % 4096
+                rb.reduce(t, "sum", out=outs[ctr[0]:ctr[0] + 1], stream=stream, mode=args.mode)
+            sec = time_calls(launch, warm, timed, stream, repeats=3)
+            gbs = m * 4 / sec / 1e9
+            sweep.append({"n": m, "us": round(sec * 1e6, 3), "GBps": round(gbs, 1),
+                          "elements_per_s": round(m / sec, 1), "frac_of_peak": round(gbs / peak, 4),
+                          "variant": f"gc{p['grid_combine']} g{p['grid']}x{p['block']} u{p['unroll']}"})
+        latency = []
+        for dt in ("int32", "float32"):
+            tdt = getattr(torch, dt)
+            src = torch.ones(1 << 20, dtype=tdt, device=dev)
+            o1 = torch.empty(4096, dtype=tdt, device=dev)
+            for m in (32, 1024, 65536):
+                warm, timed = disjoint_regions(src, 50, m)
+                ctr = [0]
+
+                def launch(t, o1=o1):
+                    ctr[0] = (ctr[0] + 1) % 4096
+                    rb.reduce(t, "sum", out=o1[ctr[0]:ctr[0] + 1], stream=stream)
+                g_us = time_calls(launch, warm, timed, stream, repeats=3) * 1e6
                 a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 a.record(stream)
-                for _ in range(50):
-                    rb.reduce(sub, "sum", out=out, stream=stream, mode=args.mode)
+                for t in timed:
+                    launch(t)
                 b.record(stream)
-                torch.cuda.synchronize(dev)
-                warm = a.elapsed_time(b) / 50
-            sweep.append({"n": m, "cold_us": round(cold * 1e3, 2), "cold_GBps": round(m * 4 / (cold * 1e-3) / 1e9, 1),
-                          "cold_frac_of_peak": round(m * 4 / (cold * 1e-3) / 1e9 / peak, 4),
-                          "warm_b2b_us": round(warm * 1e3, 2),
-                          "warm_GBps": round(m * 4 / (warm * 1e-3) / 1e9, 1),
-                          "variant": f"g{p['grid']}x{p['block']}u{p['unroll']} gc{p['grid_combine']}"})
-        del flush
+                b.synchronize()
+                s_us = a.elapsed_time(b) * 1e3 / len(timed)
+                walls = []
+                for t in timed[:20]:
+                    t0 = time.perf_counter()
+                    launch(t)
+                    stream.synchronize()
+                    walls.append(time.perf_counter() - t0)
+                latency.append({"dtype": dt, "n": m, "graph_us": round(g_us, 3), "stream_b2b_us": round(s_us, 3),
+                                "host_wall_us": round(statistics.median(walls) * 1e6, 2)})
 
     # ---- CPU baseline: the oracle on the host cores (rank 0, N = 1)
     cpu = None
@@ -374,6 +391,7 @@ def main():
             line["cpu_openmp"] = cpu_omp
         if sweep is not None:
             line["sweep"] = sweep
+            line["small_array_latency"] = latency
         if ncu_s is not None:
             line["ncu"] = {k: ncu_s[k] for k in ("source", "dram_pct_of_peak", "duration_us") if k in ncu_s}
         print(json.dumps(line), flush=True)

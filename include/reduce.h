@@ -119,15 +119,22 @@ typedef struct {
   int block_combine;  /* -1 = auto, else reduce_block_combine_t */
   int block;          /* threads per block: 0 = auto, else 32..1024, multiple of 32
                          (power of two for SMEM_TREE) */
-  int unroll;         /* 32-byte vectors per thread per tile: 0 = auto, else 1,2,4,8 */
+  int unroll;         /* 32-byte vectors per thread per tile: 0 = auto, else 1,2,4,8
+                         (register staging) or 4,8,16 (shared-memory staging) */
   int grid;           /* 0 = auto (one block per tile, capped), else max blocks;
                          for REDUCE_GC_CLUSTER: the cluster size, 1..16 (0 = 16) */
+  int stage;          /* 0 = auto; REDUCE_STAGE_REG: 256-bit loads straight into
+                         registers; REDUCE_STAGE_SMEM: cp.async 16-byte copies into a
+                         shared-memory tile (block*unroll*32 <= 128 KiB), then shared
+                         loads -- more bytes in flight per SM.  Same numerics. */
 } reduce_opts_t;
+
+typedef enum { REDUCE_STAGE_AUTO = 0, REDUCE_STAGE_REG = 1, REDUCE_STAGE_SMEM = 2 } reduce_stage_t;
 
 /* What a call will launch (filled by reduce_query_plan). */
 typedef struct {
   int grid_combine, block_combine;
-  int grid, block, unroll;
+  int grid, block, unroll, stage;
   int launches;        /* kernel launches per call: 1, or 2 for TWO_PASS */
   int slots;           /* global accumulator slots used by ATOMIC */
   int head, tail;      /* scalar elements before / after the 32-byte-aligned body */

@@ -21,6 +21,7 @@ SUM, MIN, MAX = 0, 1, 2
 MODE_FAST, MODE_DETERMINISTIC = 0, 1
 BC_SHFL, BC_SMEM_ATOMIC_WARP, BC_SMEM_ATOMIC_ALL, BC_SMEM_TREE = 0, 1, 2, 3
 GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER = 0, 1, 2, 3, 4
+STAGE_REG, STAGE_SMEM = 1, 2
 OK = 0
 
 OPS = {"sum": SUM, "min": MIN, "max": MAX}
@@ -46,13 +47,14 @@ class ReduceError(RuntimeError):
 
 class reduce_opts_t(ctypes.Structure):
     _fields_ = [("mode", ctypes.c_int), ("grid_combine", ctypes.c_int), ("block_combine", ctypes.c_int),
-                ("block", ctypes.c_int), ("unroll", ctypes.c_int), ("grid", ctypes.c_int)]
+                ("block", ctypes.c_int), ("unroll", ctypes.c_int), ("grid", ctypes.c_int),
+                ("stage", ctypes.c_int)]
 
 
 class reduce_plan_t(ctypes.Structure):
     _fields_ = [("grid_combine", ctypes.c_int), ("block_combine", ctypes.c_int),
                 ("grid", ctypes.c_int), ("block", ctypes.c_int), ("unroll", ctypes.c_int),
-                ("launches", ctypes.c_int), ("slots", ctypes.c_int),
+                ("stage", ctypes.c_int), ("launches", ctypes.c_int), ("slots", ctypes.c_int),
                 ("head", ctypes.c_int), ("tail", ctypes.c_int),
                 ("tiles", ctypes.c_longlong), ("chain", ctypes.c_longlong)]
 
@@ -110,13 +112,15 @@ def _check(status: int, where: str) -> None:
         raise ReduceError(status, where)
 
 
-def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=0, grid=0):
+def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=0, grid=0, stage=0):
     if isinstance(mode, str):
         mode = {"fast": MODE_FAST, "deterministic": MODE_DETERMINISTIC}[mode]
+    if isinstance(stage, str):
+        stage = {"auto": 0, "reg": STAGE_REG, "smem": STAGE_SMEM}[stage]
     return reduce_opts_t(-1 if mode is None else int(mode),
                          -1 if grid_combine is None else int(grid_combine),
                          -1 if block_combine is None else int(block_combine),
-                         int(block), int(unroll), int(grid))
+                         int(block), int(unroll), int(grid), int(stage))
 
 
 def _op(op) -> int:

@@ -15,7 +15,7 @@
 namespace rb {
 
 struct DispatchEntry {
-  int dtype, op, mode, max_log2_bytes, block, unroll, gc, bc, grid_cap;
+  int dtype, op, mode, max_log2_bytes, block, unroll, gc, bc, grid_cap, stage;  // stage 0 = registers
 };
 #include "dispatch_table.inc"
 
@@ -59,15 +59,16 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   if (n > (size_t)1 << 46) return fail(REDUCE_ERR_INVALID_ARG, "n too large");
 
   reduce_opts_t o;
-  o.mode = -1; o.grid_combine = -1; o.block_combine = -1; o.block = 0; o.unroll = 0; o.grid = 0;
+  o.mode = -1; o.grid_combine = -1; o.block_combine = -1; o.block = 0; o.unroll = 0; o.grid = 0; o.stage = 0;
   if (opts) o = *opts;
   int mode = o.mode < 0 ? g_mode.load() : o.mode;
   if (mode != REDUCE_MODE_FAST && mode != REDUCE_MODE_DETERMINISTIC)
     return fail(REDUCE_ERR_INVALID_ARG, "mode must be -1, REDUCE_MODE_FAST or REDUCE_MODE_DETERMINISTIC");
   if (o.grid_combine < -1 || o.grid_combine > 4) return fail(REDUCE_ERR_INVALID_ARG, "bad grid_combine");
   if (o.block_combine < -1 || o.block_combine > 3) return fail(REDUCE_ERR_INVALID_ARG, "bad block_combine");
-  if (o.unroll != 0 && o.unroll != 1 && o.unroll != 2 && o.unroll != 4 && o.unroll != 8)
-    return fail(REDUCE_ERR_INVALID_ARG, "unroll must be 0, 1, 2, 4 or 8");
+  if (o.unroll != 0 && o.unroll != 1 && o.unroll != 2 && o.unroll != 4 && o.unroll != 8 && o.unroll != 16)
+    return fail(REDUCE_ERR_INVALID_ARG, "unroll must be 0, 1, 2, 4, 8 or 16");
+  if (o.stage < 0 || o.stage > 2) return fail(REDUCE_ERR_INVALID_ARG, "stage must be 0, 1 or 2");
   if (o.block != 0 && (o.block < 32 || o.block > 1024 || o.block % 32 != 0))
     return fail(REDUCE_ERR_INVALID_ARG, "block must be 0 or a multiple of 32 in [32, 1024]");
   if (o.grid < 0) return fail(REDUCE_ERR_INVALID_ARG, "grid must be >= 0");
@@ -91,8 +92,19 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   }
   if (!e) e = &kDispatch[sizeof(kDispatch) / sizeof(kDispatch[0]) - 1];
 
+  int stage = o.stage ? o.stage : (e->stage == REDUCE_STAGE_SMEM ? REDUCE_STAGE_SMEM : REDUCE_STAGE_REG);
   int block = o.block ? o.block : e->block;
   int unroll = o.unroll ? o.unroll : e->unroll;
+  if (stage == REDUCE_STAGE_SMEM && !o.unroll && unroll < 4) unroll = 4;
+  if (stage == REDUCE_STAGE_REG && !o.unroll && unroll > 8) unroll = 8;
+  if (stage == REDUCE_STAGE_SMEM) {
+    if (unroll != 4 && unroll != 8 && unroll != 16)
+      return fail(REDUCE_ERR_INVALID_ARG, "shared-memory staging supports unroll 4, 8 or 16");
+    if ((long long)block * unroll * 32 > kMaxSmemTileBytes)
+      return fail(REDUCE_ERR_INVALID_ARG, "shared-memory tile (block*unroll*32) exceeds 128 KiB");
+  } else if (unroll > 8) {
+    return fail(REDUCE_ERR_INVALID_ARG, "register staging supports unroll 1, 2, 4 or 8");
+  }
   int bc = o.block_combine >= 0 ? o.block_combine : e->bc;
   int gc;
   if (o.grid_combine >= 0) gc = o.grid_combine;
@@ -103,9 +115,9 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
       (bc == REDUCE_BC_SMEM_ATOMIC_WARP || bc == REDUCE_BC_SMEM_ATOMIC_ALL))
     bc = REDUCE_BC_SHFL;
   const int grid_cap = o.grid > 0 ? o.grid : e->grid_cap;
-  if (block > max_block_threads(dtype, op, unroll))
+  if (block > max_block_threads(dtype, op, unroll, stage))
     return fail(REDUCE_ERR_INVALID_ARG, "block too large for this (dtype, op, unroll): max " +
-                                            std::to_string(max_block_threads(dtype, op, unroll)));
+                                            std::to_string(max_block_threads(dtype, op, unroll, stage)));
   if (bc == REDUCE_BC_SMEM_TREE && (block & (block - 1)) != 0)
     return fail(REDUCE_ERR_INVALID_ARG, "SMEM_TREE needs a power-of-two block");
 
@@ -173,12 +185,12 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   d.body = (const char*)in + head * s;
   d.body_vecs = body_vecs; d.tiles = tiles;
   d.head = (int)head; d.tail = tail;
-  d.grid = (int)grid; d.block = block; d.unroll = unroll; d.bc = bc; d.gc = gc;
+  d.grid = (int)grid; d.block = block; d.unroll = unroll; d.bc = bc; d.gc = gc; d.stage = stage;
   d.raw_out = raw_out; d.nslots = nslots;
 
   reduce_plan_t& p = P->pub;
   p.grid_combine = gc; p.block_combine = bc;
-  p.grid = (int)grid; p.block = block; p.unroll = unroll;
+  p.grid = (int)grid; p.block = block; p.unroll = unroll; p.stage = stage;
   p.launches = gc == REDUCE_GC_TWO_PASS ? 2 : 1;
   p.slots = nslots; p.head = (int)head; p.tail = tail;
   p.tiles = tiles; p.chain = chain;

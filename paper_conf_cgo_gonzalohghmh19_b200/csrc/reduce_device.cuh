@@ -35,6 +35,19 @@ __device__ __forceinline__ void ld_v8(const void* p, uint32_t (&r)[8]) {
       : "l"(p));
 }
 
+// cp.async (LDGSTS): 16 bytes global -> shared, L2 only (.cg), asynchronous.
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+// one 32-byte vector from shared memory as 8 words
+__device__ __forceinline__ void lds_v8(const void* smem, uint32_t (&r)[8]) {
+  const uint4 a = reinterpret_cast<const uint4*>(smem)[0];
+  const uint4 b = reinterpret_cast<const uint4*>(smem)[1];
+  r[0] = a.x; r[1] = a.y; r[2] = a.z; r[3] = a.w; r[4] = b.x; r[5] = b.y; r[6] = b.z; r[7] = b.w;
+}
+
 // ------------------------------------------------------- fp primitives ---
 __device__ __forceinline__ float fmax_nan(float a, float b) {
   float r; asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r;

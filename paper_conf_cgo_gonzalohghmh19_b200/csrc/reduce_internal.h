@@ -10,11 +10,21 @@ namespace rb {
 constexpr int kSlotBytes = 256;  // stride between global accumulator slots (separate L2 lines)
 constexpr int kMaxSlots = 32;
 
-// Largest block the (dtype, op, unroll) instantiation is compiled for: the
-// register budget of 64/thread at 1024 threads is too small for 8 in-flight
-// 32-byte loads, and for the fp64 min/max select+NaN-flag fold at unroll >= 2.
-constexpr int max_block_threads(int dtype, int op, int unroll) {
-  return (unroll >= 8 || (dtype == 2 && op != 0 && unroll >= 2)) ? 512 : 1024;
+// How a tile reaches the registers (step S2):
+//   STAGE_REG  : 256-bit LDG straight into registers (U loads per thread);
+//   STAGE_SMEM : cp.async (LDGSTS) 16-byte copies into a per-block shared
+//                tile, then 128-bit shared loads -- the bytes in flight are not
+//                bounded by registers, so a block can keep 64 KB in flight.
+// Both fold the same vectors in the same order (identical numerics).
+constexpr int STAGE_REG = 1, STAGE_SMEM = 2;
+constexpr int kMaxSmemTileBytes = 128 * 1024;
+
+// Largest block the (dtype, op, unroll, stage) instantiation is compiled for:
+// with register staging, the budget of 64 registers/thread at 1024 threads is
+// too small for 8 in-flight 32-byte loads, and for the fp64 min/max
+// select+NaN-flag fold at unroll >= 2.
+constexpr int max_block_threads(int dtype, int op, int unroll, int stage = STAGE_REG) {
+  return stage == STAGE_SMEM ? 1024 : ((unroll >= 8 || (dtype == 2 && op != 0 && unroll >= 2)) ? 512 : 1024);
 }
 
 // One launch of the main reduction kernel (steps S2-S5), fully resolved by the
@@ -26,7 +36,7 @@ struct LaunchDesc {
   unsigned long long body_vecs;  // 32-byte vectors in the body
   long long tiles;               // ceil(body_vecs / (block*unroll))
   int head, tail;                // scalar elements before / after the body
-  int grid, block, unroll, bc, gc;
+  int grid, block, unroll, bc, gc, stage;
   void* out;                     // device scalar (T, or the raw Grid type)
   int raw_out;                   // 1: write the un-finalised Grid value
   void* slots;                   // this (dtype, op)'s accumulator slots (GC_ATOMIC)

@@ -124,8 +124,8 @@ __device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& 
   }
 }
 
-template <int DT, int OP, int U, int BC>
-__global__ void __launch_bounds__(max_block_threads(DT, OP, U)) k_reduce(const KParams p) {
+template <int DT, int OP, int U, int BC, int STAGE>
+__global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(const KParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
   Acc a[T::NA];
@@ -138,7 +138,31 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U)) k_reduce(const K
   for (long long tile = blockIdx.x; tile < p.tiles; tile += gridDim.x) {
     const unsigned long long v0 = (unsigned long long)(tile * tile_vecs) + threadIdx.x;
     const char* ptr = p.body + v0 * kVecBytes;
-    if ((unsigned long long)((tile + 1) * tile_vecs) <= p.body_vecs) {
+    const bool full = (unsigned long long)((tile + 1) * tile_vecs) <= p.body_vecs;
+    if constexpr (STAGE == STAGE_SMEM) {
+      // Each thread stages exactly the vectors it will fold (vector v0 + u*B
+      // -> slot u*B + t), so no block barrier is needed: cp.async.wait_all
+      // waits for this thread's own copies.  All 2U copies are in flight at once.
+      extern __shared__ __align__(128) unsigned char stile[];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (full || v0 + (unsigned long long)(u * B) < p.body_vecs) {
+          unsigned char* d = stile + ((size_t)u * B + threadIdx.x) * kVecBytes;
+          const char* g = ptr + (size_t)u * B * kVecBytes;
+          cp_async16(d, g);
+          cp_async16(d + 16, g + 16);
+        }
+      }
+      cp_async_wait_all();
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (full || v0 + (unsigned long long)(u * B) < p.body_vecs) {
+          uint32_t r[8];
+          lds_v8(stile + ((size_t)u * B + threadIdx.x) * kVecBytes, r);
+          fold_vec<T>(a, aux, r);
+        }
+      }
+    } else if (full) {
       uint32_t r[U][8];
 #pragma unroll
       for (int u = 0; u < U; ++u) ld_v8(ptr + (size_t)u * B * kVecBytes, r[u]);
@@ -204,26 +228,29 @@ inline KParams make_params(const LaunchDesc& d) {
 }
 
 // Launch one k_reduce instantiation; GC_CLUSTER launches exactly one cluster
-// of d.grid CTAs (sizes above the portable 8 need the non-portable opt-in).
+// of d.grid CTAs (sizes above the portable 8 need the non-portable opt-in);
+// STAGE_SMEM needs block*U*32 bytes of dynamic shared memory (opt-in above 48 KB).
 inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& d, const KParams& p, cudaStream_t s) {
-  if (d.gc != GC_CLUSTER) {
-    kern<<<d.grid, d.block, 0, s>>>(p);
-    return cudaPeekAtLastError();
-  }
-  if (d.grid > 8) {
+  const size_t smem = d.stage == STAGE_SMEM ? (size_t)d.block * d.unroll * kVecBytes : 0;
+  if (smem > 48 * 1024 || (d.gc == GC_CLUSTER && d.grid > 8)) {
     static std::mutex mu;
     static std::unordered_set<const void*> opted;
     std::lock_guard<std::mutex> lk(mu);
     if (!opted.count((const void*)kern)) {
       cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+      if (e == cudaSuccess) e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemTileBytes);
       if (e != cudaSuccess) return e;
       opted.insert((const void*)kern);
     }
   }
+  if (d.gc != GC_CLUSTER) {
+    kern<<<d.grid, d.block, smem, s>>>(p);
+    return cudaPeekAtLastError();
+  }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(d.grid, 1, 1);
   cfg.blockDim = dim3(d.block, 1, 1);
-  cfg.dynamicSmemBytes = 0;
+  cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
@@ -235,13 +262,13 @@ inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& 
   return cudaLaunchKernelEx(&cfg, kern, p);
 }
 
-template <int DT, int OP, int U>
-cudaError_t launch_u(const LaunchDesc& d, const KParams& p, cudaStream_t s) {
+template <int DT, int OP, int U, int STAGE>
+cudaError_t launch_bc(const LaunchDesc& d, const KParams& p, cudaStream_t s) {
   switch (d.bc) {
-    case BC_SHFL: return launch_kernel(k_reduce<DT, OP, U, BC_SHFL>, d, p, s);
-    case BC_ATOMIC_WARP: return launch_kernel(k_reduce<DT, OP, U, BC_ATOMIC_WARP>, d, p, s);
-    case BC_ATOMIC_ALL: return launch_kernel(k_reduce<DT, OP, U, BC_ATOMIC_ALL>, d, p, s);
-    case BC_TREE: return launch_kernel(k_reduce<DT, OP, U, BC_TREE>, d, p, s);
+    case BC_SHFL: return launch_kernel(k_reduce<DT, OP, U, BC_SHFL, STAGE>, d, p, s);
+    case BC_ATOMIC_WARP: return launch_kernel(k_reduce<DT, OP, U, BC_ATOMIC_WARP, STAGE>, d, p, s);
+    case BC_ATOMIC_ALL: return launch_kernel(k_reduce<DT, OP, U, BC_ATOMIC_ALL, STAGE>, d, p, s);
+    case BC_TREE: return launch_kernel(k_reduce<DT, OP, U, BC_TREE, STAGE>, d, p, s);
   }
   return cudaErrorInvalidValue;
 }
@@ -250,12 +277,21 @@ template <int DT, int OP>
 cudaError_t launch_op(const LaunchDesc& d, cudaStream_t s) {
   const KParams p = make_params(d);
   cudaError_t e;
-  switch (d.unroll) {
-    case 1: e = launch_u<DT, OP, 1>(d, p, s); break;
-    case 2: e = launch_u<DT, OP, 2>(d, p, s); break;
-    case 4: e = launch_u<DT, OP, 4>(d, p, s); break;
-    case 8: e = launch_u<DT, OP, 8>(d, p, s); break;
-    default: return cudaErrorInvalidValue;
+  if (d.stage == STAGE_SMEM) {
+    switch (d.unroll) {
+      case 4: e = launch_bc<DT, OP, 4, STAGE_SMEM>(d, p, s); break;
+      case 8: e = launch_bc<DT, OP, 8, STAGE_SMEM>(d, p, s); break;
+      case 16: e = launch_bc<DT, OP, 16, STAGE_SMEM>(d, p, s); break;
+      default: return cudaErrorInvalidValue;
+    }
+  } else {
+    switch (d.unroll) {
+      case 1: e = launch_bc<DT, OP, 1, STAGE_REG>(d, p, s); break;
+      case 2: e = launch_bc<DT, OP, 2, STAGE_REG>(d, p, s); break;
+      case 4: e = launch_bc<DT, OP, 4, STAGE_REG>(d, p, s); break;
+      case 8: e = launch_bc<DT, OP, 8, STAGE_REG>(d, p, s); break;
+      default: return cudaErrorInvalidValue;
+    }
   }
   if (e != cudaSuccess || d.gc != GC_TWO_PASS) return e;
   k_combine<DT, OP><<<1, 1024, 0, s>>>(d.partials, (long long)d.grid, d.out, d.raw_out);

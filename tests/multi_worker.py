@@ -1,0 +1,65 @@
+"""Worker for tests/test_multi_gpu.py (run under torch.distributed.run, one rank
+per GPU, NCCL).  Every rank generates the SAME seeded global array, keeps its
+shard_range slice on its own GPU, calls reduce_multi, and checks the result
+against the oracle of the whole array (bit-exact for int32 and min/max; G1 for
+fp sums).  Uneven and empty shards are included.  Prints one JSON line per rank."""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+import oracle
+import synth
+import paper_conf_cgo_gonzalohghmh19_b200 as rb
+
+
+def main():
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist.init_process_group("nccl", device_id=dev)
+    rank, world = dist.get_rank(), dist.get_world_size()
+    comm = rb.Comm()
+    fails, count = [], 0
+    for dtype in ("int32", "float32", "float64"):
+        for n in (0, 1, world - 1 if world > 1 else 0, 1000, (1 << 20) + 7, (1 << 24) + 3):
+            x = synth.make(dtype, n, "int_full" if dtype == "int32" else "uniform_pm1", 7000 + n)
+            lo, hi = rb.shard_range(n, world, rank)
+            t = torch.empty(hi - lo + 1, dtype=getattr(torch, dtype), device=dev)[1:]
+            if hi > lo:
+                t.copy_(torch.from_numpy(x[lo:hi]))
+            for op in ("sum", "min", "max"):
+                for mode in ("fast", "deterministic"):
+                    out = rb.reduce_multi(t, op, comm, mode=mode)
+                    got = out.cpu().numpy()
+                    ref = oracle.reduce(x, op)
+                    count += 1
+                    if dtype == "int32" or op != "sum":
+                        bits = int(got.view(np.uint32 if dtype != "float64" else np.uint64)[0])
+                        if bits != ref.bits:
+                            fails.append((dtype, n, op, mode, bits, ref.bits))
+                    else:
+                        ok, msg = oracle.check_sum(float(got[0]), ref, x.dtype, max(n, 1))
+                        if not ok:
+                            fails.append((dtype, n, op, mode, msg))
+    # deterministic mode: identical bits on every call
+    x = synth.make("float32", (1 << 22) + 1, "uniform_pm1", 5)
+    lo, hi = rb.shard_range(x.size, world, rank)
+    t = torch.from_numpy(x[lo:hi]).to(dev)
+    vals = {int(rb.reduce_multi(t, "sum", comm, mode="deterministic").cpu().view(torch.int32).item())
+            for _ in range(20)}
+    torch.cuda.synchronize()
+    comm.destroy()
+    dist.destroy_process_group()
+    print(json.dumps({"rank": rank, "world": world, "checked": count, "fails": fails[:10],
+                      "deterministic_distinct": len(vals)}), flush=True)
+
+
+if __name__ == "__main__":
+    main()

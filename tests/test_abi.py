@@ -68,6 +68,8 @@ def test_invalid_arguments_rejected_without_cuda(args, why):
     dict(mode="deterministic", grid_combine=rb.GC_ATOMIC),
     dict(mode="deterministic", block_combine=rb.BC_SMEM_ATOMIC_ALL),
     dict(block=96, block_combine=rb.BC_SMEM_TREE),
+    dict(stage=3), dict(stage="smem", unroll=2), dict(stage="reg", unroll=16),
+    dict(stage="smem", block=1024, unroll=8), dict(grid_combine=4, grid=17),
 ])
 def test_invalid_options_rejected(kw):
     o = rb.make_opts(**kw)
@@ -117,6 +119,16 @@ def test_forced_overrides_respected():
                       grid_combine=rb.GC_LAST_BLOCK, block_combine=rb.BC_SMEM_TREE)
     assert (p["block"], p["unroll"], p["grid"], p["grid_combine"], p["block_combine"]) == (128, 8, 300, 3, 3)
     assert p["tiles"] == ((1 << 24) // 8 + 128 * 8 - 1) // (128 * 8)
+
+
+def test_query_plan_staging():
+    p = rb.query_plan("float32", "sum", 1 << 28, stage="smem", block=256, unroll=8)
+    assert p["stage"] == rb.STAGE_SMEM and p["tiles"] == (1 << 28) // (8 * 256 * 8)
+    p = rb.query_plan("float32", "sum", 1 << 28, stage="reg", unroll=4, block=256)
+    assert p["stage"] == rb.STAGE_REG
+    # fp64 min/max register staging is limited to 512 threads at unroll >= 2, smem staging is not
+    assert _ex(2, 2, 4096, 1000, 8192, rb.make_opts(block=1024, unroll=2, stage="reg")) == 1
+    assert rb.query_plan("float64", "max", 1 << 20, block=1024, unroll=4, stage="smem")["block"] == 1024
 
 
 def test_mode_default_roundtrip():

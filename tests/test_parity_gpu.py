@@ -113,8 +113,9 @@ def test_size_sweep(dtype):
 VARIANTS = []
 for bc in range(4):
     for gc in range(5):
-        for blk, u in ((32, 1), (128, 2), (256, 4), (512, 8), (1024, 1)):
-            VARIANTS.append(dict(block_combine=bc, grid_combine=gc, block=blk, unroll=u))
+        for blk, u, st in ((32, 1, 1), (128, 2, 1), (256, 4, 1), (512, 8, 1), (1024, 1, 1),
+                           (32, 16, 2), (128, 16, 2), (256, 8, 2), (1024, 4, 2)):
+            VARIANTS.append(dict(block_combine=bc, grid_combine=gc, block=blk, unroll=u, stage=st))
 
 
 @pytest.mark.parametrize("dtype", DTYPES)
@@ -124,7 +125,7 @@ def test_every_variant(dtype):
     x[[0, n // 2, n - 1]] = x[[n - 1, 0, n // 2]]
     t = to_device(x, 3)
     for v in VARIANTS:
-        if dtype == "float64" and v["block"] > 512 and v["unroll"] >= 2:
+        if dtype == "float64" and v["block"] > 512 and v["unroll"] >= 2 and v["stage"] == 1:
             continue
         got, plans = gpu_reduce_many([(t, op) for op in OPS], **v)
         for op, g, p in zip(OPS, got, plans):
@@ -154,8 +155,8 @@ def test_persistent_grids(grid):
     for dtype in DTYPES:
         x = synth.make(dtype, (1 << 20) + 5, _dist(dtype), grid)
         t = to_device(x, 1)
-        for gc in (1, 2, 3):
-            got, plans = gpu_reduce_many([(t, op) for op in OPS], grid=grid, grid_combine=gc)
+        for gc, st in ((1, 1), (2, 1), (3, 1), (1, 2), (2, 2)):
+            got, plans = gpu_reduce_many([(t, op) for op in OPS], grid=grid, grid_combine=gc, stage=st)
             for op, g, p in zip(OPS, got, plans):
                 check(x, op, g, p)
 

@@ -42,6 +42,9 @@ def candidates(dtype, op, mode, lb):
     if lb >= 12:
         for blk, u, gc in itertools.product((128, 256, 512), (1, 2, 4, 8), gcs):
             out.append(dict(block=blk, unroll=u, grid_combine=gc, block_combine=0, grid=0))
+        for blk, u, gc in itertools.product((128, 256, 512), (4, 8, 16), gcs):
+            if blk * u * 32 <= 128 * 1024:
+                out.append(dict(block=blk, unroll=u, grid_combine=gc, block_combine=0, grid=0, stage=2))
         for bc in (1, 2, 3):
             if mode == "deterministic" and bc in (1, 2):
                 continue
@@ -49,10 +52,15 @@ def candidates(dtype, op, mode, lb):
     if 10 <= lb <= 26:
         for blk, u, c in itertools.product((256, 512, 1024), (1, 2, 4), (4, 8, 16)):
             out.append(dict(block=blk, unroll=u, grid_combine=4, block_combine=0, grid=c))
+        for blk, u, c in itertools.product((256, 512), (8, 16), (8, 16)):
+            if blk * u * 32 <= 128 * 1024:
+                out.append(dict(block=blk, unroll=u, grid_combine=4, block_combine=0, grid=c, stage=2))
     if lb >= 24:
         for blk, g in itertools.product((256, 512), (148 * 2, 148 * 4, 148 * 8)):
             out.append(dict(block=blk, unroll=4, grid_combine=gcs[0], block_combine=0, grid=g))
-    return [c for c in out if c["block"] <= MAXBLK(dtype, op, c["unroll"])]
+    for c in out:
+        c.setdefault("stage", 1)
+    return [c for c in out if c["stage"] == 2 or c["block"] <= MAXBLK(dtype, op, c["unroll"])]
 
 
 def run(args):
@@ -121,7 +129,7 @@ def emit(paths, dst, tol=0.01):
     by = {}
     for r in res:
         by.setdefault((r["dtype"], r["op"], r["mode"], r["lb"]), []).append(r)
-    sig = lambda c: (c["block"], c["unroll"], c["grid_combine"], c["block_combine"], c["grid"])
+    sig = lambda c: (c["block"], c["unroll"], c["grid_combine"], c["block_combine"], c["grid"], c.get("stage", 1))
     rows = []
     groups = sorted(set(k[:3] for k in by))
     for dtype, op, mode in groups:
@@ -152,13 +160,14 @@ def emit(paths, dst, tol=0.01):
         "// (P:L681-L687, P:L691-L735, P:L739-L781).  GENERATED by tools/tune.py from",
         "// B200 measurements (device time per call, cold inputs); first match wins.",
         "//",
-        "// fields: dtype, op, mode, max_log2_bytes, block, unroll, grid_combine, block_combine, grid_cap",
-        "//   (grid_cap 0 = one block per tile)      // measured GB/s at the bucket that ended the row",
+        "// fields: dtype, op, mode, max_log2_bytes, block, unroll, grid_combine, block_combine, grid_cap, stage",
+        "//   (grid_cap 0 = one block per tile; stage 1 = registers, 2 = shared memory via cp.async)",
+        "//   trailing comment: measured GB/s at the bucket that ended the row",
         "static const DispatchEntry kDispatch[] = {",
     ]
     for r in rows:
-        lines.append("    {%d, %d, %d, %d, %d, %d, %d, %d, %d},  // %.1f GB/s" % r)
-    lines += ["    {-1, -1, -1, 63, 256, 4, -1, 0, 0},  // fallback", "};", ""]
+        lines.append("    {%d, %d, %d, %d, %d, %d, %d, %d, %d, %d},  // %.1f GB/s" % r)
+    lines += ["    {-1, -1, -1, 63, 256, 4, -1, 0, 0, 1},  // fallback", "};", ""]
     open(dst, "w").write("\n".join(lines))
     print(f"wrote {len(rows)} rows to {dst}")
 
