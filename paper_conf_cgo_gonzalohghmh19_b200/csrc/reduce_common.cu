@@ -1,4 +1,5 @@
 // reduce_common.cu -- dtype switch for the per-dtype kernel translation units.
+#include <cstdlib>
 #include "reduce_internal.h"
 
 namespace rb {
@@ -12,6 +13,14 @@ cudaError_t combine_f64(int, const void*, long long, void*, int, int, cudaStream
 cudaError_t init_i32(char*, char*, cudaStream_t);
 cudaError_t init_f32(char*, char*, cudaStream_t);
 cudaError_t init_f64(char*, char*, cudaStream_t);
+
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("REDUCE_NO_PDL");
+    return !(e && e[0] == '1');
+  }();
+  return on;
+}
 
 int grid_value_bytes(int dtype, int op) {
   if (dtype == 0) return 4;            // int32: uint32 / int32

@@ -48,6 +48,13 @@ __device__ __forceinline__ void lds_v8(const void* smem, uint32_t (&r)[8]) {
   r[0] = a.x; r[1] = a.y; r[2] = a.z; r[3] = a.w; r[4] = b.x; r[5] = b.y; r[6] = b.z; r[7] = b.w;
 }
 
+// Programmatic dependent launch (sm_90+): wait for the preceding grid of the
+// stream (a no-op when it was not launched programmatically), and let the next
+// programmatic grid be scheduled.
+constexpr unsigned kPdlTriggerWindow = 148u * 8u;  // ~ one full wave of resident blocks
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 // ------------------------------------------------------- fp primitives ---
 __device__ __forceinline__ float fmax_nan(float a, float b) {
   float r; asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r;

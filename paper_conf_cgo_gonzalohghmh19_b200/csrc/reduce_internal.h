@@ -60,6 +60,10 @@ cudaError_t launch_combine(int dtype, int op, const void* vals, long long count,
 // spaced kSlotBytes apart.
 cudaError_t launch_init_workspace(void* slots_base, void* tickets_base, cudaStream_t s);
 
+// Programmatic dependent launch of the library's kernels (default on; the
+// environment variable REDUCE_NO_PDL=1 turns it off, for A/B measurements).
+bool pdl_enabled();
+
 constexpr int kCombos = 9;  // 3 dtypes x 3 ops
 constexpr size_t kSlotRegionBytes = (size_t)kMaxSlots * kSlotBytes;
 

@@ -128,6 +128,12 @@ template <int DT, int OP, int U, int BC, int STAGE>
 __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(const KParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
+  // Programmatic dependent launch: this grid may be resident before the
+  // previous kernel of the stream has finished; nothing is read or written
+  // before the dependency resolves.  Blocks of the last wave allow the next
+  // kernel to be scheduled onto the SMs as this grid drains.
+  pdl_wait();
+  if (blockIdx.x + kPdlTriggerWindow >= gridDim.x) pdl_trigger();
   Acc a[T::NA];
 #pragma unroll
   for (int k = 0; k < T::NA; ++k) a[k] = T::ident();
@@ -195,6 +201,7 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(
 template <int DT, int OP>
 __global__ void __launch_bounds__(1024) k_combine(const void* vals, long long count, void* out, int raw_out) {
   using T = Tr<DT, OP>;
+  pdl_wait();
   typename T::Grid x = reduce_grid_values<T>((const typename T::Grid*)vals, count);
   if (threadIdx.x == 0) {
     if (raw_out) *(typename T::Grid*)out = x;
@@ -243,23 +250,43 @@ inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& 
       opted.insert((const void*)kern);
     }
   }
-  if (d.gc != GC_CLUSTER) {
-    kern<<<d.grid, d.block, smem, s>>>(p);
-    return cudaPeekAtLastError();
-  }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(d.grid, 1, 1);
   cfg.blockDim = dim3(d.block, 1, 1);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = d.grid;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
+  cudaLaunchAttribute attr[2];
+  int na = 0;
+  if (pdl_enabled()) {
+    attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+  }
+  if (d.gc == GC_CLUSTER) {
+    attr[na].id = cudaLaunchAttributeClusterDimension;
+    attr[na].val.clusterDim.x = d.grid;
+    attr[na].val.clusterDim.y = 1;
+    attr[na].val.clusterDim.z = 1;
+    ++na;
+  }
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = na;
   return cudaLaunchKernelEx(&cfg, kern, p);
+}
+
+// k_combine with the same programmatic-dependent-launch attribute.
+template <int DT, int OP>
+cudaError_t launch_combine_kernel(const void* vals, long long count, void* out, int raw_out, int block, cudaStream_t s) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(1, 1, 1);
+  cfg.blockDim = dim3(block, 1, 1);
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k_combine<DT, OP>, vals, count, out, raw_out);
 }
 
 template <int DT, int OP, int U, int STAGE>
@@ -294,8 +321,7 @@ cudaError_t launch_op(const LaunchDesc& d, cudaStream_t s) {
     }
   }
   if (e != cudaSuccess || d.gc != GC_TWO_PASS) return e;
-  k_combine<DT, OP><<<1, 1024, 0, s>>>(d.partials, (long long)d.grid, d.out, d.raw_out);
-  return cudaPeekAtLastError();
+  return launch_combine_kernel<DT, OP>(d.partials, (long long)d.grid, d.out, d.raw_out, 1024, s);
 }
 
 template <int DT>
@@ -311,12 +337,11 @@ cudaError_t launch_dt(const LaunchDesc& d, cudaStream_t s) {
 template <int DT>
 cudaError_t combine_dt(int op, const void* vals, long long count, void* out, int raw_out, int block, cudaStream_t s) {
   switch (op) {
-    case OP_SUM: k_combine<DT, OP_SUM><<<1, block, 0, s>>>(vals, count, out, raw_out); break;
-    case OP_MIN: k_combine<DT, OP_MIN><<<1, block, 0, s>>>(vals, count, out, raw_out); break;
-    case OP_MAX: k_combine<DT, OP_MAX><<<1, block, 0, s>>>(vals, count, out, raw_out); break;
-    default: return cudaErrorInvalidValue;
+    case OP_SUM: return launch_combine_kernel<DT, OP_SUM>(vals, count, out, raw_out, block, s);
+    case OP_MIN: return launch_combine_kernel<DT, OP_MIN>(vals, count, out, raw_out, block, s);
+    case OP_MAX: return launch_combine_kernel<DT, OP_MAX>(vals, count, out, raw_out, block, s);
   }
-  return cudaPeekAtLastError();
+  return cudaErrorInvalidValue;
 }
 
 template <int DT>

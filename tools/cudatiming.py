@@ -44,6 +44,9 @@ def disjoint_regions(pool, count: int, elems: int, align_elems: int = 64):
     if fit < 2:  # one region only: the caller uses this for arrays larger than L2
         r = pool[:elems]
         return [r] * count, [r] * count
-    count = max(1, min(count, fit // 2))
-    regs = [pool[i * stride:i * stride + elems] for i in range(2 * count)]
-    return regs[:count], regs[count:2 * count]
+    per = max(1, min(count, fit // 2))
+    regs = [pool[i * stride:i * stride + elems] for i in range(2 * per)]
+    warm, timed = regs[:per], regs[per:2 * per]
+    # too few disjoint regions: cycle through them (only done when the caller
+    # asks for more calls than fit, i.e. for regions far larger than L2)
+    return [warm[i % per] for i in range(count)], [timed[i % per] for i in range(count)]

@@ -90,7 +90,8 @@ def run(args):
             for lb in range(args.min_lb, args.max_lb + 1):
                 nbytes = 1 << lb
                 n = nbytes // ELEM[dtype]
-                R = max(5, min(100, (400 << 20) // nbytes))
+                # >= 20 calls per timed graph; regions repeat only when each is > 2x L2
+                R = max(20, min(100, (400 << 20) // nbytes)) if nbytes >= (256 << 20) else max(5, min(100, (400 << 20) // nbytes))
                 warm, timed = disjoint_regions(pool, R, n)
                 best = None
                 for c in candidates(dtype, op, mode, lb):
@@ -123,12 +124,13 @@ def emit(paths, dst, tol=0.01):
     candidates within `tol` of the fastest (timer noise) keep the previous size
     bucket's choice when it qualifies, so the table only changes where the
     measurements say it must."""
-    res = []
-    for p in paths:
-        res += [r for r in json.load(open(p)) if "us" in r]
     by = {}
-    for r in res:
-        by.setdefault((r["dtype"], r["op"], r["mode"], r["lb"]), []).append(r)
+    for p in paths:  # a later file replaces earlier measurements of the same bucket
+        cur = {}
+        for r in json.load(open(p)):
+            if "us" in r:
+                cur.setdefault((r["dtype"], r["op"], r["mode"], r["lb"]), []).append(r)
+        by.update(cur)
     sig = lambda c: (c["block"], c["unroll"], c["grid_combine"], c["block_combine"], c["grid"], c.get("stage", 1))
     rows = []
     groups = sorted(set(k[:3] for k in by))
