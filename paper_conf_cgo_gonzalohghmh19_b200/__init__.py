@@ -127,12 +127,17 @@ def _op(op) -> int:
     return OPS[op] if isinstance(op, str) else int(op)
 
 
+_TORCH_DT = {}
+
+
 def _torch_dtype_code(t) -> int:
-    import torch
-    m = {torch.int32: INT32, torch.float32: FLOAT32, torch.float64: FLOAT64}
-    if t.dtype not in m:
+    if not _TORCH_DT:
+        import torch
+        _TORCH_DT.update({torch.int32: INT32, torch.float32: FLOAT32, torch.float64: FLOAT64})
+    code = _TORCH_DT.get(t.dtype)
+    if code is None:
         raise TypeError(f"unsupported dtype {t.dtype} (int32, float32, float64)")
-    return m[t.dtype]
+    return code
 
 
 def _stream_handle(stream, device=None) -> int:
@@ -146,23 +151,25 @@ def _stream_handle(stream, device=None) -> int:
 
 def reduce_ptr(dtype: int, op, in_ptr: int, n: int, out_ptr: int, stream: int = 0, opts=None) -> None:
     """Raw-pointer form of reduce_ex (device pointers, stream handle)."""
-    st = lib.reduce_ex(int(dtype), _op(op), ctypes.c_void_p(in_ptr), n, ctypes.c_void_p(out_ptr),
-                       ctypes.c_void_p(stream), ctypes.byref(opts) if opts is not None else None)
-    _check(st, "reduce_ex")
+    st = lib.reduce_ex(dtype, OPS[op] if op.__class__ is str else op, in_ptr or None, n, out_ptr or None,
+                       stream or None, None if opts is None else ctypes.byref(opts))
+    if st:
+        raise ReduceError(st, "reduce_ex")
 
 
 def reduce(x, op="sum", out=None, stream=None, **opt_kw):
     """Reduce a contiguous CUDA tensor to a 1-element device tensor (async)."""
-    import torch
     if not x.is_cuda:
         raise ValueError("reduce() takes a CUDA tensor; use reduce_host() for host data")
     if not x.is_contiguous():
         raise ValueError("input must be contiguous")
     dt = _torch_dtype_code(x)
     if out is None:
+        import torch
         out = torch.empty(1, dtype=x.dtype, device=x.device)
     opts = make_opts(**opt_kw) if opt_kw else None
-    reduce_ptr(dt, op, x.data_ptr(), x.numel(), out.data_ptr(), _stream_handle(stream, x.device), opts)
+    s = stream.cuda_stream if stream is not None and not isinstance(stream, int) else _stream_handle(stream, x.device)
+    reduce_ptr(dt, op, x.data_ptr(), x.numel(), out.data_ptr(), s, opts)
     return out
 
 

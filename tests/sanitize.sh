@@ -1,0 +1,30 @@
+#!/usr/bin/env bash
+# compute-sanitizer pass over every kernel family (SURVEY section 4 "Sanitizers"):
+# memcheck, racecheck, synccheck and initcheck on small ragged sizes, every grid
+# combine (DIRECT, ATOMIC, TWO_PASS, LAST_BLOCK, CLUSTER), both staging modes.
+# Usage (GPU box): bash tests/sanitize.sh  -> exit 0 iff every tool reports 0 errors.
+set -u
+cd "$(dirname "$0")/.."
+CS=${CS:-/usr/local/cuda/bin/compute-sanitizer}
+cat > /tmp/rb_sanitize_case.py <<'PY'
+import sys, numpy as np, torch
+sys.path.insert(0, ".")
+import paper_conf_cgo_gonzalohghmh19_b200 as rb
+for dt in (torch.int32, torch.float32, torch.float64):
+    for n in (1, 33, 4097, (1 << 20) + 3):
+        x = torch.arange(n + 3, device="cuda").to(dt)[3:]
+        for op in ("sum", "min", "max"):
+            for kw in (dict(), dict(mode="deterministic"), dict(grid_combine=3), dict(grid_combine=4, grid=8),
+                       dict(stage="smem", unroll=8, block=256), dict(block_combine=1), dict(block_combine=3, block=128)):
+                rb.reduce(x, op, **kw)
+torch.cuda.synchronize()
+print("ok")
+PY
+rc=0
+for tool in memcheck racecheck synccheck initcheck; do
+  out=$($CS --tool $tool --error-exitcode 9 python /tmp/rb_sanitize_case.py 2>&1)
+  code=$?
+  echo "== $tool: exit $code; $(echo "$out" | grep -E 'ERROR SUMMARY|^ok' | tr '\n' ' ')"
+  [ $code -ne 0 ] && { echo "$out" | tail -30; rc=1; }
+done
+exit $rc
