@@ -55,6 +55,12 @@ constexpr unsigned kPdlTriggerWindow = 148u * 8u;  // ~ one full wave of residen
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
+// Split cluster barrier (all threads of every CTA of the cluster take part).
+__device__ __forceinline__ void cluster_arrive_relaxed() {
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void cluster_wait() { asm volatile("barrier.cluster.wait.aligned;" ::: "memory"); }
+
 // ------------------------------------------------------- fp primitives ---
 __device__ __forceinline__ float fmax_nan(float a, float b) {
   float r; asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b)); return r;

@@ -59,12 +59,15 @@ __device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& 
     return;
   }
   if (p.gc == GC_CLUSTER) {
-    // CTA partials meet in CTA 0's shared memory over DSMEM; one cluster
-    // barrier (release/acquire) orders the remote stores before CTA 0 reads.
+    // CTA partials meet in CTA 0's shared memory over DSMEM.  The first
+    // cluster-barrier phase (arrived at kernel start, see k_reduce) guarantees
+    // CTA 0 has started before anyone writes into its shared memory; the
+    // second (release/acquire) orders the remote stores before CTA 0 reads.
     namespace cg = cooperative_groups;
     __shared__ Grid cl_vals[16];
     cg::cluster_group cluster = cg::this_cluster();
     const unsigned r = cluster.block_rank();
+    cluster_wait();
     if (threadIdx.x == 0) cluster.map_shared_rank(&cl_vals[0], 0)[r] = g;
     cluster.sync();
     if (r == 0 && threadIdx.x < 32) {
@@ -134,6 +137,7 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(
   // kernel to be scheduled onto the SMs as this grid drains.
   pdl_wait();
   if (blockIdx.x + kPdlTriggerWindow >= gridDim.x) pdl_trigger();
+  if (p.gc == GC_CLUSTER) cluster_arrive_relaxed();  // phase 1: "this CTA has started"
   Acc a[T::NA];
 #pragma unroll
   for (int k = 0; k < T::NA; ++k) a[k] = T::ident();

@@ -22,7 +22,8 @@ print("ok")
 PY
 rc=0
 for tool in memcheck racecheck synccheck initcheck; do
-  out=$($CS --tool $tool --error-exitcode 9 python /tmp/rb_sanitize_case.py 2>&1)
+  extra=""; [ $tool = racecheck ] && extra="--racecheck-report all"
+  out=$($CS --tool $tool $extra --error-exitcode 9 python /tmp/rb_sanitize_case.py 2>&1)
   code=$?
   echo "== $tool: exit $code; $(echo "$out" | grep -E 'ERROR SUMMARY|^ok' | tr '\n' ' ')"
   [ $code -ne 0 ] && { echo "$out" | tail -30; rc=1; }
