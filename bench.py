@@ -383,6 +383,27 @@ def main():
                 latency.append({"dtype": dt, "n": m, "graph_us": round(g_us, 3), "stream_b2b_us": round(s_us, 3),
                                 "host_wall_us": round(statistics.median(walls) * 1e6, 2)})
 
+    # ---- many small arrays in one launch: batched rows of
+    # the resident input, device time per call (graph), against one reduce()
+    # per array (the sweep's per-call time at that length).
+    batched = None
+    if not args.no_sweep and world == 1:
+        batched = []
+        per_call = {e["n"]: e["us"] for e in sweep}
+        for cols in (64, 1024, 16384):
+            rows = (256 << 20) // (4 * cols)
+            xv = x[: rows * cols].view(rows, cols)
+            ob = torch.empty(rows, dtype=torch.float32, device=dev)
+
+            def launch_b(t, ob=ob, xv=xv):
+                rb.reduce_batched(xv, "sum", out=ob, stream=stream)
+            sec = time_calls(launch_b, [xv] * 3, [xv] * 10, stream, repeats=2)
+            one = per_call.get(cols)
+            batched.append({"rows": rows, "cols": cols, "us": round(sec * 1e6, 2),
+                            "GBps": round(rows * cols * 4 / sec / 1e9, 1),
+                            "arrays_per_s": round(rows / sec, 1),
+                            "speedup_vs_one_reduce_per_array": None if one is None else round(one * 1e-6 * rows / sec, 1)})
+
     # ---- CPU baseline: the oracle on the host cores (rank 0, N = 1)
     cpu = None
     if not args.no_cpu and world == 1 and rank == 0:
@@ -425,6 +446,7 @@ def main():
         if sweep is not None:
             line["sweep"] = sweep
             line["small_array_latency"] = latency
+            line["batched"] = batched
         if ncu_s is not None:
             line["ncu"] = {k: ncu_s[k] for k in ("source", "dram_pct_of_peak", "duration_us") if k in ncu_s}
         print(json.dumps(line), flush=True)

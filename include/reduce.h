@@ -123,6 +123,10 @@ typedef struct {
                          (register staging) or 4,8,16 (shared-memory staging) */
   int grid;           /* 0 = auto (one block per tile, capped), else max blocks;
                          for REDUCE_GC_CLUSTER: the cluster size, 1..16 (0 = 16) */
+  int seg_group;      /* reduce_segmented / reduce_batched only: 0 = auto (one warp per
+                         segment for uniform segments <= 4096 elements and for
+                         offset arrays, else one block), 1 = one warp per
+                         segment, 2 = one block per segment */
   int stage;          /* 0 = auto; REDUCE_STAGE_REG: 256-bit loads straight into
                          registers; REDUCE_STAGE_SMEM: cp.async 16-byte copies into a
                          shared-memory tile (block*unroll*32 <= 128 KiB), then shared
@@ -172,6 +176,22 @@ int reduce_get_mode(void);
  * return.  Uses a library-owned device staging buffer (2 x chunk bytes). */
 int reduce_host(int dtype, int op, const void* host_in, size_t n, void* host_out,
                 reduce_stream_t stream, const reduce_opts_t* opts);
+
+/* ---- many arrays in one launch ---------------------------
+ * reduce_segmented: out[i] = reduce(in[offsets[i] .. offsets[i+1])) for every
+ * i < num_segments.  `offsets` is a DEVICE array of num_segments + 1 int64
+ * element offsets (non-decreasing; a decreasing pair is treated as an empty
+ * segment, which yields the identity); `out` is a DEVICE array of
+ * num_segments elements of dtype.  One warp or one block per segment (the
+ * paper's small-array versions assign one warp / block per partition with no
+ * global atomics): one launch, no atomics, deterministic.
+ * Segment starts may have any element alignment.  Options used: block,
+ * seg_group.  reduce_batched is the uniform case: num_segments rows of seg_len
+ * contiguous elements (row i at in + i*seg_len), no offsets array. */
+int reduce_segmented(int dtype, int op, const void* in, const int64_t* offsets, size_t num_segments, void* out,
+                     reduce_stream_t stream, const reduce_opts_t* opts);
+int reduce_batched(int dtype, int op, const void* in, size_t seg_len, size_t num_segments, void* out,
+                   reduce_stream_t stream, const reduce_opts_t* opts);
 
 /* ---- sharded mode over NCCL (one process per GPU) -------------------------
  * reduce_multi: every rank of `comm` calls it with its own local shard

@@ -34,7 +34,7 @@ ABI_SYMBOLS = (
     "reduce_get_mode", "reduce_host", "reduce_multi", "reduce_multi_ex",
     "reduce_comm_unique_id_bytes", "reduce_comm_get_unique_id", "reduce_comm_init",
     "reduce_comm_destroy", "reduce_status_string", "reduce_last_error", "reduce_version",
-    "reduce_shutdown",
+    "reduce_shutdown", "reduce_segmented", "reduce_batched",
 )
 
 
@@ -48,7 +48,7 @@ class ReduceError(RuntimeError):
 class reduce_opts_t(ctypes.Structure):
     _fields_ = [("mode", ctypes.c_int), ("grid_combine", ctypes.c_int), ("block_combine", ctypes.c_int),
                 ("block", ctypes.c_int), ("unroll", ctypes.c_int), ("grid", ctypes.c_int),
-                ("stage", ctypes.c_int)]
+                ("seg_group", ctypes.c_int), ("stage", ctypes.c_int)]
 
 
 class reduce_plan_t(ctypes.Structure):
@@ -88,6 +88,8 @@ def _load() -> ctypes.CDLL:
         "reduce_last_error": (ctypes.c_char_p, []),
         "reduce_version": (i, []),
         "reduce_shutdown": (None, []),
+        "reduce_segmented": (i, [i, i, vp, vp, sz, vp, vp, opts_p]),
+        "reduce_batched": (i, [i, i, vp, sz, sz, vp, vp, opts_p]),
     }
     for name, (res, args) in sigs.items():
         f = getattr(L, name)
@@ -112,7 +114,7 @@ def _check(status: int, where: str) -> None:
         raise ReduceError(status, where)
 
 
-def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=0, grid=0, stage=0):
+def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=0, grid=0, stage=0, seg_group=0):
     if isinstance(mode, str):
         mode = {"fast": MODE_FAST, "deterministic": MODE_DETERMINISTIC}[mode]
     if isinstance(stage, str):
@@ -120,7 +122,7 @@ def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=
     return reduce_opts_t(-1 if mode is None else int(mode),
                          -1 if grid_combine is None else int(grid_combine),
                          -1 if block_combine is None else int(block_combine),
-                         int(block), int(unroll), int(grid), int(stage))
+                         int(block), int(unroll), int(grid), int(seg_group), int(stage))
 
 
 def _op(op) -> int:
@@ -170,6 +172,40 @@ def reduce(x, op="sum", out=None, stream=None, **opt_kw):
     opts = make_opts(**opt_kw) if opt_kw else None
     s = stream.cuda_stream if stream is not None and not isinstance(stream, int) else _stream_handle(stream, x.device)
     reduce_ptr(dt, op, x.data_ptr(), x.numel(), out.data_ptr(), s, opts)
+    return out
+
+
+def reduce_segmented(x, offsets, op="sum", out=None, stream=None, **opt_kw):
+    """out[i] = reduce(x[offsets[i]:offsets[i+1]]) for a CUDA tensor x and a CUDA
+    int64 tensor offsets of num_segments + 1 entries (one launch, deterministic)."""
+    import torch
+    dt = _torch_dtype_code(x)
+    nseg = offsets.numel() - 1
+    if offsets.dtype != torch.int64 or not offsets.is_cuda or not offsets.is_contiguous():
+        raise ValueError("offsets must be a contiguous CUDA int64 tensor")
+    if out is None:
+        out = torch.empty(max(nseg, 0), dtype=x.dtype, device=x.device)
+    opts = make_opts(**opt_kw) if opt_kw else None
+    st = lib.reduce_segmented(dt, _op(op), x.data_ptr() or None, offsets.data_ptr() or None, max(nseg, 0),
+                              out.data_ptr() or None, _stream_handle(stream, x.device),
+                              ctypes.byref(opts) if opts is not None else None)
+    _check(st, "reduce_segmented")
+    return out
+
+
+def reduce_batched(x, op="sum", out=None, stream=None, **opt_kw):
+    """Row reductions of a contiguous 2-D CUDA tensor (rows x seg_len) in one launch."""
+    import torch
+    dt = _torch_dtype_code(x)
+    if x.dim() != 2 or not x.is_contiguous():
+        raise ValueError("reduce_batched takes a contiguous 2-D tensor")
+    rows, cols = x.shape
+    if out is None:
+        out = torch.empty(rows, dtype=x.dtype, device=x.device)
+    opts = make_opts(**opt_kw) if opt_kw else None
+    st = lib.reduce_batched(dt, _op(op), x.data_ptr() or None, cols, rows, out.data_ptr() or None,
+                            _stream_handle(stream, x.device), ctypes.byref(opts) if opts is not None else None)
+    _check(st, "reduce_batched")
     return out
 
 

@@ -59,7 +59,8 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   if (n > (size_t)1 << 46) return fail(REDUCE_ERR_INVALID_ARG, "n too large");
 
   reduce_opts_t o;
-  o.mode = -1; o.grid_combine = -1; o.block_combine = -1; o.block = 0; o.unroll = 0; o.grid = 0; o.stage = 0;
+  o.mode = -1; o.grid_combine = -1; o.block_combine = -1; o.block = 0; o.unroll = 0; o.grid = 0; o.seg_group = 0;
+  o.stage = 0;
   if (opts) o = *opts;
   int mode = o.mode < 0 ? g_mode.load() : o.mode;
   if (mode != REDUCE_MODE_FAST && mode != REDUCE_MODE_DETERMINISTIC)
@@ -305,6 +306,51 @@ int reduce_ex(int dtype, int op, const void* in, size_t n, void* out, reduce_str
   st = get_workspace((cudaStream_t)stream, partials_needed(P), &ws);
   if (st != REDUCE_OK) return st;
   return launch_plan(&P, ws, out, (cudaStream_t)stream);
+}
+
+static int segmented_common(int dtype, int op, const void* in, const int64_t* offsets, size_t seg_len,
+                            size_t nseg, void* out, reduce_stream_t stream, const reduce_opts_t* opts) {
+  if (dtype < 0 || dtype > 2) return fail(REDUCE_ERR_INVALID_ARG, "dtype must be REDUCE_INT32/FLOAT32/FLOAT64");
+  if (op < 0 || op > 2) return fail(REDUCE_ERR_INVALID_ARG, "op must be REDUCE_SUM/MIN/MAX");
+  const int s = dtype == REDUCE_FLOAT64 ? 8 : 4;
+  if (nseg == 0) return REDUCE_OK;
+  if (out == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "out is NULL");
+  if (((uintptr_t)out % (uintptr_t)s) != 0) return fail(REDUCE_ERR_INVALID_ARG, "out is not aligned to the element size");
+  const bool uniform = offsets == nullptr;
+  if (in == nullptr && (!uniform || seg_len > 0)) return fail(REDUCE_ERR_INVALID_ARG, "in is NULL");
+  if (in && ((uintptr_t)in % (uintptr_t)s) != 0) return fail(REDUCE_ERR_INVALID_ARG, "in is not aligned to the element size");
+  if (nseg > 0x7FFFFFFFull * 32ull) return fail(REDUCE_ERR_INVALID_ARG, "too many segments");
+  int block = 256, group = 0;
+  if (opts) {
+    if (opts->block != 0 && (opts->block < 32 || opts->block > 1024 || opts->block % 32 != 0))
+      return fail(REDUCE_ERR_INVALID_ARG, "block must be 0 or a multiple of 32 in [32, 1024]");
+    if (opts->seg_group < 0 || opts->seg_group > 2) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0, 1 or 2");
+    if (opts->block) block = opts->block;
+    group = opts->seg_group;
+  }
+  const bool warp = group == 1 || (group == 0 && (!uniform || seg_len <= 4096));
+  if (!warp && nseg > 0x7FFFFFFFull) return fail(REDUCE_ERR_INVALID_ARG, "too many segments for one block each");
+  SegParams p;
+  p.in = (const char*)in;
+  p.offsets = (const long long*)offsets;
+  p.seg_len = (long long)seg_len;
+  p.nseg = (long long)nseg;
+  p.out = out;
+  p.raw_out = 0;
+  cudaError_t e = launch_segmented(dtype, op, p, warp, block, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "segmented reduction launch");
+  return REDUCE_OK;
+}
+
+int reduce_segmented(int dtype, int op, const void* in, const int64_t* offsets, size_t num_segments, void* out,
+                     reduce_stream_t stream, const reduce_opts_t* opts) {
+  if (offsets == nullptr && num_segments > 0) return fail(REDUCE_ERR_INVALID_ARG, "offsets is NULL");
+  return segmented_common(dtype, op, in, offsets, 0, num_segments, out, stream, opts);
+}
+
+int reduce_batched(int dtype, int op, const void* in, size_t seg_len, size_t num_segments, void* out,
+                   reduce_stream_t stream, const reduce_opts_t* opts) {
+  return segmented_common(dtype, op, in, nullptr, seg_len, num_segments, out, stream, opts);
 }
 
 int reduce(int dtype, int op, const void* in, size_t n, void* out, reduce_stream_t stream) {

@@ -1,6 +1,7 @@
 // reduce_i32.cu -- instantiates the reduction kernels for one dtype (split per
 // dtype so the 48 kernel instantiations per dtype compile in parallel).
 #include "reduce_kernels.cuh"
+#include "reduce_segmented.cuh"
 
 namespace rb {
 cudaError_t launch_reduce_i32(const LaunchDesc& d, cudaStream_t s) { return launch_dt<DT_I32>(d, s); }
@@ -8,4 +9,7 @@ cudaError_t combine_i32(int op, const void* v, long long c, void* out, int raw, 
   return combine_dt<DT_I32>(op, v, c, out, raw, block, s);
 }
 cudaError_t init_i32(char* slots, char* tickets, cudaStream_t s) { return init_dt<DT_I32>(slots, tickets, s); }
+cudaError_t segmented_i32(int op, const SegParams& p, bool warp_per_seg, int block, cudaStream_t s) {
+  return launch_segmented_dt<DT_I32>(op, p, warp_per_seg, block, s);
+}
 }  // namespace rb

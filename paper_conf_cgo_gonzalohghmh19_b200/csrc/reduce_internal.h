@@ -45,6 +45,17 @@ struct LaunchDesc {
   void* partials;                // Grid[grid] (GC_TWO_PASS / GC_LAST_BLOCK)
 };
 
+// One segmented / batched launch, see reduce_segmented.cuh.
+struct SegParams {
+  const char* in;
+  const long long* offsets;  // device, nseg + 1 entries; NULL: uniform segments of seg_len
+  long long seg_len;
+  long long nseg;
+  void* out;                 // T[nseg] (finalised) or Grid[nseg] (raw)
+  int raw_out;
+};
+cudaError_t launch_segmented(int dtype, int op, const SegParams& p, bool warp_per_seg, int block, cudaStream_t s);
+
 // Size in bytes of the Grid (cross-block) type of (dtype, op).
 int grid_value_bytes(int dtype, int op);
 

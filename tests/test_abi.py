@@ -131,6 +131,17 @@ def test_query_plan_staging():
     assert rb.query_plan("float64", "max", 1 << 20, block=1024, unroll=4, stage="smem")["block"] == 1024
 
 
+def test_segmented_argument_validation():
+    L = rb.lib
+    o = rb.make_opts(seg_group=3)
+    assert L.reduce_segmented(1, 0, 4096, None, 10, 8192, None, None) == 1        # offsets NULL
+    assert L.reduce_segmented(1, 0, 4096, 4096, 10, None, None, None) == 1        # out NULL
+    assert L.reduce_segmented(5, 0, 4096, 4096, 10, 8192, None, None) == 1        # dtype
+    assert L.reduce_batched(1, 0, 4096, 10, 10, 8192, None, ctypes.byref(o)) == 1  # seg_group
+    assert L.reduce_batched(2, 0, 4100, 10, 10, 8192, None, None) == 1            # misaligned fp64
+    assert L.reduce_batched(1, 0, None, 10, 0, None, None, None) == 0             # no segments: no-op
+
+
 def test_mode_default_roundtrip():
     old = rb.get_mode()
     rb.set_mode("deterministic")
