@@ -123,10 +123,10 @@ typedef struct {
                          (register staging) or 4,8,16 (shared-memory staging) */
   int grid;           /* 0 = auto (one block per tile, capped), else max blocks;
                          for REDUCE_GC_CLUSTER: the cluster size, 1..16 (0 = 16) */
-  int seg_group;      /* reduce_segmented / reduce_batched only: 0 = auto (one warp per
-                         segment for uniform segments <= 4096 elements and for
-                         offset arrays, else one block), 1 = one warp per
-                         segment, 2 = one block per segment */
+  int seg_group;      /* reduce_segmented / reduce_batched only: 0 = auto (8 lanes per
+                         segment for uniform segments <= 128 elements, one warp for
+                         <= 4096 and for offset arrays, else one block), 1 = one
+                         warp per segment, 2 = one block per segment, 3 = 8 lanes */
   int stage;          /* 0 = auto; REDUCE_STAGE_REG: 256-bit loads straight into
                          registers; REDUCE_STAGE_SMEM: cp.async 16-byte copies into a
                          shared-memory tile (block*unroll*32 <= 128 KiB), then shared

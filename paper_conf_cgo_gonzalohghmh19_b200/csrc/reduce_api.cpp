@@ -319,17 +319,16 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   const bool uniform = offsets == nullptr;
   if (in == nullptr && (!uniform || seg_len > 0)) return fail(REDUCE_ERR_INVALID_ARG, "in is NULL");
   if (in && ((uintptr_t)in % (uintptr_t)s) != 0) return fail(REDUCE_ERR_INVALID_ARG, "in is not aligned to the element size");
-  if (nseg > 0x7FFFFFFFull * 32ull) return fail(REDUCE_ERR_INVALID_ARG, "too many segments");
   int block = 256, group = 0;
   if (opts) {
     if (opts->block != 0 && (opts->block < 32 || opts->block > 1024 || opts->block % 32 != 0))
       return fail(REDUCE_ERR_INVALID_ARG, "block must be 0 or a multiple of 32 in [32, 1024]");
-    if (opts->seg_group < 0 || opts->seg_group > 2) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0, 1 or 2");
+    if (opts->seg_group < 0 || opts->seg_group > 3) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0..3");
     if (opts->block) block = opts->block;
     group = opts->seg_group;
   }
-  const bool warp = group == 1 || (group == 0 && (!uniform || seg_len <= 4096));
-  if (!warp && nseg > 0x7FFFFFFFull) return fail(REDUCE_ERR_INVALID_ARG, "too many segments for one block each");
+  if (group == 0) group = !uniform ? 1 : (seg_len <= 128 ? 3 : (seg_len <= 4096 ? 1 : 2));
+  const int lanes = group == 1 ? 32 : (group == 3 ? 8 : 0);
   SegParams p;
   p.in = (const char*)in;
   p.offsets = (const long long*)offsets;
@@ -337,7 +336,7 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   p.nseg = (long long)nseg;
   p.out = out;
   p.raw_out = 0;
-  cudaError_t e = launch_segmented(dtype, op, p, warp, block, (cudaStream_t)stream);
+  cudaError_t e = launch_segmented(dtype, op, p, lanes, block, (cudaStream_t)stream);
   if (e != cudaSuccess) return cuda_fail(e, "segmented reduction launch");
   return REDUCE_OK;
 }

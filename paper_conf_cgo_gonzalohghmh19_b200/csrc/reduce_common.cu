@@ -13,15 +13,15 @@ cudaError_t combine_f64(int, const void*, long long, void*, int, int, cudaStream
 cudaError_t init_i32(char*, char*, cudaStream_t);
 cudaError_t init_f32(char*, char*, cudaStream_t);
 cudaError_t init_f64(char*, char*, cudaStream_t);
-cudaError_t segmented_i32(int, const SegParams&, bool, int, cudaStream_t);
-cudaError_t segmented_f32(int, const SegParams&, bool, int, cudaStream_t);
-cudaError_t segmented_f64(int, const SegParams&, bool, int, cudaStream_t);
+cudaError_t segmented_i32(int, const SegParams&, int, int, cudaStream_t);
+cudaError_t segmented_f32(int, const SegParams&, int, int, cudaStream_t);
+cudaError_t segmented_f64(int, const SegParams&, int, int, cudaStream_t);
 
-cudaError_t launch_segmented(int dtype, int op, const SegParams& p, bool warp_per_seg, int block, cudaStream_t s) {
+cudaError_t launch_segmented(int dtype, int op, const SegParams& p, int group, int block, cudaStream_t s) {
   switch (dtype) {
-    case 0: return segmented_i32(op, p, warp_per_seg, block, s);
-    case 1: return segmented_f32(op, p, warp_per_seg, block, s);
-    case 2: return segmented_f64(op, p, warp_per_seg, block, s);
+    case 0: return segmented_i32(op, p, group, block, s);
+    case 1: return segmented_f32(op, p, group, block, s);
+    case 2: return segmented_f64(op, p, group, block, s);
   }
   return cudaErrorInvalidValue;
 }

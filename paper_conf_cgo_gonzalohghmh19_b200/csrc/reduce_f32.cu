@@ -9,7 +9,7 @@ cudaError_t combine_f32(int op, const void* v, long long c, void* out, int raw, 
   return combine_dt<DT_F32>(op, v, c, out, raw, block, s);
 }
 cudaError_t init_f32(char* slots, char* tickets, cudaStream_t s) { return init_dt<DT_F32>(slots, tickets, s); }
-cudaError_t segmented_f32(int op, const SegParams& p, bool warp_per_seg, int block, cudaStream_t s) {
-  return launch_segmented_dt<DT_F32>(op, p, warp_per_seg, block, s);
+cudaError_t segmented_f32(int op, const SegParams& p, int group, int block, cudaStream_t s) {
+  return launch_segmented_dt<DT_F32>(op, p, group, block, s);
 }
 }  // namespace rb

@@ -54,7 +54,8 @@ struct SegParams {
   void* out;                 // T[nseg] (finalised) or Grid[nseg] (raw)
   int raw_out;
 };
-cudaError_t launch_segmented(int dtype, int op, const SegParams& p, bool warp_per_seg, int block, cudaStream_t s);
+// group: lanes per segment (8 or 32) or 0 = one block per segment.
+cudaError_t launch_segmented(int dtype, int op, const SegParams& p, int group, int block, cudaStream_t s);
 
 // Size in bytes of the Grid (cross-block) type of (dtype, op).
 int grid_value_bytes(int dtype, int op);

@@ -55,54 +55,82 @@ __device__ __forceinline__ void seg_store(const SegParams& p, long long seg, typ
   else T::finalize(g, (char*)p.out + seg * (long long)sizeof(typename T::Elem));
 }
 
-template <int DT, int OP, bool kWarpPerSeg>
+// kGroup = 8 or 32: that many lanes per segment (4 or 1 segments per warp in
+// flight); kGroup = 0: one block per segment.  The grid is persistent (a few
+// blocks per SM) and groups stride over the segments, so millions of tiny
+// segments do not pay one CTA launch each.
+template <int DT, int OP, int kGroup>
 __global__ void __launch_bounds__(1024) k_segmented(const SegParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
   pdl_wait();
-  if (blockIdx.x + kPdlTriggerWindow >= gridDim.x) pdl_trigger();
+  pdl_trigger();  // persistent grid: every block is resident from the start
   const int lane = threadIdx.x & 31;
-  long long seg;
+  long long first, step;
   int lid, lanes;
-  if constexpr (kWarpPerSeg) {
-    seg = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-    lid = lane;
-    lanes = 32;
-    if (seg >= p.nseg) return;  // whole warp leaves together
+  if constexpr (kGroup > 0) {
+    const long long groups_per_block = blockDim.x / kGroup;
+    first = (long long)blockIdx.x * groups_per_block + threadIdx.x / kGroup;
+    step = (long long)gridDim.x * groups_per_block;
+    lid = threadIdx.x % kGroup;
+    lanes = kGroup;
   } else {
-    seg = blockIdx.x;
+    first = blockIdx.x;
+    step = gridDim.x;
     lid = threadIdx.x;
     lanes = blockDim.x;
   }
-  long long lo, hi;
-  if (p.offsets) {
-    lo = __ldg(p.offsets + seg);
-    hi = __ldg(p.offsets + seg + 1);
-  } else {
-    lo = seg * p.seg_len;
-    hi = lo + p.seg_len;
-  }
-  Acc a[T::NA];
+  // all groups of a warp (all threads of a block) run the same number of
+  // iterations -- the shuffles / barriers need every lane -- and a group past
+  // the last segment folds nothing
+  const long long base = kGroup > 0 ? first - lane / kGroup : first;
+  const long long iters = base < p.nseg ? (p.nseg - base + step - 1) / step : 0;
+  for (long long it = 0; it < iters; ++it) {
+    const long long seg = first + it * step;
+    const bool live = seg < p.nseg;
+    long long lo = 0, hi = 0;
+    if (live) {
+      if (p.offsets) {
+        lo = __ldg(p.offsets + seg);
+        hi = __ldg(p.offsets + seg + 1);
+      } else {
+        lo = seg * p.seg_len;
+        hi = lo + p.seg_len;
+      }
+    }
+    Acc a[T::NA];
 #pragma unroll
-  for (int k = 0; k < T::NA; ++k) a[k] = T::ident();
-  uint32_t aux = 0;
-  fold_range<T, 4>(a, aux, p.in, lo, hi, lid, lanes);
-  const Acc v = thread_result<T>(a, aux);
-  if constexpr (kWarpPerSeg) {
-    const Acc w = T::warp(v);
-    if (lane == 0) seg_store<T>(p, seg, T::to_grid(w));
-  } else {
-    const typename T::Grid g = block_combine<T, BC_SHFL>(v);
-    if (threadIdx.x == 0) seg_store<T>(p, seg, g);
+    for (int k = 0; k < T::NA; ++k) a[k] = T::ident();
+    uint32_t aux = 0;
+    fold_range<T, 4>(a, aux, p.in, lo, hi, lid, lanes);
+    const Acc v = thread_result<T>(a, aux);
+    if constexpr (kGroup == 32) {
+      const Acc w = T::warp(v);
+      if (lane == 0 && live) seg_store<T>(p, seg, T::to_grid(w));
+    } else if constexpr (kGroup > 0) {
+      Acc w = v;
+#pragma unroll
+      for (int o = kGroup / 2; o > 0; o >>= 1) w = T::comb(w, __shfl_xor_sync(0xffffffffu, w, o));
+      if (lid == 0 && live) seg_store<T>(p, seg, T::to_grid(w));
+    } else {
+      const typename T::Grid g = block_combine<T, BC_SHFL>(v);
+      if (threadIdx.x == 0 && live) seg_store<T>(p, seg, g);
+      __syncthreads();  // block_combine's shared scratch is reused next iteration
+    }
   }
 }
 
 template <int DT, int OP>
-cudaError_t launch_segmented_op(const SegParams& p, bool warp_per_seg, int block, cudaStream_t s) {
+cudaError_t launch_segmented_op(const SegParams& p, int group, int block, cudaStream_t s) {
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long per_block = group > 0 ? block / group : 1;
+  long long grid = (p.nseg + per_block - 1) / per_block;
+  const long long cap = (long long)sms * (2048 / block);  // one full wave
+  if (grid > cap) grid = cap;
+  if (grid < 1) grid = 1;
   cudaLaunchConfig_t cfg = {};
-  const long long per_block = warp_per_seg ? block / 32 : 1;
-  const long long grid = (p.nseg + per_block - 1) / per_block;
-  if (grid > 0x7FFFFFFFll) return cudaErrorInvalidValue;
   cfg.gridDim = dim3((unsigned)grid, 1, 1);
   cfg.blockDim = dim3(block, 1, 1);
   cfg.stream = s;
@@ -111,16 +139,17 @@ cudaError_t launch_segmented_op(const SegParams& p, bool warp_per_seg, int block
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = pdl_enabled() ? 1 : 0;
-  if (warp_per_seg) return cudaLaunchKernelEx(&cfg, k_segmented<DT, OP, true>, p);
-  return cudaLaunchKernelEx(&cfg, k_segmented<DT, OP, false>, p);
+  if (group == 8) return cudaLaunchKernelEx(&cfg, k_segmented<DT, OP, 8>, p);
+  if (group == 32) return cudaLaunchKernelEx(&cfg, k_segmented<DT, OP, 32>, p);
+  return cudaLaunchKernelEx(&cfg, k_segmented<DT, OP, 0>, p);
 }
 
 template <int DT>
-cudaError_t launch_segmented_dt(int op, const SegParams& p, bool warp_per_seg, int block, cudaStream_t s) {
+cudaError_t launch_segmented_dt(int op, const SegParams& p, int group, int block, cudaStream_t s) {
   switch (op) {
-    case OP_SUM: return launch_segmented_op<DT, OP_SUM>(p, warp_per_seg, block, s);
-    case OP_MIN: return launch_segmented_op<DT, OP_MIN>(p, warp_per_seg, block, s);
-    case OP_MAX: return launch_segmented_op<DT, OP_MAX>(p, warp_per_seg, block, s);
+    case OP_SUM: return launch_segmented_op<DT, OP_SUM>(p, group, block, s);
+    case OP_MIN: return launch_segmented_op<DT, OP_MIN>(p, group, block, s);
+    case OP_MAX: return launch_segmented_op<DT, OP_MAX>(p, group, block, s);
   }
   return cudaErrorInvalidValue;
 }

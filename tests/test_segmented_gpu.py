@@ -49,7 +49,7 @@ def _segments(rng, nseg, max_len, skew=False):
 
 
 @pytest.mark.parametrize("dtype", DTYPES)
-@pytest.mark.parametrize("group", [0, 1, 2])
+@pytest.mark.parametrize("group", [0, 1, 2, 3])
 @pytest.mark.parametrize("skew", [False, True])
 def test_segmented_matches_oracle_per_segment(dtype, group, skew):
     import torch
@@ -61,22 +61,24 @@ def test_segmented_matches_oracle_per_segment(dtype, group, skew):
     xt = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     ot = torch.from_numpy(offs).cuda()
     bounds = list(zip(offs[:-1].tolist(), offs[1:].tolist()))
-    lanes = 32 if group in (0, 1) else 256
+    lanes = {0: 32, 1: 32, 2: 256, 3: 8}[group]
     for op in OPS:
         got = rb.reduce_segmented(xt, ot, op, seg_group=group).cpu().numpy()
         _check_segments(x, bounds, op, got, lanes)
 
 
 @pytest.mark.parametrize("dtype", DTYPES)
-@pytest.mark.parametrize("rows,cols", [(1, 1), (7, 33), (1000, 1024), (64, 100003), (4096, 17)])
+@pytest.mark.parametrize("rows,cols", [(1, 1), (7, 33), (1000, 1024), (64, 100003), (4096, 17), (100003, 64),
+                                       (3000, 129)])
 def test_batched_rows(dtype, rows, cols):
     import torch
     import paper_conf_cgo_gonzalohghmh19_b200 as rb
     x = synth.make(dtype, rows * cols, "int_full" if dtype == "int32" else "uniform01", rows + cols)
     xt = torch.from_numpy(x).cuda().view(rows, cols)
     bounds = [(r * cols, (r + 1) * cols) for r in range(rows)]
-    for group in (0, 1, 2):
-        lanes = 32 if (group == 1 or (group == 0 and cols <= 4096)) else 256
+    for group in (0, 1, 2, 3):
+        auto = 8 if cols <= 128 else (32 if cols <= 4096 else 256)
+        lanes = {0: auto, 1: 32, 2: 256, 3: 8}[group]
         for op in OPS:
             got = rb.reduce_batched(xt, op, seg_group=group).cpu().numpy()
             _check_segments(x, bounds, op, got, lanes)
@@ -92,9 +94,9 @@ def test_segmented_special_values_and_determinism():
     offs = np.array([0, 10, 10, 50001, 70000, 70001, 100000], np.int64)
     xt, ot = torch.from_numpy(x).cuda(), torch.from_numpy(offs).cuda()
     bounds = list(zip(offs[:-1].tolist(), offs[1:].tolist()))
-    for group in (1, 2):
+    for group in (1, 2, 3):
         for op in OPS:
             got = rb.reduce_segmented(xt, ot, op, seg_group=group).cpu().numpy()
-            _check_segments(x, bounds, op, got, 32 if group == 1 else 256)
+            _check_segments(x, bounds, op, got, {1: 32, 2: 256, 3: 8}[group])
     outs = {rb.reduce_segmented(xt, ot, "sum").cpu().numpy().tobytes() for _ in range(20)}
     assert len(outs) == 1
