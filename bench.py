@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--sharded", action="store_true",
+                    help="use the sharded reduce_multi path even at one rank (exercises S7 on one GPU)")
     return ap.parse_args()
 
 
@@ -172,12 +174,12 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
-def workload_config(args, world, plan):
+def workload_config(args, world, plan, sharded=False):
     cfg = {"workload": f"fp32 sum of {args.n} (2^{args.n.bit_length() - 1}) elements per GPU"
                        + (" -- BASELINE configs[1] largest point" if world == 1 else
                           f" -- BASELINE configs[4] sharded sum, {world} GPUs, NCCL all-reduce of partials"),
            "n_per_gpu": args.n, "total_bytes": args.n * 4 * world, "op": "sum", "mode": args.mode,
-           "parallelism": f"shard{world}" if world > 1 else "single-gpu",
+           "parallelism": f"shard{world}" if (world > 1 or sharded) else "single-gpu",
            "l2": "inputs (4 B x n per GPU) larger than the 126 MB L2 between steps; no flush needed",
            "distribution": "U[0,1) fp32, numpy PCG64 seed 2019+1000*1+log2(n)+rank"}
     if plan is not None:
@@ -202,14 +204,19 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
+    sharded = world > 1 or args.sharded
+    if sharded:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        os.environ.setdefault("RANK", str(rank))
+        os.environ.setdefault("WORLD_SIZE", str(world))
         dist.init_process_group("nccl", device_id=dev)
     n = args.n
     x_host = synth.make("float32", n, "uniform01", synth.seed_for(1, n, rank))
     x = torch.from_numpy(x_host).to(dev)
     out = torch.empty(1, dtype=torch.float32, device=dev)
     stream = torch.cuda.Stream(dev)
-    comm = rb.Comm() if world > 1 else None
+    comm = rb.Comm() if sharded else None
     plan = rb.query_plan("float32", "sum", n, in_ptr=x.data_ptr(), mode=args.mode)
     rb.prepare(stream, n)
 
@@ -286,7 +293,7 @@ def main():
     torch.cuda.synchronize(dev)
     kern_ms = [a.elapsed_time(b) for a, b in evs]
     k_event = statistics.mean(kern_ms)
-    kavg = ms if (world == 1 and plan["launches"] == 1) else k_event
+    kavg = ms if (comm is None and plan["launches"] == 1) else k_event
     peak, peak_src = measured_peaks()
     achieved = n * 4 / (kavg * 1e-3) / 1e9
     traffic, ncu_s = ncu_traffic()
@@ -431,9 +438,9 @@ def main():
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
-            "data": "synthetic", "config": workload_config(args, world, plan),
+            "data": "synthetic", "config": workload_config(args, world, plan, comm is not None),
             "elements_per_s": round(world * n / (ms * 1e-3), 1),
-            "launch": "cuda-graph replay of the K steps" if world == 1 else "stream (K reduce_multi calls)",
+            "launch": "cuda-graph replay of the K steps" if comm is None else "stream (K reduce_multi calls)",
             "stream_launched": None if stream_ms is None else {
                 "ms_per_step": round(stream_ms, 5), "value": round(world * n * 4 / (stream_ms * 1e-3) / 1e9, 2)},
             "frac_of_hbm_peak": round(value / world / peak, 4),

@@ -45,8 +45,10 @@ __device__ __forceinline__ void fold_range(typename T::Acc (&a)[T::NA], uint32_t
     ld_v8(body + v * kVecBytes, r);
     fold_vec<T>(a, aux, r);
   }
+  // head and tail (< 8 elements each) by the first lanes, into two different
+  // accumulators (groups may be only 8 lanes wide)
   if (lid < head) fold_elem<T>(a[0], aux, __ldg((const Elem*)p + lid));
-  if (lid >= 8 && lid - 8 < tail) fold_elem<T>(a[0], aux, __ldg((const Elem*)(body + nvec * kVecBytes) + (lid - 8)));
+  if (lid < tail) fold_elem<T>(a[1], aux, __ldg((const Elem*)(body + nvec * kVecBytes) + lid));
 }
 
 template <class T>
