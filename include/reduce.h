@@ -60,7 +60,12 @@ extern "C" {
 typedef struct CUstream_st* reduce_stream_t;
 
 typedef enum { REDUCE_INT32 = 0, REDUCE_FLOAT32 = 1, REDUCE_FLOAT64 = 2 } reduce_dtype_t;
-typedef enum { REDUCE_SUM = 0, REDUCE_MIN = 1, REDUCE_MAX = 2 } reduce_op_t;
+/* REDUCE_SUM_ACCURATE (fp dtypes only): the same sum at the
+ * same bandwidth with a wider accumulator -- fp32 input accumulated in fp64 from
+ * the first addition (error <= u_f|S| + (L+1)*2^-53*sum|x|), fp64 input in
+ * double-double (Neumaier fold + TwoSum merges; error ~ u_d|S|).  The output
+ * keeps the input dtype.  Beyond the paper, which reduces in the element type. */
+typedef enum { REDUCE_SUM = 0, REDUCE_MIN = 1, REDUCE_MAX = 2, REDUCE_SUM_ACCURATE = 3 } reduce_op_t;
 typedef enum { REDUCE_MODE_FAST = 0, REDUCE_MODE_DETERMINISTIC = 1 } reduce_mode_t;
 
 typedef enum {
@@ -185,8 +190,8 @@ int reduce_host(int dtype, int op, const void* host_in, size_t n, void* host_out
  * num_segments elements of dtype.  One warp or one block per segment (the
  * paper's small-array versions assign one warp / block per partition with no
  * global atomics): one launch, no atomics, deterministic.
- * Segment starts may have any element alignment.  Options used: block,
- * seg_group.  reduce_batched is the uniform case: num_segments rows of seg_len
+ * Segment starts may have any element alignment.  Options used: block
+ * (32..512, default 256), seg_group.  reduce_batched is the uniform case: num_segments rows of seg_len
  * contiguous elements (row i at in + i*seg_len), no offsets array. */
 int reduce_segmented(int dtype, int op, const void* in, const int64_t* offsets, size_t num_segments, void* out,
                      reduce_stream_t stream, const reduce_opts_t* opts);

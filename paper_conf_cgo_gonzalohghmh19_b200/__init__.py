@@ -17,14 +17,14 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_PKG, "libreduce_b200.so")
 
 INT32, FLOAT32, FLOAT64 = 0, 1, 2
-SUM, MIN, MAX = 0, 1, 2
+SUM, MIN, MAX, SUM_ACCURATE = 0, 1, 2, 3
 MODE_FAST, MODE_DETERMINISTIC = 0, 1
 BC_SHFL, BC_SMEM_ATOMIC_WARP, BC_SMEM_ATOMIC_ALL, BC_SMEM_TREE = 0, 1, 2, 3
 GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER = 0, 1, 2, 3, 4
 STAGE_REG, STAGE_SMEM = 1, 2
 OK = 0
 
-OPS = {"sum": SUM, "min": MIN, "max": MAX}
+OPS = {"sum": SUM, "min": MIN, "max": MAX, "sum_accurate": SUM_ACCURATE}
 DTYPE_NAMES = {"int32": INT32, "float32": FLOAT32, "float64": FLOAT64}
 ELEM_BYTES = {INT32: 4, FLOAT32: 4, FLOAT64: 8}
 

@@ -51,7 +51,9 @@ static int ilog2_ceil(unsigned long long v) {
 
 int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* opts, int raw_out, Plan* P) {
   if (dtype < 0 || dtype > 2) return fail(REDUCE_ERR_INVALID_ARG, "dtype must be REDUCE_INT32/FLOAT32/FLOAT64");
-  if (op < 0 || op > 2) return fail(REDUCE_ERR_INVALID_ARG, "op must be REDUCE_SUM/MIN/MAX");
+  if (op < 0 || op > 3) return fail(REDUCE_ERR_INVALID_ARG, "op must be REDUCE_SUM/MIN/MAX/SUM_ACCURATE");
+  if (op == REDUCE_SUM_ACCURATE && dtype == REDUCE_INT32)
+    return fail(REDUCE_ERR_INVALID_ARG, "REDUCE_SUM_ACCURATE needs a floating-point dtype (int32 sums are exact mod 2^32)");
   const int s = elem_bytes(dtype);
   if (n > 0 && in == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "in is NULL with n > 0");
   if (n > 0 && ((uintptr_t)in % (uintptr_t)s) != 0)
@@ -80,12 +82,19 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
       return fail(REDUCE_ERR_INVALID_ARG, "deterministic mode forbids shared-atomic block combines");
   }
 
-  // ---- S0: table lookup by ceil(log2(bytes))
+  const bool dd = op == REDUCE_SUM_ACCURATE && dtype == REDUCE_FLOAT64;  // double-double: no atomics on values
+  if (dd && o.grid_combine == REDUCE_GC_ATOMIC)
+    return fail(REDUCE_ERR_INVALID_ARG, "fp64 accurate sums have no ATOMIC grid combine (double-double values)");
+  if (dd && (o.block_combine == REDUCE_BC_SMEM_ATOMIC_WARP || o.block_combine == REDUCE_BC_SMEM_ATOMIC_ALL))
+    return fail(REDUCE_ERR_INVALID_ARG, "fp64 accurate sums have no shared-atomic block combine");
+
+  // ---- S0: table lookup by ceil(log2(bytes)); the accurate sum uses the sum rows
+  const int op_row = op == REDUCE_SUM_ACCURATE ? REDUCE_SUM : op;
   const unsigned long long bytes = (unsigned long long)n * (unsigned long long)s;
   const int lb = ilog2_ceil(bytes ? bytes : 1);
   const DispatchEntry* e = nullptr;
   for (const DispatchEntry& r : kDispatch) {
-    if ((r.dtype < 0 || r.dtype == dtype) && (r.op < 0 || r.op == op) && (r.mode < 0 || r.mode == mode) &&
+    if ((r.dtype < 0 || r.dtype == dtype) && (r.op < 0 || r.op == op_row) && (r.mode < 0 || r.mode == mode) &&
         lb <= r.max_log2_bytes) {
       e = &r;
       break;
@@ -112,10 +121,12 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   else if (e->gc >= 0) gc = e->gc;
   else gc = mode == REDUCE_MODE_DETERMINISTIC ? REDUCE_GC_TWO_PASS : REDUCE_GC_ATOMIC;
   if (o.grid_combine < 0 && mode == REDUCE_MODE_DETERMINISTIC && gc == REDUCE_GC_ATOMIC) gc = REDUCE_GC_TWO_PASS;
-  if (o.block_combine < 0 && mode == REDUCE_MODE_DETERMINISTIC &&
+  if (o.grid_combine < 0 && dd && gc == REDUCE_GC_ATOMIC) gc = REDUCE_GC_LAST_BLOCK;
+  if (o.block_combine < 0 && (mode == REDUCE_MODE_DETERMINISTIC || dd) &&
       (bc == REDUCE_BC_SMEM_ATOMIC_WARP || bc == REDUCE_BC_SMEM_ATOMIC_ALL))
     bc = REDUCE_BC_SHFL;
   const int grid_cap = o.grid > 0 ? o.grid : e->grid_cap;
+  if (!o.block && block > max_block_threads(dtype, op, unroll, stage)) block = max_block_threads(dtype, op, unroll, stage);
   if (block > max_block_threads(dtype, op, unroll, stage))
     return fail(REDUCE_ERR_INVALID_ARG, "block too large for this (dtype, op, unroll): max " +
                                             std::to_string(max_block_threads(dtype, op, unroll, stage)));
@@ -153,7 +164,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
 
   // ---- longest fp addition chain L of this variant (for the G2 gate)
   long long chain = 0;
-  if (op == REDUCE_SUM && dtype != REDUCE_INT32) {
+  if ((op == REDUCE_SUM || op == REDUCE_SUM_ACCURATE) && dtype != REDUCE_INT32) {
     const int na = dtype == REDUCE_FLOAT64 ? 4 : 8;
     const long long tpb = (tiles + grid - 1) / grid;
     const int nw = block / 32;
@@ -164,7 +175,17 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
       case REDUCE_BC_SMEM_ATOMIC_ALL: chain += block; break;
       case REDUCE_BC_SMEM_TREE: chain += ilog2_ceil(block); break;
     }
-    if (dtype == REDUCE_FLOAT32) {
+    if (op == REDUCE_SUM_ACCURATE) {
+      // the whole chain runs in fp64 (fp32 input) or double-double (fp64
+      // input): L counts additions of that wider format, plus the final rounding
+      switch (gc) {
+        case REDUCE_GC_ATOMIC: chain += (grid + nslots - 1) / nslots + 5; break;
+        case REDUCE_GC_TWO_PASS: chain += (grid + 1023) / 1024 + 10; break;
+        case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + ilog2_ceil(block); break;
+        case REDUCE_GC_CLUSTER: chain += 5; break;
+        default: break;
+      }
+    } else if (dtype == REDUCE_FLOAT32) {
       // blocks combine in fp64: the cross-block error is < grid * 2^-53 relative,
       // far below one fp32 ulp; the single fp64 -> fp32 rounding adds 1.
       chain += gc == REDUCE_GC_DIRECT ? 0 : 1;
@@ -272,7 +293,7 @@ int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
 
 int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream) {
   LaunchDesc& d = P->d;
-  const int combo = d.dtype * 3 + d.op;
+  const int combo = combo_index(d.dtype, d.op);
   d.out = out;
   d.slots = ws->slots + combo * kSlotRegionBytes;
   d.ticket = (unsigned*)(ws->tickets + combo * (size_t)kSlotBytes);
@@ -311,7 +332,9 @@ int reduce_ex(int dtype, int op, const void* in, size_t n, void* out, reduce_str
 static int segmented_common(int dtype, int op, const void* in, const int64_t* offsets, size_t seg_len,
                             size_t nseg, void* out, reduce_stream_t stream, const reduce_opts_t* opts) {
   if (dtype < 0 || dtype > 2) return fail(REDUCE_ERR_INVALID_ARG, "dtype must be REDUCE_INT32/FLOAT32/FLOAT64");
-  if (op < 0 || op > 2) return fail(REDUCE_ERR_INVALID_ARG, "op must be REDUCE_SUM/MIN/MAX");
+  if (op < 0 || op > 3) return fail(REDUCE_ERR_INVALID_ARG, "op must be REDUCE_SUM/MIN/MAX/SUM_ACCURATE");
+  if (op == REDUCE_SUM_ACCURATE && dtype == REDUCE_INT32)
+    return fail(REDUCE_ERR_INVALID_ARG, "REDUCE_SUM_ACCURATE needs a floating-point dtype");
   const int s = dtype == REDUCE_FLOAT64 ? 8 : 4;
   if (nseg == 0) return REDUCE_OK;
   if (out == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "out is NULL");
@@ -321,8 +344,8 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   if (in && ((uintptr_t)in % (uintptr_t)s) != 0) return fail(REDUCE_ERR_INVALID_ARG, "in is not aligned to the element size");
   int block = 256, group = 0;
   if (opts) {
-    if (opts->block != 0 && (opts->block < 32 || opts->block > 1024 || opts->block % 32 != 0))
-      return fail(REDUCE_ERR_INVALID_ARG, "block must be 0 or a multiple of 32 in [32, 1024]");
+    if (opts->block != 0 && (opts->block < 32 || opts->block > 512 || opts->block % 32 != 0))
+      return fail(REDUCE_ERR_INVALID_ARG, "segmented block must be 0 or a multiple of 32 in [32, 512]");
     if (opts->seg_group < 0 || opts->seg_group > 3) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0..3");
     if (opts->block) block = opts->block;
     group = opts->seg_group;

@@ -35,9 +35,9 @@ bool pdl_enabled() {
 }
 
 int grid_value_bytes(int dtype, int op) {
-  if (dtype == 0) return 4;            // int32: uint32 / int32
-  if (dtype == 1) return op == 0 ? 8 : 4;  // fp32: double sum / uint32 key
-  return 8;                            // fp64: double / uint64 key
+  if (dtype == 0) return 4;                                // int32: uint32 / int32
+  if (dtype == 1) return (op == 0 || op == 3) ? 8 : 4;     // fp32: double sums / uint32 key
+  return op == 3 ? 16 : 8;                                 // fp64: double-double / double / uint64 key
 }
 
 cudaError_t launch_reduce(const LaunchDesc& d, cudaStream_t s) {

@@ -20,7 +20,7 @@
 namespace rb {
 
 constexpr int DT_I32 = 0, DT_F32 = 1, DT_F64 = 2;
-constexpr int OP_SUM = 0, OP_MIN = 1, OP_MAX = 2;
+constexpr int OP_SUM = 0, OP_MIN = 1, OP_MAX = 2, OP_SUMACC = 3;
 constexpr int BC_SHFL = 0, BC_ATOMIC_WARP = 1, BC_ATOMIC_ALL = 2, BC_TREE = 3;
 constexpr int GC_DIRECT = 0, GC_ATOMIC = 1, GC_TWO_PASS = 2, GC_LAST_BLOCK = 3, GC_CLUSTER = 4;
 constexpr int kVecBytes = 32;    // one 256-bit load per thread per vector
@@ -112,11 +112,18 @@ __device__ __forceinline__ unsigned long long unkey64(unsigned long long k) {
   return (k >> 63) ? (k & 0x7FFFFFFFFFFFFFFFull) : ~k;
 }
 
-// Generic butterfly for any 4/8-byte type with a combine functor; result in all lanes.
+// Butterfly exchange for scalar types and for double2 (double-double pairs).
+template <class V>
+__device__ __forceinline__ V shfl_xor(V v, int o) { return __shfl_xor_sync(0xffffffffu, v, o); }
+__device__ __forceinline__ double2 shfl_xor(double2 v, int o) {
+  return make_double2(__shfl_xor_sync(0xffffffffu, v.x, o), __shfl_xor_sync(0xffffffffu, v.y, o));
+}
+
+// Generic butterfly with a combine functor; result in all lanes.
 template <class V, class F>
 __device__ __forceinline__ V warp_butterfly(V v, F f) {
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v = f(v, __shfl_xor_sync(0xffffffffu, v, o));
+  for (int o = 16; o > 0; o >>= 1) v = f(v, shfl_xor(v, o));
   return v;
 }
 
@@ -265,9 +272,74 @@ template <int OP> struct TrF64 {
   }
 };
 
+// ---- accurate sums: same bandwidth, tighter error --------
+// fp32 input, fp64 accumulation from the first add: error <= u_f|S| + (L+1) u_d sum|x|.
+struct TrF32Acc {
+  using Elem = float;
+  using Acc = double;
+  using Grid = double;
+  static constexpr int VE = 8, NA = 8, kLaneWords = 1;
+  __device__ static Acc ident() { return 0.0; }
+  __device__ static Acc comb(Acc a, Acc b) { return a + b; }
+  __device__ static void fold(Acc& a, uint32_t&, uint32_t w) { a += (double)__uint_as_float(w); }
+  __device__ static Acc warp(Acc v) { return warp_butterfly(v, [](double x, double y) { return x + y; }); }
+  __device__ static Acc finish(Acc a, uint32_t) { return a; }
+  __device__ static Grid to_grid(Acc a) { return a; }
+  __device__ static Grid gident() { return 0.0; }
+  __device__ static Grid gcomb(Grid a, Grid b) { return a + b; }
+  __device__ static Grid gwarp(Grid v) { return warp(v); }
+  __device__ static void gred(Grid* p, Grid v) { atomicAdd(p, v); }
+  __device__ static Grid gexch(Grid* p, Grid v) {
+    return __longlong_as_double((long long)atomicExch((unsigned long long*)p, (unsigned long long)__double_as_longlong(v)));
+  }
+  __device__ static void finalize(Grid g, void* out) {
+    const float f = (float)g;
+    *(uint32_t*)out = (f != f) ? 0x7FC00000u : __float_as_uint(f);
+  }
+};
+
+// fp64 input, double-double accumulation: each accumulator is (hi, lo) with
+// Neumaier's fold (Neumaier 1974) and Knuth's TwoSum for merging pairs; the
+// result is hi + lo rounded once.  Non-finite inputs are carried by hi alone
+// (hi is the plain running sum), so inf / NaN follow reading R2.
+struct TrF64Acc {
+  using Elem = double;
+  using Acc = double2;  // x = hi, y = lo
+  using Grid = double2;
+  static constexpr int VE = 4, NA = 4, kLaneWords = 2;
+  __device__ static Acc ident() { return make_double2(0.0, 0.0); }
+  __device__ static Acc comb(Acc a, Acc b) {
+    const double s = a.x + b.x;                       // TwoSum(a.hi, b.hi)
+    const double bb = s - a.x;
+    const double e = (a.x - (s - bb)) + (b.x - bb);
+    const double lo = a.y + b.y + e;
+    const double hi = s + lo;                         // FastTwoSum renormalise
+    return make_double2(isfinite(s) ? hi : s, isfinite(s) ? lo - (hi - s) : 0.0);
+  }
+  __device__ static void fold(Acc& a, uint32_t&, double x) {
+    const double t = a.x + x;
+    a.y += (fabs(a.x) >= fabs(x)) ? (a.x - t) + x : (x - t) + a.x;
+    a.x = t;
+  }
+  __device__ static Acc warp(Acc v) { return warp_butterfly(v, [](double2 x, double2 y) { return comb(x, y); }); }
+  __device__ static Acc finish(Acc a, uint32_t) { return a; }
+  __device__ static Grid to_grid(Acc a) { return a; }
+  __device__ static Grid gident() { return ident(); }
+  __device__ static Grid gcomb(Grid a, Grid b) { return comb(a, b); }
+  __device__ static Grid gwarp(Grid v) { return warp(v); }
+  __device__ static void gred(Grid*, Grid) { __trap(); }        // no 128-bit fp atomics: ATOMIC is never planned
+  __device__ static Grid gexch(Grid*, Grid) { __trap(); return ident(); }
+  __device__ static void finalize(Grid g, void* out) {
+    const double r = isfinite(g.x) ? g.x + g.y : g.x;
+    *(unsigned long long*)out = (r != r) ? 0x7FF8000000000000ull : (unsigned long long)__double_as_longlong(r);
+  }
+};
+
 template <int OP> struct Tr<DT_I32, OP> : TrI32<OP> {};
 template <int OP> struct Tr<DT_F32, OP> : TrF32<OP> {};
 template <int OP> struct Tr<DT_F64, OP> : TrF64<OP> {};
+template <> struct Tr<DT_F32, OP_SUMACC> : TrF32Acc {};
+template <> struct Tr<DT_F64, OP_SUMACC> : TrF64Acc {};
 
 // Fold one 32-byte vector into the NA per-thread accumulators (lane k of the
 // vector goes to accumulator k: NA independent chains).

@@ -22,7 +22,7 @@ using namespace rb;
 extern "C" int reduce_host(int dtype, int op, const void* host_in, size_t n, void* host_out, reduce_stream_t stream,
                            const reduce_opts_t* opts) {
   if (dtype < 0 || dtype > 2) return fail(REDUCE_ERR_INVALID_ARG, "dtype must be REDUCE_INT32/FLOAT32/FLOAT64");
-  if (op < 0 || op > 2) return fail(REDUCE_ERR_INVALID_ARG, "op must be REDUCE_SUM/MIN/MAX");
+  if (op < 0 || op > 3) return fail(REDUCE_ERR_INVALID_ARG, "op must be REDUCE_SUM/MIN/MAX/SUM_ACCURATE");
   if (host_out == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "host_out is NULL");
   if (n > 0 && host_in == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "host_in is NULL with n > 0");
   const size_t s = dtype == REDUCE_FLOAT64 ? 8 : 4;
@@ -49,7 +49,7 @@ extern "C" int reduce_host(int dtype, int op, const void* host_in, size_t n, voi
   if ((st = get_workspace(cs, pbytes, &ws)) != REDUCE_OK) return st;
 
   // staging: 2 x chunk_bytes, then the per-chunk raw values
-  const size_t vals_bytes = (size_t)kMaxChunks * 8;
+  const size_t vals_bytes = (size_t)kMaxChunks * 16;  // up to 16-byte raw values (double-double)
   if (ws->staging_bytes < chunk_bytes) {
     if (ws->staging) {
       cudaStreamSynchronize(cs);

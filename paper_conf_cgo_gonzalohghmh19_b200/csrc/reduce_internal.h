@@ -24,7 +24,9 @@ constexpr int kMaxSmemTileBytes = 128 * 1024;
 // too small for 8 in-flight 32-byte loads, and for the fp64 min/max
 // select+NaN-flag fold at unroll >= 2.
 constexpr int max_block_threads(int dtype, int op, int unroll, int stage = STAGE_REG) {
-  return stage == STAGE_SMEM ? 1024 : ((unroll >= 8 || (dtype == 2 && op != 0 && unroll >= 2)) ? 512 : 1024);
+  return stage == STAGE_SMEM ? (op == 3 ? 512 : 1024)
+                             : ((unroll >= 8 || (dtype == 2 && op != 0 && unroll >= 2) || (op == 3 && unroll >= 4))
+                                    ? 512 : 1024);
 }
 
 // One launch of the main reduction kernel (steps S2-S5), fully resolved by the
@@ -76,7 +78,8 @@ cudaError_t launch_init_workspace(void* slots_base, void* tickets_base, cudaStre
 // environment variable REDUCE_NO_PDL=1 turns it off, for A/B measurements).
 bool pdl_enabled();
 
-constexpr int kCombos = 9;  // 3 dtypes x 3 ops
+constexpr int kCombos = 12;  // 3 dtypes x 4 ops (sum, min, max, accurate sum)
+constexpr int combo_index(int dtype, int op) { return dtype * 4 + op; }
 constexpr size_t kSlotRegionBytes = (size_t)kMaxSlots * kSlotBytes;
 
 }  // namespace rb

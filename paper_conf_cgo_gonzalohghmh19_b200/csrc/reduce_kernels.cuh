@@ -295,6 +295,11 @@ cudaError_t launch_combine_kernel(const void* vals, long long count, void* out, 
 
 template <int DT, int OP, int U, int STAGE>
 cudaError_t launch_bc(const LaunchDesc& d, const KParams& p, cudaStream_t s) {
+  if constexpr (DT == DT_F64 && OP == OP_SUMACC) {  // no shared atomics on double-double pairs
+    if (d.bc == BC_SHFL) return launch_kernel(k_reduce<DT, OP, U, BC_SHFL, STAGE>, d, p, s);
+    if (d.bc == BC_TREE) return launch_kernel(k_reduce<DT, OP, U, BC_TREE, STAGE>, d, p, s);
+    return cudaErrorInvalidValue;
+  }
   switch (d.bc) {
     case BC_SHFL: return launch_kernel(k_reduce<DT, OP, U, BC_SHFL, STAGE>, d, p, s);
     case BC_ATOMIC_WARP: return launch_kernel(k_reduce<DT, OP, U, BC_ATOMIC_WARP, STAGE>, d, p, s);
@@ -334,6 +339,9 @@ cudaError_t launch_dt(const LaunchDesc& d, cudaStream_t s) {
     case OP_SUM: return launch_op<DT, OP_SUM>(d, s);
     case OP_MIN: return launch_op<DT, OP_MIN>(d, s);
     case OP_MAX: return launch_op<DT, OP_MAX>(d, s);
+    case OP_SUMACC:
+      if constexpr (DT != DT_I32) return launch_op<DT, OP_SUMACC>(d, s);
+      break;
   }
   return cudaErrorInvalidValue;
 }
@@ -344,18 +352,24 @@ cudaError_t combine_dt(int op, const void* vals, long long count, void* out, int
     case OP_SUM: return launch_combine_kernel<DT, OP_SUM>(vals, count, out, raw_out, block, s);
     case OP_MIN: return launch_combine_kernel<DT, OP_MIN>(vals, count, out, raw_out, block, s);
     case OP_MAX: return launch_combine_kernel<DT, OP_MAX>(vals, count, out, raw_out, block, s);
+    case OP_SUMACC:
+      if constexpr (DT != DT_I32) return launch_combine_kernel<DT, OP_SUMACC>(vals, count, out, raw_out, block, s);
+      break;
   }
   return cudaErrorInvalidValue;
 }
 
 template <int DT>
 cudaError_t init_dt(char* slots_base, char* tickets_base, cudaStream_t s) {
-  k_init_slots<DT, OP_SUM><<<1, 32, 0, s>>>(slots_base + (DT * 3 + OP_SUM) * kSlotRegionBytes,
-                                             (unsigned*)(tickets_base + (DT * 3 + OP_SUM) * kSlotBytes));
-  k_init_slots<DT, OP_MIN><<<1, 32, 0, s>>>(slots_base + (DT * 3 + OP_MIN) * kSlotRegionBytes,
-                                             (unsigned*)(tickets_base + (DT * 3 + OP_MIN) * kSlotBytes));
-  k_init_slots<DT, OP_MAX><<<1, 32, 0, s>>>(slots_base + (DT * 3 + OP_MAX) * kSlotRegionBytes,
-                                             (unsigned*)(tickets_base + (DT * 3 + OP_MAX) * kSlotBytes));
+  k_init_slots<DT, OP_SUM><<<1, 32, 0, s>>>(slots_base + combo_index(DT, OP_SUM) * kSlotRegionBytes,
+                                             (unsigned*)(tickets_base + combo_index(DT, OP_SUM) * kSlotBytes));
+  k_init_slots<DT, OP_MIN><<<1, 32, 0, s>>>(slots_base + combo_index(DT, OP_MIN) * kSlotRegionBytes,
+                                             (unsigned*)(tickets_base + combo_index(DT, OP_MIN) * kSlotBytes));
+  k_init_slots<DT, OP_MAX><<<1, 32, 0, s>>>(slots_base + combo_index(DT, OP_MAX) * kSlotRegionBytes,
+                                             (unsigned*)(tickets_base + combo_index(DT, OP_MAX) * kSlotBytes));
+  if constexpr (DT != DT_I32)
+    k_init_slots<DT, OP_SUMACC><<<1, 32, 0, s>>>(slots_base + combo_index(DT, OP_SUMACC) * kSlotRegionBytes,
+                                                  (unsigned*)(tickets_base + combo_index(DT, OP_SUMACC) * kSlotBytes));
   return cudaPeekAtLastError();
 }
 

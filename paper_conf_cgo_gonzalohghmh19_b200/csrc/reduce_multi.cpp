@@ -72,10 +72,12 @@ int nccl_fail(ncclResult_t r, const char* what) {
 // block-combine value; fp min/max as order-preserving unsigned keys.
 ncclDataType_t raw_type(int dtype, int op) {
   if (dtype == REDUCE_INT32) return op == REDUCE_SUM ? ncclUint32 : ncclInt32;
-  if (dtype == REDUCE_FLOAT32) return op == REDUCE_SUM ? ncclFloat64 : ncclUint32;
-  return op == REDUCE_SUM ? ncclFloat64 : ncclUint64;
+  if (dtype == REDUCE_FLOAT32) return (op == REDUCE_SUM || op == REDUCE_SUM_ACCURATE) ? ncclFloat64 : ncclUint32;
+  return (op == REDUCE_SUM || op == REDUCE_SUM_ACCURATE) ? ncclFloat64 : ncclUint64;
 }
-ncclRedOp_t raw_op(int op) { return op == REDUCE_SUM ? ncclSum : (op == REDUCE_MIN ? ncclMin : ncclMax); }
+ncclRedOp_t raw_op(int op) {
+  return (op == REDUCE_SUM || op == REDUCE_SUM_ACCURATE) ? ncclSum : (op == REDUCE_MIN ? ncclMin : ncclMax);
+}
 
 }  // namespace
 }  // namespace rb
@@ -141,7 +143,10 @@ int reduce_multi_ex(int dtype, int op, const void* in_local, size_t n_local, voi
   const ncclDataType_t t = raw_type(dtype, op);
   void* raw = direct ? out : (void*)ws->scalars;
 
-  if (P.mode != REDUCE_MODE_DETERMINISTIC) {
+  // double-double raw values cannot be summed by NCCL: gather them instead
+  const bool gather = P.mode == REDUCE_MODE_DETERMINISTIC || (dtype == REDUCE_FLOAT64 && op == REDUCE_SUM_ACCURATE);
+  const size_t raw_count = (size_t)grid_value_bytes(dtype, op) / (t == ncclFloat64 || t == ncclUint64 ? 8 : 4);
+  if (!gather) {
     if ((st = launch_plan(&P, ws, raw, cs)) != REDUCE_OK) return st;
     ncclResult_t r = g_nccl.AllReduce(raw, raw, 1, t, raw_op(op), c, cs);
     if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
@@ -155,13 +160,13 @@ int reduce_multi_ex(int dtype, int op, const void* in_local, size_t n_local, voi
   int nranks = 0;
   ncclResult_t r = g_nccl.CommCount(c, &nranks);
   if (r != ncclSuccess) return nccl_fail(r, "ncclCommCount");
-  if ((size_t)nranks * 8 + kScalarBytes > (size_t)kNumScalars * kScalarBytes)
+  if ((size_t)nranks * 16 + kScalarBytes > (size_t)kNumScalars * kScalarBytes)
     return fail(REDUCE_ERR_UNSUPPORTED, "too many ranks for the deterministic gather buffer");
   P.d.raw_out = 1;
   raw = ws->scalars;
   void* gathered = ws->scalars + kScalarBytes;
   if ((st = launch_plan(&P, ws, raw, cs)) != REDUCE_OK) return st;
-  r = g_nccl.AllGather(raw, gathered, 1, t, c, cs);
+  r = g_nccl.AllGather(raw, gathered, raw_count, t, c, cs);
   if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather");
   cudaError_t e = launch_combine(dtype, op, gathered, nranks, out, 0, 32, cs);
   if (e != cudaSuccess) return cuda_fail(e, "rank-order combine kernel");

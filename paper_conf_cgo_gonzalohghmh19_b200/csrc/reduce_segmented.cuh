@@ -62,7 +62,7 @@ __device__ __forceinline__ void seg_store(const SegParams& p, long long seg, typ
 // blocks per SM) and groups stride over the segments, so millions of tiny
 // segments do not pay one CTA launch each.
 template <int DT, int OP, int kGroup>
-__global__ void __launch_bounds__(1024) k_segmented(const SegParams p) {
+__global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
   pdl_wait();
@@ -112,7 +112,7 @@ __global__ void __launch_bounds__(1024) k_segmented(const SegParams p) {
     } else if constexpr (kGroup > 0) {
       Acc w = v;
 #pragma unroll
-      for (int o = kGroup / 2; o > 0; o >>= 1) w = T::comb(w, __shfl_xor_sync(0xffffffffu, w, o));
+      for (int o = kGroup / 2; o > 0; o >>= 1) w = T::comb(w, shfl_xor(w, o));
       if (lid == 0 && live) seg_store<T>(p, seg, T::to_grid(w));
     } else {
       const typename T::Grid g = block_combine<T, BC_SHFL>(v);
@@ -152,6 +152,9 @@ cudaError_t launch_segmented_dt(int op, const SegParams& p, int group, int block
     case OP_SUM: return launch_segmented_op<DT, OP_SUM>(p, group, block, s);
     case OP_MIN: return launch_segmented_op<DT, OP_MIN>(p, group, block, s);
     case OP_MAX: return launch_segmented_op<DT, OP_MAX>(p, group, block, s);
+    case OP_SUMACC:
+      if constexpr (DT != DT_I32) return launch_segmented_op<DT, OP_SUMACC>(p, group, block, s);
+      break;
   }
   return cudaErrorInvalidValue;
 }
