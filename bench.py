@@ -390,6 +390,24 @@ def main():
                 latency.append({"dtype": dt, "n": m, "graph_us": round(g_us, 3), "stream_b2b_us": round(s_us, 3),
                                 "host_wall_us": round(statistics.median(walls) * 1e6, 2)})
 
+    # ---- every (dtype, op) at 1 GiB (the resident input reinterpreted; > L2):
+    # device time per call from a graph of 20 calls, default dispatch.
+    ops_1gib = None
+    if not args.no_sweep and world == 1:
+        ops_1gib = []
+        for dt_name, tdt in (("int32", torch.int32), ("float32", torch.float32), ("float64", torch.float64)):
+            xv = x.view(tdt)
+            for op in ("sum", "min", "max") + (("sum_accurate",) if dt_name != "int32" else ()):
+                o1 = torch.empty(1, dtype=tdt, device=dev)
+
+                def launch_o(t, op=op, o1=o1):
+                    rb.reduce(t, op, out=o1, stream=stream, mode=args.mode)
+                sec = time_calls(launch_o, [xv] * 3, [xv] * 20, stream, repeats=2)
+                pp = rb.query_plan(dt_name, op, xv.numel(), in_ptr=xv.data_ptr(), mode=args.mode)
+                ops_1gib.append({"dtype": dt_name, "op": op, "us": round(sec * 1e6, 2),
+                                 "GBps": round(n * 4 / sec / 1e9, 1), "frac_of_peak": round(n * 4 / sec / 1e9 / peak, 4),
+                                 "variant": f"gc{pp['grid_combine']} g{pp['grid']}x{pp['block']} u{pp['unroll']} st{pp['stage']}"})
+
     # ---- many small arrays in one launch: batched rows of
     # the resident input, device time per call (graph), against one reduce()
     # per array (the sweep's per-call time at that length).
@@ -454,6 +472,7 @@ def main():
             line["sweep"] = sweep
             line["small_array_latency"] = latency
             line["batched"] = batched
+            line["ops_1GiB"] = ops_1gib
         if ncu_s is not None:
             line["ncu"] = {k: ncu_s[k] for k in ("source", "dram_pct_of_peak", "duration_us") if k in ncu_s}
         print(json.dumps(line), flush=True)

@@ -274,14 +274,28 @@ template <int OP> struct TrF64 {
 
 // ---- accurate sums: same bandwidth, tighter error --------
 // fp32 input, fp64 accumulation from the first add: error <= u_f|S| + (L+1) u_d sum|x|.
+// Per thread: Neumaier pairs (s, c) in fp32 -- FP32-pipe work only, since the
+// B200's FP64 pipe cannot convert and add 2^28 elements at HBM speed -- then
+// s and c are converted to fp64 once per thread (exactly) and everything above
+// the thread runs in fp64.  The per-thread residual is O(n_t u_f^2) sum|x|.
 struct TrF32Acc {
   using Elem = float;
   using Acc = double;
   using Grid = double;
+  using Part = float2;  // x = s, y = c
   static constexpr int VE = 8, NA = 8, kLaneWords = 1;
   __device__ static Acc ident() { return 0.0; }
+  __device__ static Part part_ident() { return make_float2(0.0f, 0.0f); }
+  __device__ static Acc part_to_acc(Part p) { return isfinite(p.x) ? (double)p.x + (double)p.y : (double)p.x; }
   __device__ static Acc comb(Acc a, Acc b) { return a + b; }
-  __device__ static void fold(Acc& a, uint32_t&, uint32_t w) { a += (double)__uint_as_float(w); }
+  __device__ static void fold(Part& a, uint32_t&, uint32_t w) {
+    const float x = __uint_as_float(w);
+    const float t = a.x + x;
+    const bool s_big = fabsf(a.x) >= fabsf(x);
+    const float big = s_big ? a.x : x, small = s_big ? x : a.x;
+    a.y += (big - t) + small;
+    a.x = t;
+  }
   __device__ static Acc warp(Acc v) { return warp_butterfly(v, [](double x, double y) { return x + y; }); }
   __device__ static Acc finish(Acc a, uint32_t) { return a; }
   __device__ static Grid to_grid(Acc a) { return a; }
@@ -341,10 +355,24 @@ template <int OP> struct Tr<DT_F64, OP> : TrF64<OP> {};
 template <> struct Tr<DT_F32, OP_SUMACC> : TrF32Acc {};
 template <> struct Tr<DT_F64, OP_SUMACC> : TrF64Acc {};
 
+// Per-thread accumulator ("part"): the traits' Part type if it declares one
+// (the fp32 accurate sum keeps Neumaier (s, c) pairs in fp32), else Acc.
+template <class T, class = void> struct PartOf {
+  using type = typename T::Acc;
+  __device__ static type ident() { return T::ident(); }
+  __device__ static typename T::Acc to_acc(type p) { return p; }
+};
+template <class T> struct PartOf<T, std::void_t<typename T::Part>> {
+  using type = typename T::Part;
+  __device__ static type ident() { return T::part_ident(); }
+  __device__ static typename T::Acc to_acc(type p) { return T::part_to_acc(p); }
+};
+template <class T> using Part = typename PartOf<T>::type;
+
 // Fold one 32-byte vector into the NA per-thread accumulators (lane k of the
 // vector goes to accumulator k: NA independent chains).
 template <class T>
-__device__ __forceinline__ void fold_vec(typename T::Acc (&a)[T::NA], uint32_t& aux, const uint32_t (&r)[8]) {
+__device__ __forceinline__ void fold_vec(Part<T> (&a)[T::NA], uint32_t& aux, const uint32_t (&r)[8]) {
   if constexpr (T::kLaneWords == 1) {
 #pragma unroll
     for (int k = 0; k < 8; ++k) T::fold(a[k], aux, r[k]);
@@ -355,14 +383,23 @@ __device__ __forceinline__ void fold_vec(typename T::Acc (&a)[T::NA], uint32_t& 
 }
 
 template <class T>
-__device__ __forceinline__ void fold_elem(typename T::Acc& a, uint32_t& aux, typename T::Elem e) {
+__device__ __forceinline__ void fold_elem(Part<T>& a, uint32_t& aux, typename T::Elem e) {
   if constexpr (T::kLaneWords == 1) T::fold(a, aux, *reinterpret_cast<const uint32_t*>(&e));
   else T::fold(a, aux, e);
 }
 
-// Pairwise tree over the NA accumulators (depth log2 NA).
 template <class T>
-__device__ __forceinline__ typename T::Acc thread_result(typename T::Acc (&a)[T::NA], uint32_t aux) {
+__device__ __forceinline__ void init_parts(Part<T> (&a)[T::NA]) {
+#pragma unroll
+  for (int k = 0; k < T::NA; ++k) a[k] = PartOf<T>::ident();
+}
+
+// Pairwise tree over the NA accumulators (depth log2 NA), in the Acc type.
+template <class T>
+__device__ __forceinline__ typename T::Acc thread_result(Part<T> (&p)[T::NA], uint32_t aux) {
+  typename T::Acc a[T::NA];
+#pragma unroll
+  for (int k = 0; k < T::NA; ++k) a[k] = PartOf<T>::to_acc(p[k]);
 #pragma unroll
   for (int w = T::NA / 2; w > 0; w >>= 1)
 #pragma unroll

@@ -138,9 +138,8 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(
   pdl_wait();
   if (blockIdx.x + kPdlTriggerWindow >= gridDim.x) pdl_trigger();
   if (p.gc == GC_CLUSTER) cluster_arrive_relaxed();  // phase 1: "this CTA has started"
-  Acc a[T::NA];
-#pragma unroll
-  for (int k = 0; k < T::NA; ++k) a[k] = T::ident();
+  Part<T> a[T::NA];
+  init_parts<T>(a);
   uint32_t aux = 0;
 
   const long long B = blockDim.x;

@@ -19,7 +19,7 @@ namespace rb {
 
 // Fold in[lo, hi) by `lanes` cooperating threads (this one is `lid`).
 template <class T, int U>
-__device__ __forceinline__ void fold_range(typename T::Acc (&a)[T::NA], uint32_t& aux, const char* base,
+__device__ __forceinline__ void fold_range(Part<T> (&a)[T::NA], uint32_t& aux, const char* base,
                                            long long lo, long long hi, int lid, int lanes) {
   using Elem = typename T::Elem;
   constexpr int s = sizeof(Elem);
@@ -100,9 +100,8 @@ __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
         hi = lo + p.seg_len;
       }
     }
-    Acc a[T::NA];
-#pragma unroll
-    for (int k = 0; k < T::NA; ++k) a[k] = T::ident();
+    Part<T> a[T::NA];
+    init_parts<T>(a);
     uint32_t aux = 0;
     fold_range<T, 4>(a, aux, p.in, lo, hi, lid, lanes);
     const Acc v = thread_result<T>(a, aux);

@@ -1,8 +1,10 @@
-"""REDUCE_SUM_ACCURATE: fp32 with fp64 accumulation and fp64
-with double-double accumulation, checked against the EXACT sum (math.fsum via
-oracle/ref.py): |r - S| <= u|S| + (L+1)*v*sum|x| with u the output unit
-roundoff and v the accumulator's (2^-53 for fp64 accumulation, 2^-100 for
-double-double), L the variant's chain length.  Plus cancellation pins a plain
+"""REDUCE_SUM_ACCURATE: fp32 with per-thread fp32 Neumaier
+pairs then fp64 above the thread, and fp64 with double-double accumulation,
+checked against the EXACT sum (math.fsum via oracle/ref.py):
+|r - S| <= u|S| + E*sum|x| with u the output unit roundoff and E the
+accumulation error: (L+1)^2 * 2^-48 for fp32 (compensated fp32 chains of
+length <= L, then fp64), (L+1) * 2^-100 for double-double; L is the variant's
+chain length.  Plus cancellation pins a plain
 sum fails, special values, every grid combine, segmented and host entry."""
 import math
 
@@ -23,9 +25,9 @@ def _rb():
 
 
 def _gate(dtype, S, A, L):
-    u = 2.0 ** -24 if dtype == "float32" else 2.0 ** -53
-    v = 2.0 ** -53 if dtype == "float32" else 2.0 ** -100
-    return u * abs(S) + (L + 1) * v * A + 1e-300
+    if dtype == "float32":
+        return 2.0 ** -24 * abs(S) + (L + 1) ** 2 * 2.0 ** -48 * A + 1e-300
+    return 2.0 ** -53 * abs(S) + (L + 1) * 2.0 ** -100 * A + 1e-300
 
 
 def _check(x, r, plan):
@@ -118,4 +120,4 @@ def test_accurate_segmented_and_host():
     xf = synth.make("float32", (1 << 24) + 7, "uniform01", 3)
     r = rb.reduce_host(xf, "sum_accurate")
     S = oracle.reduce(xf, "sum")
-    assert abs(float(r) - S.value) <= 2.0 ** -24 * abs(S.value) + 1e-6 * 0 + 4 * 2.0 ** -53 * S.abs_sum * 64
+    assert abs(float(r) - S.value) <= _gate("float32", S.value, S.abs_sum, 64)
