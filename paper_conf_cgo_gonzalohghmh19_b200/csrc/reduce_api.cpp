@@ -88,16 +88,20 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   if (dd && (o.block_combine == REDUCE_BC_SMEM_ATOMIC_WARP || o.block_combine == REDUCE_BC_SMEM_ATOMIC_ALL))
     return fail(REDUCE_ERR_INVALID_ARG, "fp64 accurate sums have no shared-atomic block combine");
 
-  // ---- S0: table lookup by ceil(log2(bytes)); the accurate sum uses the sum rows
-  const int op_row = op == REDUCE_SUM_ACCURATE ? REDUCE_SUM : op;
+  // ---- S0: table lookup by ceil(log2(bytes)); an op without tuned rows (the
+  // accurate sum, if the table predates it) falls back to the sum rows
   const unsigned long long bytes = (unsigned long long)n * (unsigned long long)s;
   const int lb = ilog2_ceil(bytes ? bytes : 1);
   const DispatchEntry* e = nullptr;
-  for (const DispatchEntry& r : kDispatch) {
-    if ((r.dtype < 0 || r.dtype == dtype) && (r.op < 0 || r.op == op_row) && (r.mode < 0 || r.mode == mode) &&
-        lb <= r.max_log2_bytes) {
-      e = &r;
-      break;
+  for (int pass = 0; pass < 2 && (e == nullptr || e->dtype < 0); ++pass) {
+    const int op_row = pass == 0 ? op : REDUCE_SUM;
+    if (pass == 1 && op != REDUCE_SUM_ACCURATE) break;
+    for (const DispatchEntry& r : kDispatch) {
+      if ((r.dtype < 0 || r.dtype == dtype) && (r.op < 0 || r.op == op_row) && (r.mode < 0 || r.mode == mode) &&
+          lb <= r.max_log2_bytes) {
+        if (e == nullptr || r.dtype >= 0) e = &r;
+        break;
+      }
     }
   }
   if (!e) e = &kDispatch[sizeof(kDispatch) / sizeof(kDispatch[0]) - 1];

@@ -28,13 +28,16 @@ sys.path.insert(0, os.path.join(ROOT, "tools"))
 
 ELEM = {"int32": 4, "float32": 4, "float64": 8}
 DT = {"int32": 0, "float32": 1, "float64": 2}
-OPC = {"sum": 0, "min": 1, "max": 2}
+OPC = {"sum": 0, "min": 1, "max": 2, "sum_accurate": 3}
 MODE = {"fast": 0, "deterministic": 1}
-MAXBLK = lambda dt, op, u: 512 if (u >= 8 or (dt == "float64" and op != "sum" and u >= 2)) else 1024
+MAXBLK = lambda dt, op, u: 512 if (u >= 8 or (dt == "float64" and op != "sum" and u >= 2)
+                                   or (op == "sum_accurate" and u >= 4)) else 1024
 
 
 def candidates(dtype, op, mode, lb):
     gcs = [1, 2, 3] if mode == "fast" else [2, 3]
+    if op == "sum_accurate" and dtype == "float64":
+        gcs = [g for g in gcs if g != 1]  # double-double: no value atomics
     out = []
     if lb <= 18:
         for blk, u in itertools.product((32, 128, 256, 512, 1024), (1, 2, 4)):
@@ -46,7 +49,7 @@ def candidates(dtype, op, mode, lb):
             if blk * u * 32 <= 128 * 1024:
                 out.append(dict(block=blk, unroll=u, grid_combine=gc, block_combine=0, grid=0, stage=2))
         for bc in (1, 2, 3):
-            if mode == "deterministic" and bc in (1, 2):
+            if (mode == "deterministic" or (op == "sum_accurate" and dtype == "float64")) and bc in (1, 2):
                 continue
             out.append(dict(block=256, unroll=2, grid_combine=gcs[0], block_combine=bc, grid=0))
     if 10 <= lb <= 26:
@@ -60,7 +63,9 @@ def candidates(dtype, op, mode, lb):
             out.append(dict(block=blk, unroll=4, grid_combine=gcs[0], block_combine=0, grid=g))
     for c in out:
         c.setdefault("stage", 1)
-    return [c for c in out if c["stage"] == 2 or c["block"] <= MAXBLK(dtype, op, c["unroll"])]
+    ok = lambda c: (c["block"] <= (512 if op == "sum_accurate" else 1024) if c["stage"] == 2
+                    else c["block"] <= MAXBLK(dtype, op, c["unroll"]))
+    return [c for c in out if ok(c)]
 
 
 def run(args):
