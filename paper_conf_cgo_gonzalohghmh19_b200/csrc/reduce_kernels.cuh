@@ -242,7 +242,8 @@ inline KParams make_params(const LaunchDesc& d) {
 // STAGE_SMEM needs block*U*32 bytes of dynamic shared memory (opt-in above 48 KB).
 inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& d, const KParams& p, cudaStream_t s) {
   const size_t smem = d.stage == STAGE_SMEM ? (size_t)d.block * d.unroll * kVecBytes : 0;
-  if (smem > 48 * 1024 || (d.gc == GC_CLUSTER && d.grid > 8)) {
+  // any dynamic tile opts in (static scratch + a 32 KB tile can already pass the 48 KB default)
+  if (smem > 0 || (d.gc == GC_CLUSTER && d.grid > 8)) {
     static std::mutex mu;
     static std::unordered_set<const void*> opted;
     std::lock_guard<std::mutex> lk(mu);
