@@ -73,6 +73,8 @@ def lib() -> ctypes.CDLL:
                 ("oracle_max_f64_bits", ctypes.c_uint64, [vp, sz]),
                 ("oracle_omp_sum_f32", ctypes.c_float, [vp, sz]),
                 ("oracle_omp_threads", ctypes.c_int, []),
+                ("oracle_histogram_i32", None, [vp, sz, ctypes.c_double, ctypes.c_double, ctypes.c_int, vp]),
+                ("oracle_histogram_f32", None, [vp, sz, ctypes.c_double, ctypes.c_double, ctypes.c_int, vp]),
             ]:
                 f = getattr(L, name)
                 f.restype = res
@@ -128,6 +130,18 @@ def reduce(x: np.ndarray, op: str) -> Result:
         b = int(f(p, n))
         return Result(np.uint64(b).view(np.float64), bits=b)
     raise TypeError(f"oracle: unsupported dtype {dt}")
+
+
+def histogram(x: np.ndarray, lo: float, hi: float, nbins: int) -> np.ndarray:
+    """counts[b] = #{lo <= x < hi, b = floor((x - lo) * nbins / (hi - lo))} (oracle.c)."""
+    x = np.ascontiguousarray(x)
+    counts = np.zeros(nbins, np.uint32)
+    f = lib().oracle_histogram_i32 if x.dtype == np.int32 else lib().oracle_histogram_f32
+    if x.dtype not in (np.int32, np.float32):
+        raise TypeError("histogram: int32 or float32 input")
+    f(ctypes.c_void_p(x.ctypes.data if x.size else 0), x.size, float(lo), float(hi), int(nbins),
+      ctypes.c_void_p(counts.ctypes.data))
+    return counts
 
 
 def omp_sum_f32(x: np.ndarray) -> float:

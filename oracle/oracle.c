@@ -138,6 +138,34 @@ uint64_t oracle_max_f64_bits(const double* x, size_t n) {
   uint64_t b; memcpy(&b, &m, 8); return b;
 }
 
+/* ------------------------------------------------------------ histogram --- */
+
+/* the paper motivates shared-memory atomics with histograms
+ * (P:L59).  Plain definition: counts[b] = #{ i : lo <= x_i < hi and
+ * b = floor((x_i - lo) * nbins / (hi - lo)) }, the bin computed in double with
+ * one subtraction, one multiplication and one division, each rounded to
+ * nearest, in that order (reading R13 -- the CUDA side takes the same
+ * decision in the same precision).  Elements outside [lo, hi) and NaN are not
+ * counted.  counts is overwritten. */
+static void hist_add(double x, double lo, double hi, int nbins, uint32_t* counts) {
+  if (!(x >= lo && x < hi)) return;
+  double t = x - lo;
+  t = t * (double)nbins;
+  t = t / (hi - lo);
+  long long b = (long long)floor(t);
+  if (b >= 0 && b < nbins) counts[b] += 1u;
+}
+
+void oracle_histogram_i32(const int32_t* x, size_t n, double lo, double hi, int nbins, uint32_t* counts) {
+  for (int b = 0; b < nbins; ++b) counts[b] = 0u;
+  for (size_t i = 0; i < n; ++i) hist_add((double)x[i], lo, hi, nbins, counts);
+}
+
+void oracle_histogram_f32(const float* x, size_t n, double lo, double hi, int nbins, uint32_t* counts) {
+  for (int b = 0; b < nbins; ++b) counts[b] = 0u;
+  for (size_t i = 0; i < n; ++i) hist_add((double)x[i], lo, hi, nbins, counts);
+}
+
 /* --------------------------------------------- paper-style CPU baseline -- */
 
 /* The paper's CPU comparison is an OpenMP 4.0 `reduce` pragma over fp32

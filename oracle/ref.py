@@ -72,3 +72,21 @@ def minmax_fp_bits(xs, op: str, width: int) -> int:
         return _bits(math.inf if op == "min" else -math.inf, width)
     pick = min(vals, key=_rank) if op == "min" else max(vals, key=_rank)
     return _bits(pick, width)
+
+
+def histogram(xs, lo, hi, nbins):
+    """Exact-rational histogram: b = floor((x - lo) * nbins / (hi - lo)) with
+    Fractions (no rounding at all).  Agrees with the double-precision rule of
+    oracle.c except where a rounding moves x across a bin edge, which the tests
+    avoid by choosing edges on exactly representable grids."""
+    from fractions import Fraction
+    counts = [0] * nbins
+    flo, fhi = Fraction(lo), Fraction(hi)
+    for v in xs:
+        v = float(v)
+        if v != v or not (lo <= v < hi):
+            continue
+        b = int((Fraction(v) - flo) * nbins / (fhi - flo))
+        if 0 <= b < nbins:
+            counts[b] += 1
+    return counts

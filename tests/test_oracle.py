@@ -243,3 +243,33 @@ def test_omp_baseline_runs():
     x = synth.make("float32", 1 << 16, "ones", 0)
     assert oracle.omp_sum_f32(x) == float(1 << 16)
     assert oracle.omp_threads() >= 1
+
+
+# ------------------------------------------------------------ histogram (N4)
+def test_histogram_closed_forms():
+    # iota over [0, 1024) into 16 bins: 64 each; out-of-range values not counted
+    x = np.arange(-100, 1124, dtype=np.int32)
+    c = oracle.histogram(x, 0, 1024, 16)
+    assert c.tolist() == [64] * 16
+    assert oracle.histogram(np.ones(1000, np.int32), 0, 10, 10).tolist() == [0, 1000] + [0] * 8
+    assert oracle.histogram(np.zeros(0, np.int32), 0, 10, 3).tolist() == [0, 0, 0]
+    f = np.array([np.nan, np.inf, -np.inf, 0.5, 0.25, 0.999, 1.0, -0.0], np.float32)
+    assert oracle.histogram(f, 0.0, 1.0, 4).tolist() == [1, 1, 1, 1]  # -0.0 is in [0, 1)
+
+
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+@pytest.mark.parametrize("nbins", [1, 7, 64, 1000])
+def test_histogram_vs_exact_rational(dtype, nbins):
+    rng = np.random.Generator(np.random.PCG64(nbins))
+    if dtype == "int32":
+        x = rng.integers(-50, 5000, 3000).astype(np.int32)
+        lo, hi = 0, 4096  # power-of-two range: every edge is exact
+    else:
+        x = (rng.random(3000, dtype=np.float32) * 2 - 0.5).astype(np.float32)
+        lo, hi = 0.0, 1.0
+    c = oracle.histogram(x, lo, hi, nbins)
+    want = ref.histogram(x, lo, hi, nbins)
+    if nbins in (1, 64):  # power-of-two bins on a power-of-two range: no rounding anywhere
+        assert c.tolist() == want
+    assert int(c.sum()) == sum(want) == int(((x >= lo) & (x < hi)).sum())
+    assert np.abs(c.astype(np.int64) - np.array(want)).sum() <= 2 * max(1, nbins // 100) + 2
