@@ -408,6 +408,19 @@ def main():
                                  "GBps": round(n * 4 / sec / 1e9, 1), "frac_of_peak": round(n * 4 / sec / 1e9 / peak, 4),
                                  "variant": f"gc{pp['grid_combine']} g{pp['grid']}x{pp['block']} u{pp['unroll']} st{pp['stage']}"})
 
+    # ---- histogram of the resident 1 GiB, 256 and 65536 bins
+    hist = None
+    if not args.no_sweep and world == 1:
+        hist = []
+        for nbins in (256, 65536):
+            hc = torch.empty(nbins, dtype=torch.int32, device=dev)
+
+            def launch_h(t, hc=hc, nbins=nbins):
+                rb.histogram(t, 0.0, 1.0, nbins, counts=hc, stream=stream)
+            sec = time_calls(launch_h, [x] * 2, [x] * 10, stream, repeats=2)
+            hist.append({"dtype": "float32", "n": n, "nbins": nbins, "us": round(sec * 1e6, 2),
+                         "GBps": round(n * 4 / sec / 1e9, 1)})
+
     # ---- many small arrays in one launch: batched rows of
     # the resident input, device time per call (graph), against one reduce()
     # per array (the sweep's per-call time at that length).
@@ -473,6 +486,7 @@ def main():
             line["small_array_latency"] = latency
             line["batched"] = batched
             line["ops_1GiB"] = ops_1gib
+            line["histogram"] = hist
         if ncu_s is not None:
             line["ncu"] = {k: ncu_s[k] for k in ("source", "dram_pct_of_peak", "duration_us") if k in ncu_s}
         print(json.dumps(line), flush=True)

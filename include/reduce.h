@@ -198,6 +198,20 @@ int reduce_segmented(int dtype, int op, const void* in, const int64_t* offsets, 
 int reduce_batched(int dtype, int op, const void* in, size_t seg_len, size_t num_segments, void* out,
                    reduce_stream_t stream, const reduce_opts_t* opts);
 
+/* ---- histogram -------------------------------------------
+ * The workload the paper motivates shared-memory atomics with (P:L59,
+ * P:L253-L255): counts[b] = #{ i : lo <= in[i] < hi and
+ * b = floor((in[i] - lo) * nbins / (hi - lo)) } for int32 or fp32 input, the bin
+ * decided in fp64 (one subtraction, one multiplication, one division, each
+ * rounded to nearest, in that order); values outside [lo, hi) and NaN are not
+ * counted.  `counts` is a DEVICE array of nbins uint32, overwritten (a memset
+ * node precedes the kernel).  Per-block shared-memory histograms with
+ * shared atomics (the paper's "VA1" codelet per bin), merged with global
+ * atomics; nbins > 16384 counts in global memory directly.  Counts are exact
+ * (integer atomics commute). */
+int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, int nbins, uint32_t* counts,
+                     reduce_stream_t stream);
+
 /* ---- sharded mode over NCCL (one process per GPU) -------------------------
  * reduce_multi: every rank of `comm` calls it with its own local shard
  * (n_local may differ per rank, and may be 0); each rank's local result is

@@ -34,7 +34,7 @@ ABI_SYMBOLS = (
     "reduce_get_mode", "reduce_host", "reduce_multi", "reduce_multi_ex",
     "reduce_comm_unique_id_bytes", "reduce_comm_get_unique_id", "reduce_comm_init",
     "reduce_comm_destroy", "reduce_status_string", "reduce_last_error", "reduce_version",
-    "reduce_shutdown", "reduce_segmented", "reduce_batched",
+    "reduce_shutdown", "reduce_segmented", "reduce_batched", "reduce_histogram",
 )
 
 
@@ -90,6 +90,7 @@ def _load() -> ctypes.CDLL:
         "reduce_shutdown": (None, []),
         "reduce_segmented": (i, [i, i, vp, vp, sz, vp, vp, opts_p]),
         "reduce_batched": (i, [i, i, vp, sz, sz, vp, vp, opts_p]),
+        "reduce_histogram": (i, [i, vp, sz, ctypes.c_double, ctypes.c_double, i, vp, vp]),
     }
     for name, (res, args) in sigs.items():
         f = getattr(L, name)
@@ -207,6 +208,18 @@ def reduce_batched(x, op="sum", out=None, stream=None, **opt_kw):
                             _stream_handle(stream, x.device), ctypes.byref(opts) if opts is not None else None)
     _check(st, "reduce_batched")
     return out
+
+
+def histogram(x, lo: float, hi: float, nbins: int, counts=None, stream=None):
+    """counts[b] = #{lo <= x < hi, b = floor((x - lo) * nbins / (hi - lo))} (CUDA int32/fp32 tensor)."""
+    import torch
+    dt = _torch_dtype_code(x)
+    if counts is None:
+        counts = torch.empty(nbins, dtype=torch.int32, device=x.device)  # bit pattern of uint32 counts
+    st = lib.reduce_histogram(dt, x.data_ptr() or None, x.numel(), float(lo), float(hi), int(nbins),
+                              counts.data_ptr(), _stream_handle(stream, x.device))
+    _check(st, "reduce_histogram")
+    return counts
 
 
 def query_plan(dtype, op, n: int, in_ptr: int = 0, **opt_kw) -> dict:

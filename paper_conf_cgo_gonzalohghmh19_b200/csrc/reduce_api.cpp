@@ -379,6 +379,37 @@ int reduce_batched(int dtype, int op, const void* in, size_t seg_len, size_t num
   return segmented_common(dtype, op, in, nullptr, seg_len, num_segments, out, stream, opts);
 }
 
+int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, int nbins, uint32_t* counts,
+                     reduce_stream_t stream) {
+  if (dtype != REDUCE_INT32 && dtype != REDUCE_FLOAT32)
+    return fail(REDUCE_ERR_INVALID_ARG, "histogram input must be REDUCE_INT32 or REDUCE_FLOAT32");
+  if (nbins < 1 || nbins > (1 << 24)) return fail(REDUCE_ERR_INVALID_ARG, "nbins must be in [1, 2^24]");
+  if (!(lo < hi) || !std::isfinite(lo) || !std::isfinite(hi)) return fail(REDUCE_ERR_INVALID_ARG, "need finite lo < hi");
+  if (counts == nullptr || ((uintptr_t)counts % 4u) != 0) return fail(REDUCE_ERR_INVALID_ARG, "counts is NULL or misaligned");
+  if (n > 0 && (in == nullptr || ((uintptr_t)in % 4u) != 0))
+    return fail(REDUCE_ERR_INVALID_ARG, "in is NULL or not aligned to the element size");
+  HistParams p;
+  p.in = (const char*)in;
+  size_t head = 0;
+  if (n > 0) {
+    const uintptr_t mis = (uintptr_t)in % 32u;
+    head = mis ? (32u - mis) / 4u : 0;
+    if (head > n) head = n;
+  }
+  p.body = (const char*)in + head * 4;
+  p.body_vecs = (n - head) / 8;
+  p.head = (int)head;
+  p.tail = (int)((n - head) % 8);
+  p.lo = lo;
+  p.hi = hi;
+  p.range = hi - lo;
+  p.nbins = nbins;
+  p.counts = counts;
+  cudaError_t e = launch_histogram(dtype, p, 256, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "histogram launch");
+  return REDUCE_OK;
+}
+
 int reduce(int dtype, int op, const void* in, size_t n, void* out, reduce_stream_t stream) {
   return reduce_ex(dtype, op, in, n, out, stream, nullptr);
 }

@@ -17,6 +17,15 @@ cudaError_t segmented_i32(int, const SegParams&, int, int, cudaStream_t);
 cudaError_t segmented_f32(int, const SegParams&, int, int, cudaStream_t);
 cudaError_t segmented_f64(int, const SegParams&, int, int, cudaStream_t);
 
+cudaError_t histogram_i32(const HistParams&, int, cudaStream_t);
+cudaError_t histogram_f32(const HistParams&, int, cudaStream_t);
+
+cudaError_t launch_histogram(int dtype, const HistParams& p, int block, cudaStream_t s) {
+  if (dtype == 0) return histogram_i32(p, block, s);
+  if (dtype == 1) return histogram_f32(p, block, s);
+  return cudaErrorInvalidValue;
+}
+
 cudaError_t launch_segmented(int dtype, int op, const SegParams& p, int group, int block, cudaStream_t s) {
   switch (dtype) {
     case 0: return segmented_i32(op, p, group, block, s);

@@ -59,6 +59,18 @@ struct SegParams {
 // group: lanes per segment (8 or 32) or 0 = one block per segment.
 cudaError_t launch_segmented(int dtype, int op, const SegParams& p, int group, int block, cudaStream_t s);
 
+// One histogram launch, see reduce_histogram.cuh.
+struct HistParams {
+  const char* in;               // element-aligned input (4-byte elements)
+  const char* body;             // first 32-byte-aligned element
+  unsigned long long body_vecs;
+  int head, tail;
+  double lo, hi, range;         // range = hi - lo
+  int nbins;
+  unsigned* counts;             // device, nbins
+};
+cudaError_t launch_histogram(int dtype, const HistParams& p, int block, cudaStream_t s);
+
 // Size in bytes of the Grid (cross-block) type of (dtype, op).
 int grid_value_bytes(int dtype, int op);
 

@@ -142,6 +142,16 @@ def test_segmented_argument_validation():
     assert L.reduce_batched(1, 0, None, 10, 0, None, None, None) == 0             # no segments: no-op
 
 
+def test_histogram_argument_validation():
+    L = rb.lib
+    assert L.reduce_histogram(2, 4096, 10, 0.0, 1.0, 8, 8192, None) == 1   # fp64 input
+    assert L.reduce_histogram(0, 4096, 10, 1.0, 1.0, 8, 8192, None) == 1   # lo == hi
+    assert L.reduce_histogram(0, 4096, 10, 0.0, float("inf"), 8, 8192, None) == 1
+    assert L.reduce_histogram(0, 4096, 10, 0.0, 1.0, 0, 8192, None) == 1   # nbins
+    assert L.reduce_histogram(0, 4096, 10, 0.0, 1.0, 8, None, None) == 1   # counts NULL
+    assert L.reduce_histogram(0, 4098, 10, 0.0, 1.0, 8, 8192, None) == 1   # misaligned
+
+
 def test_mode_default_roundtrip():
     old = rb.get_mode()
     rb.set_mode("deterministic")
