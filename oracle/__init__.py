@@ -133,7 +133,8 @@ def reduce(x: np.ndarray, op: str) -> Result:
 
 
 def histogram(x: np.ndarray, lo: float, hi: float, nbins: int) -> np.ndarray:
-    """counts[b] = #{lo <= x < hi, b = floor((x - lo) * nbins / (hi - lo))} (oracle.c)."""
+    """Histogram counts (oracle.c, reading R13): exact integer bins for int32,
+    fp32 bins floor(fl32(fl32(x - lo) * scale)) for fp32."""
     x = np.ascontiguousarray(x)
     counts = np.zeros(nbins, np.uint32)
     f = lib().oracle_histogram_i32 if x.dtype == np.int32 else lib().oracle_histogram_f32

@@ -141,29 +141,39 @@ uint64_t oracle_max_f64_bits(const double* x, size_t n) {
 /* ------------------------------------------------------------ histogram --- */
 
 /* the paper motivates shared-memory atomics with histograms
- * (P:L59).  Plain definition: counts[b] = #{ i : lo <= x_i < hi and
- * b = floor((x_i - lo) * nbins / (hi - lo)) }, the bin computed in double with
- * one subtraction, one multiplication and one division, each rounded to
- * nearest, in that order (reading R13 -- the CUDA side takes the same
- * decision in the same precision).  Elements outside [lo, hi) and NaN are not
- * counted.  counts is overwritten. */
-static void hist_add(double x, double lo, double hi, int nbins, uint32_t* counts) {
-  if (!(x >= lo && x < hi)) return;
-  double t = x - lo;
-  t = t * (double)nbins;
-  t = t / (hi - lo);
-  long long b = (long long)floor(t);
-  if (b >= 0 && b < nbins) counts[b] += 1u;
-}
-
+ * (P:L59).  Plain definition (reading R13), bins decided
+ * in the input's own arithmetic -- the CUDA side takes the same decisions:
+ *   int32: lo, hi integers; x counted iff lo <= x < hi, in bin
+ *          b = floor((x - lo) * nbins / (hi - lo))   (exact integer arithmetic);
+ *   fp32 : lo_f = (float)lo, hi_f = (float)hi, scale = (float)(nbins / (hi - lo))
+ *          (the quotient in double, then rounded to float); x counted iff
+ *          lo_f <= x < hi_f and 0 <= b < nbins with
+ *          b = floor(fl32(fl32(x - lo_f) * scale))   (two fp32 RN operations).
+ * NaN is never counted.  counts is overwritten. */
 void oracle_histogram_i32(const int32_t* x, size_t n, double lo, double hi, int nbins, uint32_t* counts) {
   for (int b = 0; b < nbins; ++b) counts[b] = 0u;
-  for (size_t i = 0; i < n; ++i) hist_add((double)x[i], lo, hi, nbins, counts);
+  const long long l = (long long)lo, h = (long long)hi;
+  const unsigned long long range = (unsigned long long)(h - l);
+  for (size_t i = 0; i < n; ++i) {
+    const long long v = (long long)x[i];
+    if (v < l || v >= h) continue;
+    const unsigned long long num = (unsigned long long)(v - l) * (unsigned long long)nbins;
+    counts[num / range] += 1u;
+  }
 }
 
 void oracle_histogram_f32(const float* x, size_t n, double lo, double hi, int nbins, uint32_t* counts) {
   for (int b = 0; b < nbins; ++b) counts[b] = 0u;
-  for (size_t i = 0; i < n; ++i) hist_add((double)x[i], lo, hi, nbins, counts);
+  const float lo_f = (float)lo, hi_f = (float)hi;
+  const float scale = (float)((double)nbins / (hi - lo));
+  for (size_t i = 0; i < n; ++i) {
+    const float v = x[i];
+    if (!(v >= lo_f && v < hi_f)) continue;
+    volatile float d = v - lo_f;   /* each operation rounded to fp32, no contraction */
+    volatile float t = d * scale;
+    const long long b = (long long)floorf(t);
+    if (b >= 0 && b < nbins) counts[b] += 1u;
+  }
 }
 
 /* --------------------------------------------- paper-style CPU baseline -- */

@@ -76,9 +76,9 @@ def minmax_fp_bits(xs, op: str, width: int) -> int:
 
 def histogram(xs, lo, hi, nbins):
     """Exact-rational histogram: b = floor((x - lo) * nbins / (hi - lo)) with
-    Fractions (no rounding at all).  Agrees with the double-precision rule of
-    oracle.c except where a rounding moves x across a bin edge, which the tests
-    avoid by choosing edges on exactly representable grids."""
+    Fractions (no rounding at all).  Equal to oracle.c's integer rule for int32;
+    for fp32 it differs only where an fp32 rounding moves x across a bin edge
+    (none when nbins and hi - lo are powers of two)."""
     from fractions import Fraction
     counts = [0] * nbins
     flo, fhi = Fraction(lo), Fraction(hi)
