@@ -201,10 +201,11 @@ int reduce_batched(int dtype, int op, const void* in, size_t seg_len, size_t num
 /* ---- histogram -------------------------------------------
  * The workload the paper motivates shared-memory atomics with (P:L59,
  * P:L253-L255): counts[b] = #{ i : lo <= in[i] < hi and
- * b = floor((in[i] - lo) * nbins / (hi - lo)) } for int32 or fp32 input, the bin
- * decided in fp64 (one subtraction, one multiplication, one division, each
- * rounded to nearest, in that order); values outside [lo, hi) and NaN are not
- * counted.  `counts` is a DEVICE array of nbins uint32, overwritten (a memset
+ * b = floor((in[i] - lo) * nbins / (hi - lo)) }.  int32 input: lo and hi must
+ * be integers (|.| <= 2^32) and the bin is exact integer arithmetic.  fp32
+ * input: with lo_f = (float)lo, hi_f = (float)hi, scale = (float)(nbins/(hi-lo)),
+ * x is counted iff lo_f <= x < hi_f, in bin floor(fl32(fl32(x - lo_f) * scale))
+ * when that is in [0, nbins).  NaN is never counted.  `counts` is a DEVICE array of nbins uint32, overwritten (a memset
  * node precedes the kernel).  Per-block shared-memory histograms with
  * shared atomics (the paper's "VA1" codelet per bin), merged with global
  * atomics; nbins > 16384 counts in global memory directly.  Counts are exact

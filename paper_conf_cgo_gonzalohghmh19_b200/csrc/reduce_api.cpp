@@ -400,9 +400,18 @@ int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, 
   p.body_vecs = (n - head) / 8;
   p.head = (int)head;
   p.tail = (int)((n - head) % 8);
-  p.lo = lo;
-  p.hi = hi;
-  p.range = hi - lo;
+  if (dtype == REDUCE_INT32) {
+    if (lo != std::floor(lo) || hi != std::floor(hi) || lo < -4294967296.0 || hi > 4294967296.0)
+      return fail(REDUCE_ERR_INVALID_ARG, "int32 histograms need integer lo, hi within +-2^32");
+    p.lo_i = (long long)lo;
+    p.hi_i = (long long)hi;
+    p.range_i = (unsigned long long)(p.hi_i - p.lo_i);
+    p.magic = ~0ull / p.range_i;
+  } else {
+    p.lo_f = (float)lo;
+    p.hi_f = (float)hi;
+    p.scale_f = (float)((double)nbins / (hi - lo));
+  }
   p.nbins = nbins;
   p.counts = counts;
   cudaError_t e = launch_histogram(dtype, p, 256, (cudaStream_t)stream);

@@ -65,7 +65,10 @@ struct HistParams {
   const char* body;             // first 32-byte-aligned element
   unsigned long long body_vecs;
   int head, tail;
-  double lo, hi, range;         // range = hi - lo
+  long long lo_i, hi_i;         // int32 input: integer bounds
+  unsigned long long range_i;   //   hi_i - lo_i
+  unsigned long long magic;     //   floor((2^64 - 1) / range_i): quotient by multiply-high
+  float lo_f, hi_f, scale_f;    // fp32 input: (float)lo, (float)hi, (float)(nbins / (hi - lo))
   int nbins;
   unsigned* counts;             // device, nbins
 };

@@ -150,6 +150,7 @@ def test_histogram_argument_validation():
     assert L.reduce_histogram(0, 4096, 10, 0.0, 1.0, 0, 8192, None) == 1   # nbins
     assert L.reduce_histogram(0, 4096, 10, 0.0, 1.0, 8, None, None) == 1   # counts NULL
     assert L.reduce_histogram(0, 4098, 10, 0.0, 1.0, 8, 8192, None) == 1   # misaligned
+    assert L.reduce_histogram(0, 4096, 10, 0.5, 10.0, 8, 8192, None) == 1  # int32 needs integer bounds
 
 
 def test_mode_default_roundtrip():

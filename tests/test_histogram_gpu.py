@@ -18,13 +18,13 @@ def _rb():
 
 
 @pytest.mark.parametrize("dtype", ["int32", "float32"])
-@pytest.mark.parametrize("nbins", [1, 7, 256, 1000, 16384, 16385, 100000])
+@pytest.mark.parametrize("nbins", [1, 7, 256, 1000, 16384, 16385, 100000, 1 << 20])
 def test_histogram_bit_exact(dtype, nbins):
     rb = _rb()
     for k, n in enumerate([0, 1, 13, 4097, (1 << 20) + 3]):
         if dtype == "int32":
             x = synth.make("int32", n, "int_small", 40 + k)
-            lo, hi = -900.0, 1000.0 - 0.5 * k
+            lo, hi = -900.0, 1000.0 - 7 * k
         else:
             x = synth.make("float32", n, "uniform_pm1", 40 + k)
             lo, hi = -0.75, 0.8 + 0.01 * k
