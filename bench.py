@@ -408,6 +408,24 @@ def main():
                                  "GBps": round(n * 4 / sec / 1e9, 1), "frac_of_peak": round(n * 4 / sec / 1e9 / peak, 4),
                                  "variant": f"gc{pp['grid_combine']} g{pp['grid']}x{pp['block']} u{pp['unroll']} st{pp['stage']}"})
 
+    # ---- BASELINE configs[4] at k = 1: one 8 GiB (2^31 fp32) array on one GPU
+    # (64-bit indexing); timing only (its parity is tests/test_parity_gpu.py's
+    # full-size test), so the array is drawn on the device.
+    big = None
+    if not args.no_sweep and world == 1:
+        xb = torch.rand(1 << 31, dtype=torch.float32, device=dev, generator=torch.Generator(dev).manual_seed(2019))
+        ob = torch.empty(1, dtype=torch.float32, device=dev)
+
+        def launch_big(t):
+            rb.reduce(t, "sum", out=ob, stream=stream, mode=args.mode)
+        sec = time_calls(launch_big, [xb] * 2, [xb] * 10, stream, repeats=2)
+        pb = rb.query_plan("float32", "sum", xb.numel(), in_ptr=xb.data_ptr(), mode=args.mode)
+        big = {"n": 1 << 31, "bytes": (1 << 31) * 4, "us": round(sec * 1e6, 1),
+               "GBps": round((1 << 31) * 4 / sec / 1e9, 1), "frac_of_peak": round((1 << 31) * 4 / sec / 1e9 / peak, 4),
+               "variant": f"gc{pb['grid_combine']} g{pb['grid']}x{pb['block']} u{pb['unroll']} st{pb['stage']}"}
+        del xb
+        torch.cuda.empty_cache()
+
     # ---- histogram of the resident 1 GiB, 256 and 65536 bins
     hist = None
     if not args.no_sweep and world == 1:
@@ -487,6 +505,7 @@ def main():
             line["batched"] = batched
             line["ops_1GiB"] = ops_1gib
             line["histogram"] = hist
+            line["config5_8GiB_one_gpu"] = big
         if ncu_s is not None:
             line["ncu"] = {k: ncu_s[k] for k in ("source", "dram_pct_of_peak", "duration_us") if k in ncu_s}
         print(json.dumps(line), flush=True)
