@@ -17,6 +17,17 @@ for dt in (torch.int32, torch.float32, torch.float64):
             for kw in (dict(), dict(mode="deterministic"), dict(grid_combine=3), dict(grid_combine=4, grid=8),
                        dict(stage="smem", unroll=8, block=256), dict(block_combine=1), dict(block_combine=3, block=128)):
                 rb.reduce(x, op, **kw)
+        if dt != torch.int32:
+            rb.reduce(x, "sum_accurate")
+            rb.reduce(x, "sum_accurate", mode="deterministic")
+    offs = torch.tensor([0, 0, 1, 33, 100, 4097], dtype=torch.int64, device="cuda")
+    base = torch.arange(5000, device="cuda").to(dt)[1:]
+    for g in (0, 1, 2, 3):
+        rb.reduce_segmented(base, offs, "sum", seg_group=g)
+        rb.reduce_batched(base[:4096].view(64, 64), "max", seg_group=g)
+    if dt != torch.float64:
+        for nb in (7, 20000, 1 << 20):
+            rb.histogram(base, 0, 4000, nb)
 torch.cuda.synchronize()
 print("ok")
 PY
