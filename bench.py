@@ -344,6 +344,11 @@ def main():
     if not args.no_sweep and world == 1:
         sys.path.insert(0, os.path.join(ROOT, "tools"))
         from cudatiming import time_calls, disjoint_regions
+        try:
+            from tests import cub as cubref
+            cubref.lib()
+        except Exception:
+            cubref = None
         outs = torch.empty(4096, dtype=torch.float32, device=dev)
         sweep = []
         for k in range(6, 29, 2):
@@ -358,7 +363,17 @@ def main():
                 rb.reduce(t, "sum", out=outs[ctr[0]:ctr[0] + 1], stream=stream, mode=args.mode)
             sec = time_calls(launch, warm, timed, stream, repeats=3)
             gbs = m * 4 / sec / 1e9
+            cub_sec = None
+            if cubref is not None:  # the paper's comparison system, on the same device (context)
+                def launch_cub(t):
+                    ctr[0] = (ctr[0] + 1) % 4096
+                    cubref.reduce(1, 0, t.data_ptr(), t.numel(), outs[ctr[0]:ctr[0] + 1].data_ptr(), stream.cuda_stream)
+                cubref.reduce(1, 0, timed[0].data_ptr(), m, outs.data_ptr(), stream.cuda_stream)  # size temp storage
+                torch.cuda.synchronize(dev)
+                cub_sec = time_calls(launch_cub, warm, timed, stream, repeats=3)
             sweep.append({"n": m, "us": round(sec * 1e6, 3), "GBps": round(gbs, 1),
+                          "cub_us": None if cub_sec is None else round(cub_sec * 1e6, 3),
+                          "speedup_vs_cub": None if cub_sec is None else round(cub_sec / sec, 3),
                           "elements_per_s": round(m / sec, 1), "frac_of_peak": round(gbs / peak, 4),
                           "variant": f"gc{p['grid_combine']} g{p['grid']}x{p['block']} u{p['unroll']}"})
         latency = []
