@@ -133,10 +133,14 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(
   using Acc = typename T::Acc;
   // Programmatic dependent launch: this grid may be resident before the
   // previous kernel of the stream has finished; nothing is read or written
-  // before the dependency resolves.  Blocks of the last wave allow the next
-  // kernel to be scheduled onto the SMs as this grid drains.
+  // before the dependency resolves.  The next kernel may be scheduled once
+  // every block has triggered: in a many-wave grid the last wave triggers at
+  // its start (the next grid fills SMs as this one drains); in a one-wave or
+  // persistent grid every block triggers after its main loop (triggering at
+  // the start would park the next grid's CTAs on the SMs for the whole run).
   pdl_wait();
-  if (blockIdx.x + kPdlTriggerWindow >= gridDim.x) pdl_trigger();
+  const bool early_trigger = gridDim.x > kPdlTriggerWindow && blockIdx.x + kPdlTriggerWindow >= gridDim.x;
+  if (early_trigger) pdl_trigger();
   if (p.gc == GC_CLUSTER) cluster_arrive_relaxed();  // phase 1: "this CTA has started"
   Part<T> a[T::NA];
   init_parts<T>(a);
@@ -188,6 +192,7 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(
       }
     }
   }
+  if (!early_trigger && gridDim.x <= kPdlTriggerWindow) pdl_trigger();
   if (blockIdx.x == gridDim.x - 1) {
     using Elem = typename T::Elem;
     const int t = threadIdx.x;

@@ -66,7 +66,6 @@ __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
   pdl_wait();
-  pdl_trigger();  // persistent grid: every block is resident from the start
   const int lane = threadIdx.x & 31;
   long long first, step;
   int lid, lanes;
@@ -119,6 +118,7 @@ __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
       __syncthreads();  // block_combine's shared scratch is reused next iteration
     }
   }
+  pdl_trigger();  // persistent grid: let the next kernel in only as this one finishes
 }
 
 template <int DT, int OP>
