@@ -55,6 +55,17 @@ constexpr unsigned kPdlTriggerWindow = 148u * 8u;  // ~ one full wave of residen
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
+// Ticket increment with acquire-release semantics at GPU scope: the release
+// half publishes this thread's earlier stores / reductions (the block's
+// partial) before the increment, the acquire half makes every earlier
+// publisher's data visible to the thread that draws the last ticket.  Replaces
+// __threadfence() (fence.sc.gpu) + a relaxed atomic on the combine's critical path.
+__device__ __forceinline__ unsigned ticket_acq_rel(unsigned* t) {
+  unsigned old;
+  asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(old) : "l"(t) : "memory");
+  return old;
+}
+
 // Split cluster barrier (all threads of every CTA of the cluster take part).
 __device__ __forceinline__ void cluster_arrive_relaxed() {
   asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
@@ -458,24 +469,25 @@ __device__ __forceinline__ typename T::Grid block_combine(typename T::Acc v) {
 }
 
 // Fixed-order reduction of `count` Grid values by the whole block: thread t
-// folds t, t+B, t+2B, ... then a shared tree over the B thread values.  Reads
-// with ld.global.cg (L2) since the values were written by other SMs.
+// folds t, t+B, t+2B, ... then a warp butterfly, the warps' results meet in
+// shared memory and warp 0 butterflies them (two barriers, deterministic).
+// Reads with ld.global.cg (L2) since the values were written by other SMs.
 template <class T>
 __device__ __forceinline__ typename T::Grid reduce_grid_values(const typename T::Grid* vals, long long count) {
   using Grid = typename T::Grid;
-  __shared__ Grid gtmp[1024];
+  __shared__ Grid gpart[32];
   Grid x = T::gident();
   for (long long i = threadIdx.x; i < count; i += blockDim.x) x = T::gcomb(x, __ldcg(vals + i));
-  gtmp[threadIdx.x] = x;
+  x = T::gwarp(x);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+  __syncthreads();  // gpart may still be read by a previous use in this block
+  if (lane == 0) gpart[wid] = x;
   __syncthreads();
-  int p2 = 1;
-  while (p2 < (int)blockDim.x) p2 <<= 1;
-  for (int s = p2 >> 1; s > 0; s >>= 1) {
-    if ((int)threadIdx.x < s && (int)threadIdx.x + s < (int)blockDim.x)
-      gtmp[threadIdx.x] = T::gcomb(gtmp[threadIdx.x], gtmp[threadIdx.x + s]);
-    __syncthreads();
+  if (wid == 0) {
+    Grid y = lane < nw ? gpart[lane] : T::gident();
+    x = T::gwarp(y);
   }
-  return gtmp[0];
+  return x;  // valid in thread 0
 }
 
 }  // namespace rb

@@ -90,13 +90,11 @@ __device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& 
     if (threadIdx.x == 0) {
       Grid* slot = (Grid*)((char*)p.slots + (size_t)(blockIdx.x % p.nslots) * kSlotBytes);
       T::gred(slot, g);
-      __threadfence();
-      unsigned tk = atomicAdd(p.ticket, 1u);
+      const unsigned tk = ticket_acq_rel(p.ticket);  // release: the red above; acquire: everyone's
       s_last = (tk == gridDim.x - 1);
     }
     __syncthreads();
     if (s_last && threadIdx.x < 32) {
-      __threadfence();
       const int lane = threadIdx.x;
       Grid x = T::gident();
       if (lane < p.nslots) x = T::gexch((Grid*)((char*)p.slots + (size_t)lane * kSlotBytes), T::gident());
@@ -112,13 +110,11 @@ __device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& 
   // order (deterministic; the only atomic touches the integer ticket).
   if (threadIdx.x == 0) {
     ((Grid*)p.partials)[blockIdx.x] = g;
-    __threadfence();
-    unsigned tk = atomicAdd(p.ticket, 1u);
+    const unsigned tk = ticket_acq_rel(p.ticket);  // release: the store above; acquire: everyone's
     s_last = (tk == gridDim.x - 1);
   }
   __syncthreads();
   if (s_last) {
-    __threadfence();
     Grid x = reduce_grid_values<T>((const Grid*)p.partials, gridDim.x);
     if (threadIdx.x == 0) {
       store_out<T>(x, p);
