@@ -126,7 +126,9 @@ typedef struct {
                          (power of two for SMEM_TREE) */
   int unroll;         /* 32-byte vectors per thread per tile: 0 = auto, else 1,2,4,8
                          (register staging) or 4,8,16 (shared-memory staging) */
-  int grid;           /* 0 = auto (one block per tile, capped), else max blocks;
+  int grid;           /* 0 = auto (the dispatch table's grid cap when the launch shape
+                         is also the table's, else one block per tile), -1 = one
+                         block per tile, > 0 = at most this many blocks (persistent);
                          for REDUCE_GC_CLUSTER: the cluster size, 1..16 (0 = 16) */
   int seg_group;      /* reduce_segmented / reduce_batched only: 0 = auto (8 lanes per
                          segment for uniform segments <= 128 elements, one warp for

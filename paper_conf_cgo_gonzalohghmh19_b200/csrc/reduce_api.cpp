@@ -74,7 +74,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   if (o.stage < 0 || o.stage > 2) return fail(REDUCE_ERR_INVALID_ARG, "stage must be 0, 1 or 2");
   if (o.block != 0 && (o.block < 32 || o.block > 1024 || o.block % 32 != 0))
     return fail(REDUCE_ERR_INVALID_ARG, "block must be 0 or a multiple of 32 in [32, 1024]");
-  if (o.grid < 0) return fail(REDUCE_ERR_INVALID_ARG, "grid must be >= 0");
+  if (o.grid < -1) return fail(REDUCE_ERR_INVALID_ARG, "grid must be >= -1");
   if (mode == REDUCE_MODE_DETERMINISTIC) {
     if (o.grid_combine == REDUCE_GC_ATOMIC)
       return fail(REDUCE_ERR_INVALID_ARG, "deterministic mode forbids the ATOMIC grid combine");
@@ -129,7 +129,11 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   if (o.block_combine < 0 && (mode == REDUCE_MODE_DETERMINISTIC || dd) &&
       (bc == REDUCE_BC_SMEM_ATOMIC_WARP || bc == REDUCE_BC_SMEM_ATOMIC_ALL))
     bc = REDUCE_BC_SHFL;
-  const int grid_cap = o.grid > 0 ? o.grid : e->grid_cap;
+  // grid: > 0 forced cap, -1 forced "one block per tile"; 0 takes the table's
+  // cap, but only when the launch shape is the table's own (a cap tuned for
+  // another block / unroll / staging would mis-shape a forced launch)
+  const bool shape_forced = o.block || o.unroll || o.stage || o.grid_combine >= 0;
+  const int grid_cap = o.grid > 0 ? o.grid : ((o.grid < 0 || shape_forced) ? 0 : e->grid_cap);
   if (!o.block && block > max_block_threads(dtype, op, unroll, stage)) block = max_block_threads(dtype, op, unroll, stage);
   if (block > max_block_threads(dtype, op, unroll, stage))
     return fail(REDUCE_ERR_INVALID_ARG, "block too large for this (dtype, op, unroll): max " +

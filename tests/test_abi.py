@@ -64,7 +64,7 @@ def test_invalid_arguments_rejected_without_cuda(args, why):
 
 @pytest.mark.parametrize("kw", [
     dict(mode=7), dict(grid_combine=9), dict(block_combine=5), dict(unroll=3),
-    dict(block=48), dict(block=2048), dict(block=1024, unroll=8), dict(grid=-2),
+    dict(block=48), dict(block=2048), dict(block=1024, unroll=8), dict(grid=-2), dict(grid=-5),
     dict(mode="deterministic", grid_combine=rb.GC_ATOMIC),
     dict(mode="deterministic", block_combine=rb.BC_SMEM_ATOMIC_ALL),
     dict(block=96, block_combine=rb.BC_SMEM_TREE),
@@ -151,6 +151,14 @@ def test_histogram_argument_validation():
     assert L.reduce_histogram(0, 4096, 10, 0.0, 1.0, 8, None, None) == 1   # counts NULL
     assert L.reduce_histogram(0, 4098, 10, 0.0, 1.0, 8, 8192, None) == 1   # misaligned
     assert L.reduce_histogram(0, 4096, 10, 0.5, 10.0, 8, 8192, None) == 1  # int32 needs integer bounds
+
+
+def test_forced_shape_ignores_table_grid_cap():
+    n = 1 << 24
+    free = rb.query_plan("float32", "sum", n, block=256, unroll=2, grid_combine=2)
+    assert free["grid"] == free["tiles"] == n // (256 * 2 * 8)
+    assert rb.query_plan("float32", "sum", n, grid=-1)["grid"] == rb.query_plan("float32", "sum", n, grid=-1)["tiles"]
+    assert rb.query_plan("float32", "sum", n, block=256, unroll=2, grid=300)["grid"] == 300
 
 
 def test_mode_default_roundtrip():

@@ -41,17 +41,17 @@ def candidates(dtype, op, mode, lb):
     out = []
     if lb <= 18:
         for blk, u in itertools.product((32, 128, 256, 512, 1024), (1, 2, 4)):
-            out.append(dict(block=blk, unroll=u, grid_combine=0, block_combine=0, grid=0))
+            out.append(dict(block=blk, unroll=u, grid_combine=0, block_combine=0, grid=-1))
     if lb >= 12:
         for blk, u, gc in itertools.product((128, 256, 512), (1, 2, 4, 8), gcs):
-            out.append(dict(block=blk, unroll=u, grid_combine=gc, block_combine=0, grid=0))
+            out.append(dict(block=blk, unroll=u, grid_combine=gc, block_combine=0, grid=-1))
         for blk, u, gc in itertools.product((128, 256, 512), (4, 8, 16), gcs):
             if blk * u * 32 <= 128 * 1024:
-                out.append(dict(block=blk, unroll=u, grid_combine=gc, block_combine=0, grid=0, stage=2))
+                out.append(dict(block=blk, unroll=u, grid_combine=gc, block_combine=0, grid=-1, stage=2))
         for bc in (1, 2, 3):
             if (mode == "deterministic" or (op == "sum_accurate" and dtype == "float64")) and bc in (1, 2):
                 continue
-            out.append(dict(block=256, unroll=2, grid_combine=gcs[0], block_combine=bc, grid=0))
+            out.append(dict(block=256, unroll=2, grid_combine=gcs[0], block_combine=bc, grid=-1))
     if 10 <= lb <= 26:
         for blk, u, c in itertools.product((256, 512, 1024), (1, 2, 4), (4, 8, 16)):
             out.append(dict(block=blk, unroll=u, grid_combine=4, block_combine=0, grid=c))
@@ -154,7 +154,9 @@ def emit(paths, dst, tol=0.01):
         for i, (lb, pick) in enumerate(chosen):
             last = i == len(chosen) - 1
             if last or sig(chosen[i + 1][1]["cfg"]) != sig(pick["cfg"]):
-                rows.append((DT[dtype], OPC[op], MODE[mode], 63 if last else lb) + sig(pick["cfg"]) +
+                c = dict(pick["cfg"])
+            c["grid"] = max(0, c["grid"])  # table: 0 = one block per tile
+            rows.append((DT[dtype], OPC[op], MODE[mode], 63 if last else lb) + sig(c) +
                             (round(pick["gbps"], 1),))
         # min mirrors max when only max was tuned
         if op == "max" and (dtype, "min", mode) not in groups:

@@ -21,10 +21,10 @@ def main():
     pool = torch.rand((2 << 30) // 4, device=dev)
     rb.prepare(s, pool.numel())
     outs = torch.empty(4096, device=dev)
-    variants = {"default": {}, "256x2 atomic": dict(block=256, unroll=2, grid_combine=1),
-                "256x2 2pass": dict(block=256, unroll=2, grid_combine=2),
-                "256x2 lastblk": dict(block=256, unroll=2, grid_combine=3),
-                "256x4 atomic": dict(block=256, unroll=4, grid_combine=1),
+    variants = {"default": {}, "256x2 atomic": dict(block=256, unroll=2, grid_combine=1, grid=-1),
+                "256x2 2pass": dict(block=256, unroll=2, grid_combine=2, grid=-1),
+                "256x2 lastblk": dict(block=256, unroll=2, grid_combine=3, grid=-1),
+                "256x4 atomic": dict(block=256, unroll=4, grid_combine=1, grid=-1),
                 "cluster16 1024x2": dict(block=1024, unroll=2, grid_combine=4, grid=16)}
     rows = []
     for lb in range(16, 29, 2):
