@@ -155,8 +155,8 @@ def emit(paths, dst, tol=0.01):
             last = i == len(chosen) - 1
             if last or sig(chosen[i + 1][1]["cfg"]) != sig(pick["cfg"]):
                 c = dict(pick["cfg"])
-            c["grid"] = max(0, c["grid"])  # table: 0 = one block per tile
-            rows.append((DT[dtype], OPC[op], MODE[mode], 63 if last else lb) + sig(c) +
+                c["grid"] = max(0, c["grid"])  # table: 0 = one block per tile
+                rows.append((DT[dtype], OPC[op], MODE[mode], 63 if last else lb) + sig(c) +
                             (round(pick["gbps"], 1),))
         # min mirrors max when only max was tuned
         if op == "max" and (dtype, "min", mode) not in groups:
