@@ -173,10 +173,15 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   // ---- longest fp addition chain L of this variant (for the G2 gate)
   long long chain = 0;
   if ((op == REDUCE_SUM || op == REDUCE_SUM_ACCURATE) && dtype != REDUCE_INT32) {
-    const int na = dtype == REDUCE_FLOAT64 ? 4 : 8;
     const long long tpb = (tiles + grid - 1) / grid;
     const int nw = block / 32;
-    chain = (long long)unroll * tpb + 1 + ilog2_ceil(na);  // per-thread lanes (+head/tail) + lane tree
+    if (op == REDUCE_SUM) {
+      // vector tree (depth log2 VE) into 2 accumulators, +1 head/tail, +1 merging the two
+      chain = (long long)((unroll + 1) / 2) * tpb + ilog2_ceil(32 / s) + 2;
+    } else {
+      const int na = dtype == REDUCE_FLOAT64 ? 4 : 8;  // one accumulator per vector lane
+      chain = (long long)unroll * tpb + 1 + ilog2_ceil(na);
+    }
     switch (bc) {
       case REDUCE_BC_SHFL: chain += 5 + (nw > 1 ? 5 : 0); break;
       case REDUCE_BC_SMEM_ATOMIC_WARP: chain += 5 + nw; break;

@@ -148,7 +148,9 @@ template <int OP> struct TrI32 {
   using Elem = int32_t;
   using Acc = typename std::conditional<OP == OP_SUM, uint32_t, int32_t>::type;
   using Grid = Acc;
-  static constexpr int VE = 8, NA = 8, kLaneWords = 1;
+  static constexpr int VE = 8, NA = 2, kLaneWords = 1;
+  static constexpr bool kVecTree = true;
+  __device__ static Acc lift(uint32_t w) { return Acc(w); }
   __device__ static Acc ident() {
     return OP == OP_SUM ? Acc(0) : (OP == OP_MIN ? Acc(0x7FFFFFFF) : Acc(0x80000000));
   }
@@ -179,8 +181,10 @@ template <int OP> struct TrF32 {
   using Elem = float;
   using Acc = float;
   using Grid = typename std::conditional<OP == OP_SUM, double, uint32_t>::type;
-  static constexpr int VE = 8, NA = 8, kLaneWords = 1;
+  static constexpr int VE = 8, NA = 2, kLaneWords = 1;
+  static constexpr bool kVecTree = true;
   static constexpr bool kMax = OP == OP_MAX;
+  __device__ static float lift(uint32_t w) { return __uint_as_float(w); }
   __device__ static Acc ident() {
     return OP == OP_SUM ? 0.0f : (OP == OP_MIN ? __int_as_float(0x7F800000) : __int_as_float(0xFF800000));
   }
@@ -232,8 +236,11 @@ template <int OP> struct TrF64 {
   using Elem = double;
   using Acc = double;
   using Grid = typename std::conditional<OP == OP_SUM, double, unsigned long long>::type;
-  static constexpr int VE = 4, NA = 4, kLaneWords = 2;
+  // sums: vector tree into 2 accumulators; min/max: per-lane select + NaN flag
+  static constexpr int VE = 4, NA = OP == OP_SUM ? 2 : 4, kLaneWords = 2;
+  static constexpr bool kVecTree = OP == OP_SUM;
   static constexpr bool kMax = OP == OP_MAX;
+  __device__ static double lift(double x) { return x; }
   __device__ static Acc ident() {
     return OP == OP_SUM ? 0.0 : __longlong_as_double(OP == OP_MIN ? 0x7FF0000000000000ll : (long long)0xFFF0000000000000ull);
   }
@@ -295,6 +302,7 @@ struct TrF32Acc {
   using Grid = double;
   using Part = float2;  // x = s, y = c
   static constexpr int VE = 8, NA = 8, kLaneWords = 1;
+  static constexpr bool kVecTree = false;
   __device__ static Acc ident() { return 0.0; }
   __device__ static Part part_ident() { return make_float2(0.0f, 0.0f); }
   __device__ static Acc part_to_acc(Part p) { return isfinite(p.x) ? (double)p.x + (double)p.y : (double)p.x; }
@@ -332,6 +340,7 @@ struct TrF64Acc {
   using Acc = double2;  // x = hi, y = lo
   using Grid = double2;
   static constexpr int VE = 4, NA = 4, kLaneWords = 2;
+  static constexpr bool kVecTree = false;
   __device__ static Acc ident() { return make_double2(0.0, 0.0); }
   __device__ static Acc comb(Acc a, Acc b) {
     const double s = a.x + b.x;                       // TwoSum(a.hi, b.hi)
@@ -380,11 +389,29 @@ template <class T> struct PartOf<T, std::void_t<typename T::Part>> {
 };
 template <class T> using Part = typename PartOf<T>::type;
 
-// Fold one 32-byte vector into the NA per-thread accumulators (lane k of the
-// vector goes to accumulator k: NA independent chains).
+// Fold one 32-byte vector into the per-thread accumulators.
+//   kVecTree (plain sums, min, max): the vector's lanes are reduced by a
+//     pairwise tree in registers (depth log2 VE) and the result is folded into
+//     accumulator `slot % NA` (NA = 2: two independent chains) -- the same
+//     addition depth as one accumulator per lane, with 6 fewer live registers,
+//     which keeps the small-unroll kernels at 32 registers (full occupancy).
+//   otherwise (accurate sums, fp64 min/max): lane k folds into accumulator k.
 template <class T>
-__device__ __forceinline__ void fold_vec(Part<T> (&a)[T::NA], uint32_t& aux, const uint32_t (&r)[8]) {
-  if constexpr (T::kLaneWords == 1) {
+__device__ __forceinline__ void fold_vec(Part<T> (&a)[T::NA], uint32_t& aux, const uint32_t (&r)[8], int slot) {
+  if constexpr (T::kVecTree) {
+    using Acc = typename T::Acc;
+    Acc t;
+    if constexpr (T::kLaneWords == 1) {
+      const Acc t01 = T::comb(T::lift(r[0]), T::lift(r[1])), t23 = T::comb(T::lift(r[2]), T::lift(r[3]));
+      const Acc t45 = T::comb(T::lift(r[4]), T::lift(r[5])), t67 = T::comb(T::lift(r[6]), T::lift(r[7]));
+      t = T::comb(T::comb(t01, t23), T::comb(t45, t67));
+    } else {
+      const Acc t01 = T::comb(T::lift(__hiloint2double((int)r[1], (int)r[0])), T::lift(__hiloint2double((int)r[3], (int)r[2])));
+      const Acc t23 = T::comb(T::lift(__hiloint2double((int)r[5], (int)r[4])), T::lift(__hiloint2double((int)r[7], (int)r[6])));
+      t = T::comb(t01, t23);
+    }
+    a[slot % T::NA] = T::comb(a[slot % T::NA], t);
+  } else if constexpr (T::kLaneWords == 1) {
 #pragma unroll
     for (int k = 0; k < 8; ++k) T::fold(a[k], aux, r[k]);
   } else {

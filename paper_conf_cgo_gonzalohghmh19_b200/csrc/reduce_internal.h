@@ -23,6 +23,15 @@ constexpr int kMaxSmemTileBytes = 128 * 1024;
 // with register staging, the budget of 64 registers/thread at 1024 threads is
 // too small for 8 in-flight 32-byte loads, and for the fp64 min/max
 // select+NaN-flag fold at unroll >= 2.
+// Minimum resident blocks requested from ptxas for the small-unroll register
+// instantiations: at 2048 threads per SM this caps them at 32 registers, i.e.
+// full occupancy (the mid-size regime is latency-bound: 8 x 256-thread blocks
+// keep 33 % more bytes in flight than the 6 blocks 35-36 registers allow).
+constexpr int min_blocks_hint(int dtype, int op, int unroll, int stage, int max_threads) {
+  return (stage == STAGE_REG && (unroll == 1 || (unroll == 2 && dtype != 0)) && op != 3 && !(dtype == 2 && op != 0))
+             ? 2048 / max_threads : 1;
+}
+
 constexpr int max_block_threads(int dtype, int op, int unroll, int stage = STAGE_REG) {
   return stage == STAGE_SMEM ? (op == 3 ? 512 : 1024)
                              : ((unroll >= 8 || (dtype == 2 && op != 0 && unroll >= 2) || (op == 3 && unroll >= 4))

@@ -124,7 +124,9 @@ __device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& 
 }
 
 template <int DT, int OP, int U, int BC, int STAGE>
-__global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(const KParams p) {
+__global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
+                                  min_blocks_hint(DT, OP, U, STAGE, max_block_threads(DT, OP, U, STAGE)))
+    k_reduce(const KParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
   // Programmatic dependent launch: this grid may be resident before the
@@ -168,7 +170,7 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(
         if (full || v0 + (unsigned long long)(u * B) < p.body_vecs) {
           uint32_t r[8];
           lds_v8(stile + ((size_t)u * B + threadIdx.x) * kVecBytes, r);
-          fold_vec<T>(a, aux, r);
+          fold_vec<T>(a, aux, r, u);
         }
       }
     } else if (full) {
@@ -176,14 +178,14 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE)) k_reduce(
 #pragma unroll
       for (int u = 0; u < U; ++u) ld_v8(ptr + (size_t)u * B * kVecBytes, r[u]);
 #pragma unroll
-      for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, r[u]);
+      for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, r[u], u);
     } else {  // the ragged last tile
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         if (v0 + (unsigned long long)(u * B) < p.body_vecs) {
           uint32_t r[8];
           ld_v8(ptr + (size_t)u * B * kVecBytes, r);
-          fold_vec<T>(a, aux, r);
+          fold_vec<T>(a, aux, r, u);
         }
       }
     }

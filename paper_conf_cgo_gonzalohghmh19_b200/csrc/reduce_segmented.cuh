@@ -38,17 +38,17 @@ __device__ __forceinline__ void fold_range(Part<T> (&a)[T::NA], uint32_t& aux, c
 #pragma unroll
     for (int u = 0; u < U; ++u) ld_v8(body + (v + (long long)u * lanes) * kVecBytes, r[u]);
 #pragma unroll
-    for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, r[u]);
+    for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, r[u], u);
   }
   for (; v < nvec; v += lanes) {
     uint32_t r[8];
     ld_v8(body + v * kVecBytes, r);
-    fold_vec<T>(a, aux, r);
+    fold_vec<T>(a, aux, r, 0);
   }
   // head and tail (< 8 elements each) by the first lanes, into two different
   // accumulators (groups may be only 8 lanes wide)
   if (lid < head) fold_elem<T>(a[0], aux, __ldg((const Elem*)p + lid));
-  if (lid < tail) fold_elem<T>(a[1], aux, __ldg((const Elem*)(body + nvec * kVecBytes) + lid));
+  if (lid < tail) fold_elem<T>(a[T::NA - 1], aux, __ldg((const Elem*)(body + nvec * kVecBytes) + lid));
 }
 
 template <class T>

@@ -17,9 +17,11 @@ OPS = ["sum", "min", "max"]
 
 
 def _chain(length, dtype, lanes):
+    # per-thread: m vectors through a lane tree (depth log2 VE) into 2 accumulators
+    # (or one accumulator per lane), + head/tail, + merge; then group / block combines
     ve = 4 if dtype == "float64" else 8
-    na = 4 if dtype == "float64" else 8
-    return math.ceil(length / (ve * lanes)) + 1 + int(math.log2(na)) + 5 + (5 if lanes > 32 else 0)
+    m = math.ceil(length / (ve * lanes))
+    return m + int(math.log2(ve)) + 3 + 5 + (5 if lanes > 32 else 0)
 
 
 def _check_segments(x, bounds, op, got, lanes):
