@@ -193,8 +193,8 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
       // input): L counts additions of that wider format, plus the final rounding
       switch (gc) {
         case REDUCE_GC_ATOMIC: chain += (grid + nslots - 1) / nslots + 5; break;
-        case REDUCE_GC_TWO_PASS: chain += (grid + 1023) / 1024 + 10; break;
-        case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + ilog2_ceil(block); break;
+        case REDUCE_GC_TWO_PASS: chain += (grid + 255) / 256 + 2 + 10; break;
+        case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + 2 + 10; break;
         case REDUCE_GC_CLUSTER: chain += 5; break;
         default: break;
       }
@@ -205,8 +205,8 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
     } else {
       switch (gc) {
         case REDUCE_GC_ATOMIC: chain += (grid + nslots - 1) / nslots + 5; break;
-        case REDUCE_GC_TWO_PASS: chain += (grid + 1023) / 1024 + 10; break;
-        case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + ilog2_ceil(block); break;
+        case REDUCE_GC_TWO_PASS: chain += (grid + 255) / 256 + 2 + 10; break;
+        case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + 2 + 10; break;
         case REDUCE_GC_CLUSTER: chain += 5; break;
         default: break;
       }

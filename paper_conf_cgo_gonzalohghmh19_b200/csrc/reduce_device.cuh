@@ -503,8 +503,19 @@ template <class T>
 __device__ __forceinline__ typename T::Grid reduce_grid_values(const typename T::Grid* vals, long long count) {
   using Grid = typename T::Grid;
   __shared__ Grid gpart[32];
-  Grid x = T::gident();
-  for (long long i = threadIdx.x; i < count; i += blockDim.x) x = T::gcomb(x, __ldcg(vals + i));
+  // 4 independent loads in flight per thread (values are L2-resident)
+  Grid x0 = T::gident(), x1 = T::gident(), x2 = T::gident(), x3 = T::gident();
+  const long long B = blockDim.x;
+  long long i = threadIdx.x;
+  for (; i + 3 * B < count; i += 4 * B) {
+    const Grid v0 = __ldcg(vals + i), v1 = __ldcg(vals + i + B), v2 = __ldcg(vals + i + 2 * B), v3 = __ldcg(vals + i + 3 * B);
+    x0 = T::gcomb(x0, v0);
+    x1 = T::gcomb(x1, v1);
+    x2 = T::gcomb(x2, v2);
+    x3 = T::gcomb(x3, v3);
+  }
+  for (; i < count; i += B) x0 = T::gcomb(x0, __ldcg(vals + i));
+  Grid x = T::gcomb(T::gcomb(x0, x1), T::gcomb(x2, x3));
   x = T::gwarp(x);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
   __syncthreads();  // gpart may still be read by a previous use in this block

@@ -333,7 +333,9 @@ cudaError_t launch_op(const LaunchDesc& d, cudaStream_t s) {
     }
   }
   if (e != cudaSuccess || d.gc != GC_TWO_PASS) return e;
-  return launch_combine_kernel<DT, OP>(d.partials, (long long)d.grid, d.out, d.raw_out, 1024, s);
+  // the second pass: one block, 4 loads in flight per thread; 256 threads up to
+  // 4096 partials, else 1024
+  return launch_combine_kernel<DT, OP>(d.partials, (long long)d.grid, d.out, d.raw_out, d.grid <= 4096 ? 256 : 1024, s);
 }
 
 template <int DT>
