@@ -168,7 +168,9 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
     if ((gc == REDUCE_GC_TWO_PASS || gc == REDUCE_GC_LAST_BLOCK) && grid > kMaxPartialBlocks) grid = kMaxPartialBlocks;
     if (grid > 0x7FFFFFFFll) grid = 0x7FFFFFFFll;
   }
-  const int nslots = gc == REDUCE_GC_ATOMIC ? (int)(grid < 32 ? grid : 32) : 0;
+  int nslots = 0;  // ATOMIC: a power of two <= min(grid, 32) (the kernel masks, no modulo)
+  if (gc == REDUCE_GC_ATOMIC)
+    for (nslots = 1; nslots * 2 <= 32 && nslots * 2 <= grid;) nslots *= 2;
 
   // ---- longest fp addition chain L of this variant (for the G2 gate)
   long long chain = 0;

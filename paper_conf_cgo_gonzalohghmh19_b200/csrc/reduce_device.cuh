@@ -507,6 +507,7 @@ __device__ __forceinline__ typename T::Grid reduce_grid_values(const typename T:
   Grid x0 = T::gident(), x1 = T::gident(), x2 = T::gident(), x3 = T::gident();
   const long long B = blockDim.x;
   long long i = threadIdx.x;
+#pragma unroll 1
   for (; i + 3 * B < count; i += 4 * B) {
     const Grid v0 = __ldcg(vals + i), v1 = __ldcg(vals + i + B), v2 = __ldcg(vals + i + 2 * B), v3 = __ldcg(vals + i + 3 * B);
     x0 = T::gcomb(x0, v0);
@@ -514,6 +515,7 @@ __device__ __forceinline__ typename T::Grid reduce_grid_values(const typename T:
     x2 = T::gcomb(x2, v2);
     x3 = T::gcomb(x3, v3);
   }
+#pragma unroll 1
   for (; i < count; i += B) x0 = T::gcomb(x0, __ldcg(vals + i));
   Grid x = T::gcomb(T::gcomb(x0, x1), T::gcomb(x2, x3));
   x = T::gwarp(x);

@@ -88,7 +88,7 @@ __device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& 
     // collects the slots (atomicExch resets them to the identity, so no memset
     // is ever needed) and publishes the result.
     if (threadIdx.x == 0) {
-      Grid* slot = (Grid*)((char*)p.slots + (size_t)(blockIdx.x % p.nslots) * kSlotBytes);
+      Grid* slot = (Grid*)((char*)p.slots + (size_t)(blockIdx.x & (p.nslots - 1)) * kSlotBytes);  // nslots: power of 2
       T::gred(slot, g);
       const unsigned tk = ticket_acq_rel(p.ticket);  // release: the red above; acquire: everyone's
       s_last = (tk == gridDim.x - 1);
@@ -146,6 +146,11 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
 
   const long long B = blockDim.x;
   const long long tile_vecs = B * U;
+  // no unrolling: an unrolled loop makes the compiler compute the trip count
+  // with a 64-bit division (a CALL to the division routine) in every block's
+  // prologue -- measurable latency at medium sizes, where the default grid
+  // runs this loop exactly once
+#pragma unroll 1
   for (long long tile = blockIdx.x; tile < p.tiles; tile += gridDim.x) {
     const unsigned long long v0 = (unsigned long long)(tile * tile_vecs) + threadIdx.x;
     const char* ptr = p.body + v0 * kVecBytes;

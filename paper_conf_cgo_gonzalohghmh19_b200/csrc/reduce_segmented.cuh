@@ -86,6 +86,7 @@ __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
   // the last segment folds nothing
   const long long base = kGroup > 0 ? first - lane / kGroup : first;
   const long long iters = base < p.nseg ? (p.nseg - base + step - 1) / step : 0;
+#pragma unroll 1
   for (long long it = 0; it < iters; ++it) {
     const long long seg = first + it * step;
     const bool live = seg < p.nseg;
