@@ -423,6 +423,47 @@ def main():
                                  "GBps": round(n * 4 / sec / 1e9, 1), "frac_of_peak": round(n * 4 / sec / 1e9 / peak, 4),
                                  "variant": f"gc{pp['grid_combine']} g{pp['grid']}x{pp['block']} u{pp['unroll']} st{pp['stage']}"})
 
+    # ---- BASELINE configs[0]: int32 sum of 1 M full-range elements vs the CPU
+    # oracle (bit-exact) -- device time per call, and the oracle on the host
+    cfg1 = cfg3 = None
+    if not args.no_sweep and world == 1:
+        import oracle
+        m = 1 << 20
+        xi_h = synth.make("int32", m, "int_full", synth.seed_for(0, m))
+        xi = torch.from_numpy(xi_h).to(dev)
+        oi = torch.empty(4096, dtype=torch.int32, device=dev)
+        warm_i, timed_i = disjoint_regions(x.view(torch.int32), 50, m)
+        ctr = [0]
+
+        def launch_i(t):
+            ctr[0] = (ctr[0] + 1) % 4096
+            rb.reduce(t, "sum", out=oi[ctr[0]:ctr[0] + 1], stream=stream)
+        gpu_us = time_calls(launch_i, warm_i, timed_i, stream, repeats=3) * 1e6
+        got = int(rb.reduce(xi, "sum", stream=stream).cpu().item())
+        t0 = time.perf_counter()
+        want = int(oracle.reduce(xi_h, "sum").value)
+        cpu_us = (time.perf_counter() - t0) * 1e6
+        cfg1 = {"n": m, "gpu_us": round(gpu_us, 3), "GBps": round(m * 4 / gpu_us / 1e3, 1), "cpu_oracle_us": round(cpu_us, 1),
+                "bit_exact": got == want}
+        # ---- BASELINE configs[2]: int32 / fp64 sum, min, max at 64 M elements,
+        # atomic (fast) vs deterministic-tree grid combine
+        cfg3 = []
+        for dt_name, tdt, es in (("int32", torch.int32, 4), ("float64", torch.float64, 8)):
+            m = 1 << 26
+            regs_w, regs_t = disjoint_regions(x.view(tdt), 4, m)
+            o3 = torch.empty(4096, dtype=tdt, device=dev)
+            for op in ("sum", "min", "max"):
+                row = {"dtype": dt_name, "op": op, "n": m}
+                for mode in ("fast", "deterministic"):
+                    def launch_3(t, op=op, mode=mode, o3=o3):
+                        ctr[0] = (ctr[0] + 1) % 4096
+                        rb.reduce(t, op, out=o3[ctr[0]:ctr[0] + 1], stream=stream, mode=mode)
+                    sec = time_calls(launch_3, regs_w, regs_t, stream, repeats=2)
+                    pp = rb.query_plan(dt_name, op, m, in_ptr=regs_t[0].data_ptr(), mode=mode)
+                    row[mode] = {"us": round(sec * 1e6, 2), "GBps": round(m * es / sec / 1e9, 1),
+                                 "grid_combine": ["direct", "atomic", "two_pass", "last_block", "cluster"][pp["grid_combine"]]}
+                cfg3.append(row)
+
     # ---- BASELINE configs[4] at k = 1: one 8 GiB (2^31 fp32) array on one GPU
     # (64-bit indexing); timing only (its parity is tests/test_parity_gpu.py's
     # full-size test), so the array is drawn on the device.
@@ -521,6 +562,8 @@ def main():
             line["ops_1GiB"] = ops_1gib
             line["histogram"] = hist
             line["config5_8GiB_one_gpu"] = big
+            line["config1_int32_1M"] = cfg1
+            line["config3_64M_atomic_vs_tree"] = cfg3
         if ncu_s is not None:
             line["ncu"] = {k: ncu_s[k] for k in ("source", "dram_pct_of_peak", "duration_us") if k in ncu_s}
         print(json.dumps(line), flush=True)
