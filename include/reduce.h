@@ -237,6 +237,30 @@ int reduce_comm_get_unique_id(void* id_out);     /* rank 0; broadcast the bytes 
 int reduce_comm_init(void** comm_out, const void* id, int nranks, int rank); /* after cudaSetDevice */
 int reduce_comm_destroy(void* comm);
 
+/* ---- sharded mode with the cross-GPU combine fused into the kernel --------
+ * (the one-shot combine "fused as the epilogue of the last
+ * block").  A team is k ranks (one per GPU, or several on one GPU); each owns a
+ * small device buffer that every member maps: across processes through CUDA
+ * IPC handles (peer memory over NVLink / NVSwitch), within one process through
+ * plain pointers.  reduce_multi_team: every member calls it (same order of
+ * calls on every rank) with its local shard; the block that completes a
+ * rank's local reduction stores the raw value into every member's buffer
+ * (P2P), raises a flag (release, system scope), waits for all k flags and
+ * combines the k values in rank order -- no collective launch, deterministic
+ * for a fixed team.  Every member's *out receives the global result.
+ *   reduce_team_create(&t, k, rank, handle_out)  handle_out: reduce_team_ipc_handle_bytes() bytes (or NULL)
+ *   reduce_team_connect(t, handles)             k handles, rank order, from every member (IPC)
+ *   reduce_team_connect_local(t, bufs)          k device pointers (reduce_team_buffer of each member)
+ * A member that never calls leaves the others waiting (as with any collective). */
+int reduce_team_create(void** team_out, int nranks, int rank, void* ipc_handle_out);
+int reduce_team_ipc_handle_bytes(void);
+void* reduce_team_buffer(void* team);
+int reduce_team_connect(void* team, const void* handles);
+int reduce_team_connect_local(void* team, void* const* bufs);
+int reduce_team_destroy(void* team);
+int reduce_multi_team(int dtype, int op, const void* in_local, size_t n_local, void* out, reduce_stream_t stream,
+                      void* team, const reduce_opts_t* opts);
+
 /* ---- diagnostics ---------------------------------------------------------- */
 const char* reduce_status_string(int status);
 const char* reduce_last_error(void);   /* thread-local detail of the last failure */

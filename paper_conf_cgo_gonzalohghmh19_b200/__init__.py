@@ -35,6 +35,8 @@ ABI_SYMBOLS = (
     "reduce_comm_unique_id_bytes", "reduce_comm_get_unique_id", "reduce_comm_init",
     "reduce_comm_destroy", "reduce_status_string", "reduce_last_error", "reduce_version",
     "reduce_shutdown", "reduce_segmented", "reduce_batched", "reduce_histogram",
+    "reduce_team_create", "reduce_team_ipc_handle_bytes", "reduce_team_buffer", "reduce_team_connect",
+    "reduce_team_connect_local", "reduce_team_destroy", "reduce_multi_team",
 )
 
 
@@ -91,6 +93,13 @@ def _load() -> ctypes.CDLL:
         "reduce_segmented": (i, [i, i, vp, vp, sz, vp, vp, opts_p]),
         "reduce_batched": (i, [i, i, vp, sz, sz, vp, vp, opts_p]),
         "reduce_histogram": (i, [i, vp, sz, ctypes.c_double, ctypes.c_double, i, vp, vp]),
+        "reduce_team_create": (i, [ctypes.POINTER(vp), i, i, vp]),
+        "reduce_team_ipc_handle_bytes": (i, []),
+        "reduce_team_buffer": (vp, [vp]),
+        "reduce_team_connect": (i, [vp, vp]),
+        "reduce_team_connect_local": (i, [vp, ctypes.POINTER(vp)]),
+        "reduce_team_destroy": (i, [vp]),
+        "reduce_multi_team": (i, [i, i, vp, sz, vp, vp, vp, opts_p]),
     }
     for name, (res, args) in sigs.items():
         f = getattr(L, name)
@@ -320,6 +329,61 @@ def reduce_multi(x, op, comm: Comm, out=None, stream=None, **opt_kw):
                              ctypes.c_void_p(out.data_ptr()), ctypes.c_void_p(_stream_handle(stream, x.device)),
                              ctypes.c_void_p(comm.handle), ctypes.byref(opts) if opts is not None else None)
     _check(st, "reduce_multi_ex")
+    return out
+
+
+class Team:
+    """Ranks whose per-rank results meet through peer memory inside the kernel
+    (reduce_multi_team).  Team(group) exchanges CUDA IPC handles
+    over a torch.distributed group (one process per GPU, or several processes on
+    one GPU); Team.local(k) makes k in-process members (e.g. one per stream)."""
+
+    def __init__(self, group=None, _local=None):
+        if _local is not None:
+            self.handle, self.rank, self.world = _local
+            return
+        import torch.distributed as dist
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        nb = lib.reduce_team_ipc_handle_bytes()
+        hbuf = (ctypes.c_char * nb)()
+        handle = ctypes.c_void_p()
+        _check(lib.reduce_team_create(ctypes.byref(handle), world, rank, ctypes.cast(hbuf, ctypes.c_void_p)),
+               "reduce_team_create")
+        allh = [None] * world
+        dist.all_gather_object(allh, bytes(hbuf), group=group)
+        joined = (ctypes.c_char * (nb * world)).from_buffer_copy(b"".join(allh))
+        _check(lib.reduce_team_connect(handle, ctypes.cast(joined, ctypes.c_void_p)), "reduce_team_connect")
+        self.handle, self.rank, self.world = handle.value, rank, world
+
+    @classmethod
+    def local(cls, k: int):
+        hs = []
+        for r in range(k):
+            h = ctypes.c_void_p()
+            _check(lib.reduce_team_create(ctypes.byref(h), k, r, None), "reduce_team_create")
+            hs.append(h.value)
+        bufs = (ctypes.c_void_p * k)(*[lib.reduce_team_buffer(h) for h in hs])
+        for h in hs:
+            _check(lib.reduce_team_connect_local(h, bufs), "reduce_team_connect_local")
+        return [cls(_local=(h, r, k)) for r, h in enumerate(hs)]
+
+    def destroy(self) -> None:
+        if self.handle:
+            _check(lib.reduce_team_destroy(self.handle), "reduce_team_destroy")
+            self.handle = None
+
+
+def reduce_multi_team(x, op, team: Team, out=None, stream=None, **opt_kw):
+    """Every team member passes its local CUDA shard; every member gets the global result."""
+    import torch
+    dt = _torch_dtype_code(x)
+    if out is None:
+        out = torch.empty(1, dtype=x.dtype, device=x.device)
+    opts = make_opts(**opt_kw) if opt_kw else None
+    st = lib.reduce_multi_team(dt, _op(op), x.data_ptr() or None, x.numel(), out.data_ptr(),
+                               _stream_handle(stream, x.device), team.handle,
+                               ctypes.byref(opts) if opts is not None else None)
+    _check(st, "reduce_multi_team")
     return out
 
 

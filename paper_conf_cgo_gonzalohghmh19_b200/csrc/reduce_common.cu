@@ -7,9 +7,9 @@ namespace rb {
 cudaError_t launch_reduce_i32(const LaunchDesc&, cudaStream_t);
 cudaError_t launch_reduce_f32(const LaunchDesc&, cudaStream_t);
 cudaError_t launch_reduce_f64(const LaunchDesc&, cudaStream_t);
-cudaError_t combine_i32(int, const void*, long long, void*, int, int, cudaStream_t);
-cudaError_t combine_f32(int, const void*, long long, void*, int, int, cudaStream_t);
-cudaError_t combine_f64(int, const void*, long long, void*, int, int, cudaStream_t);
+cudaError_t combine_i32(int, const void*, long long, void*, int, int, cudaStream_t, TeamArgs);
+cudaError_t combine_f32(int, const void*, long long, void*, int, int, cudaStream_t, TeamArgs);
+cudaError_t combine_f64(int, const void*, long long, void*, int, int, cudaStream_t, TeamArgs);
 cudaError_t init_i32(char*, char*, cudaStream_t);
 cudaError_t init_f32(char*, char*, cudaStream_t);
 cudaError_t init_f64(char*, char*, cudaStream_t);
@@ -59,11 +59,11 @@ cudaError_t launch_reduce(const LaunchDesc& d, cudaStream_t s) {
 }
 
 cudaError_t launch_combine(int dtype, int op, const void* vals, long long count, void* out, int raw_out,
-                           int block, cudaStream_t s) {
+                           int block, cudaStream_t s, TeamArgs team) {
   switch (dtype) {
-    case 0: return combine_i32(op, vals, count, out, raw_out, block, s);
-    case 1: return combine_f32(op, vals, count, out, raw_out, block, s);
-    case 2: return combine_f64(op, vals, count, out, raw_out, block, s);
+    case 0: return combine_i32(op, vals, count, out, raw_out, block, s, team);
+    case 1: return combine_f32(op, vals, count, out, raw_out, block, s, team);
+    case 2: return combine_f64(op, vals, count, out, raw_out, block, s, team);
   }
   return cudaErrorInvalidValue;
 }

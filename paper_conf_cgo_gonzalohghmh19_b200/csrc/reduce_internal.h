@@ -38,6 +38,22 @@ constexpr int max_block_threads(int dtype, int op, int unroll, int stage = STAGE
                                     ? 512 : 1024);
 }
 
+// Team = the ranks of a sharded reduction whose per-rank raw results are
+// exchanged through peer memory inside the reduction kernel itself (SURVEY
+// 8(f) N2, the "one-shot combine fused as the epilogue of the last block").
+// Every rank owns one buffer of kTeamBufBytes; bufs[j] is rank j's buffer as
+// seen from this GPU (a CUDA-IPC / peer mapping over NVLink, or a local pointer).
+//   [0, 2*kTeamMaxRanks*16)           slots[parity][rank]   raw values (<= 16 B)
+//   [kTeamFlagOff, + 2*kTeamMaxRanks*4) flags[parity][rank]  epoch of the value
+struct TeamArgs {
+  char* const* bufs;  // device array of k pointers (nullptr when not a team call)
+  int k, rank;
+  unsigned epoch;     // 1, 2, 3, ... per call; parity = epoch & 1
+};
+constexpr int kTeamMaxRanks = 256;
+constexpr size_t kTeamFlagOff = 2 * kTeamMaxRanks * 16;
+constexpr size_t kTeamBufBytes = kTeamFlagOff + 2 * kTeamMaxRanks * 4;
+
 // One launch of the main reduction kernel (steps S2-S5), fully resolved by the
 // host dispatcher (step S0).
 struct LaunchDesc {
@@ -54,6 +70,7 @@ struct LaunchDesc {
   int nslots;
   unsigned* ticket;              // this (dtype, op)'s ticket (GC_ATOMIC / GC_LAST_BLOCK)
   void* partials;                // Grid[grid] (GC_TWO_PASS / GC_LAST_BLOCK)
+  TeamArgs team;                 // team.k > 0: exchange the raw result with the team first
 };
 
 // One segmented / batched launch, see reduce_segmented.cuh.
@@ -91,7 +108,7 @@ cudaError_t launch_reduce(const LaunchDesc& d, cudaStream_t s);
 // Reduce `count` Grid-typed values in a fixed order with one block of
 // `block` threads and write the finalised (or raw) result to `out`.
 cudaError_t launch_combine(int dtype, int op, const void* vals, long long count, void* out,
-                           int raw_out, int block, cudaStream_t s);
+                           int raw_out, int block, cudaStream_t s, TeamArgs team = TeamArgs{nullptr, 0, 0, 0});
 
 // Write the identity into every accumulator slot of every (dtype, op) and zero
 // the tickets.  slots_base: 9 regions of kMaxSlots*kSlotBytes; tickets: 9 words

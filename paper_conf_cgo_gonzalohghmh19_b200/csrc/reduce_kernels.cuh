@@ -42,10 +42,55 @@ struct KParams {
   int nslots;
   unsigned* ticket;
   void* partials;
+  TeamArgs team;
 };
+
+// ---- one-shot cross-GPU combine through peer memory ------
+// Executed by ONE thread of the block that owns this rank's raw result x:
+// write x into slot [parity][rank] of every team member's buffer (P2P stores
+// over NVLink), make them visible system-wide, raise flag [parity][rank] =
+// epoch in every buffer (release, system scope), then wait until all k flags
+// of the own buffer carry this epoch (acquire) and combine slots 0..k-1 in rank
+// order (deterministic for a fixed team).  Parity double-buffering: a rank can
+// reuse parity p only after every member has set its flag for the following
+// call, i.e. after everyone finished reading parity p.
+__device__ __forceinline__ void st_release_sys(unsigned* p, unsigned v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+template <class T>
+__device__ __noinline__ typename T::Grid team_exchange(typename T::Grid x, const TeamArgs& t) {
+  using Grid = typename T::Grid;
+  const int par = t.epoch & 1;
+  for (int j = 0; j < t.k; ++j)
+    __stcg((Grid*)(t.bufs[j] + ((size_t)par * kTeamMaxRanks + t.rank) * 16), x);  // L2 (peer: remote L2)
+  __threadfence_system();
+  for (int j = 0; j < t.k; ++j)
+    st_release_sys((unsigned*)(t.bufs[j] + kTeamFlagOff + ((size_t)par * kTeamMaxRanks + t.rank) * 4), t.epoch);
+  const char* own = t.bufs[t.rank];
+  Grid acc = T::gident();
+  for (int j = 0; j < t.k; ++j) {
+    const unsigned* f = (const unsigned*)(own + kTeamFlagOff + ((size_t)par * kTeamMaxRanks + j) * 4);
+    const long long t0 = clock64();
+    while (ld_acquire_sys(f) != t.epoch) {
+      __nanosleep(64);
+      // a member that never arrives must not hang the GPU: after ~2^35 cycles
+      // (> 15 s) abort the kernel -- the error surfaces at the caller's sync
+      if (clock64() - t0 > (1ll << 35)) __trap();
+    }
+    acc = T::gcomb(acc, __ldcv((const Grid*)(own + ((size_t)par * kTeamMaxRanks + j) * 16)));  // no stale L1
+  }
+  return acc;
+}
 
 template <class T>
 __device__ __forceinline__ void store_out(typename T::Grid g, const KParams& p) {
+  if (p.team.k > 0) g = team_exchange<T>(g, p.team);
   if (p.raw_out) *(typename T::Grid*)p.out = g;
   else T::finalize(g, p.out);
 }
@@ -210,11 +255,13 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
 
 // Second pass of GC_TWO_PASS and the cross-chunk / cross-rank combine.
 template <int DT, int OP>
-__global__ void __launch_bounds__(1024) k_combine(const void* vals, long long count, void* out, int raw_out) {
+__global__ void __launch_bounds__(1024) k_combine(const void* vals, long long count, void* out, int raw_out,
+                                                 TeamArgs team) {
   using T = Tr<DT, OP>;
   pdl_wait();
   typename T::Grid x = reduce_grid_values<T>((const typename T::Grid*)vals, count);
   if (threadIdx.x == 0) {
+    if (team.k > 0) x = team_exchange<T>(x, team);
     if (raw_out) *(typename T::Grid*)out = x;
     else T::finalize(x, out);
   }
@@ -242,6 +289,9 @@ inline KParams make_params(const LaunchDesc& d) {
   p.nslots = d.nslots < 1 ? 1 : d.nslots;
   p.ticket = d.ticket;
   p.partials = d.partials;
+  p.team = d.team;
+  // TWO_PASS: the exchange happens in the second kernel, not per block
+  if (d.gc == GC_TWO_PASS) p.team.k = 0;
   return p;
 }
 
@@ -288,7 +338,8 @@ inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& 
 
 // k_combine with the same programmatic-dependent-launch attribute.
 template <int DT, int OP>
-cudaError_t launch_combine_kernel(const void* vals, long long count, void* out, int raw_out, int block, cudaStream_t s) {
+cudaError_t launch_combine_kernel(const void* vals, long long count, void* out, int raw_out, int block, cudaStream_t s,
+                                  TeamArgs team) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(1, 1, 1);
   cfg.blockDim = dim3(block, 1, 1);
@@ -298,8 +349,9 @@ cudaError_t launch_combine_kernel(const void* vals, long long count, void* out, 
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = pdl_enabled() ? 1 : 0;
-  return cudaLaunchKernelEx(&cfg, k_combine<DT, OP>, vals, count, out, raw_out);
+  return cudaLaunchKernelEx(&cfg, k_combine<DT, OP>, vals, count, out, raw_out, team);
 }
+
 
 template <int DT, int OP, int U, int STAGE>
 cudaError_t launch_bc(const LaunchDesc& d, const KParams& p, cudaStream_t s) {
@@ -340,7 +392,8 @@ cudaError_t launch_op(const LaunchDesc& d, cudaStream_t s) {
   if (e != cudaSuccess || d.gc != GC_TWO_PASS) return e;
   // the second pass: one block, 4 loads in flight per thread; 256 threads up to
   // 4096 partials, else 1024
-  return launch_combine_kernel<DT, OP>(d.partials, (long long)d.grid, d.out, d.raw_out, d.grid <= 4096 ? 256 : 1024, s);
+  return launch_combine_kernel<DT, OP>(d.partials, (long long)d.grid, d.out, d.raw_out, d.grid <= 4096 ? 256 : 1024, s,
+                                       d.team);
 }
 
 template <int DT>
@@ -357,13 +410,14 @@ cudaError_t launch_dt(const LaunchDesc& d, cudaStream_t s) {
 }
 
 template <int DT>
-cudaError_t combine_dt(int op, const void* vals, long long count, void* out, int raw_out, int block, cudaStream_t s) {
+cudaError_t combine_dt(int op, const void* vals, long long count, void* out, int raw_out, int block, cudaStream_t s,
+                       TeamArgs t) {
   switch (op) {
-    case OP_SUM: return launch_combine_kernel<DT, OP_SUM>(vals, count, out, raw_out, block, s);
-    case OP_MIN: return launch_combine_kernel<DT, OP_MIN>(vals, count, out, raw_out, block, s);
-    case OP_MAX: return launch_combine_kernel<DT, OP_MAX>(vals, count, out, raw_out, block, s);
+    case OP_SUM: return launch_combine_kernel<DT, OP_SUM>(vals, count, out, raw_out, block, s, t);
+    case OP_MIN: return launch_combine_kernel<DT, OP_MIN>(vals, count, out, raw_out, block, s, t);
+    case OP_MAX: return launch_combine_kernel<DT, OP_MAX>(vals, count, out, raw_out, block, s, t);
     case OP_SUMACC:
-      if constexpr (DT != DT_I32) return launch_combine_kernel<DT, OP_SUMACC>(vals, count, out, raw_out, block, s);
+      if constexpr (DT != DT_I32) return launch_combine_kernel<DT, OP_SUMACC>(vals, count, out, raw_out, block, s, t);
       break;
   }
   return cudaErrorInvalidValue;
