@@ -51,7 +51,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--sharded", action="store_true",
-                    help="use the sharded reduce_multi path even at one rank (exercises S7 on one GPU)")
+                    help="use the sharded path even at one rank (exercises S7 on one GPU)")
+    ap.add_argument("--collective", default="team", choices=["team", "nccl"],
+                    help="cross-GPU combine: 'team' = fused into the reduction kernel over peer memory "
+                         "(reduce_multi_team), 'nccl' = one ncclAllReduce of the per-rank scalar")
     return ap.parse_args()
 
 
@@ -177,9 +180,12 @@ def run_reference(args, rank, world):
 def workload_config(args, world, plan, sharded=False):
     cfg = {"workload": f"fp32 sum of {args.n} (2^{args.n.bit_length() - 1}) elements per GPU"
                        + (" -- BASELINE configs[1] largest point" if world == 1 else
-                          f" -- BASELINE configs[4] sharded sum, {world} GPUs, NCCL all-reduce of partials"),
+                          f" -- BASELINE configs[4] sharded sum, {world} GPUs, per-rank partials combined "
+                          + ("in the reduction kernel over peer memory (reduce_multi_team)" if args.collective == "team"
+                             else "by one NCCL all-reduce")),
            "n_per_gpu": args.n, "total_bytes": args.n * 4 * world, "op": "sum", "mode": args.mode,
            "parallelism": f"shard{world}" if (world > 1 or sharded) else "single-gpu",
+           "collective": args.collective if (world > 1 or sharded) else None,
            "l2": "inputs (4 B x n per GPU) larger than the 126 MB L2 between steps; no flush needed",
            "distribution": "U[0,1) fp32, numpy PCG64 seed 2019+1000*1+log2(n)+rank"}
     if plan is not None:
@@ -216,13 +222,17 @@ def main():
     x = torch.from_numpy(x_host).to(dev)
     out = torch.empty(1, dtype=torch.float32, device=dev)
     stream = torch.cuda.Stream(dev)
-    comm = rb.Comm() if sharded else None
+    comm = None
+    if sharded:
+        comm = rb.Team() if args.collective == "team" else rb.Comm()
     plan = rb.query_plan("float32", "sum", n, in_ptr=x.data_ptr(), mode=args.mode)
     rb.prepare(stream, n)
 
     def step():
         if comm is None:
             rb.reduce(x, "sum", out=out, stream=stream, mode=args.mode)
+        elif args.collective == "team":
+            rb.reduce_multi_team(x, "sum", comm, out=out, stream=stream, mode=args.mode)
         else:
             rb.reduce_multi(x, "sum", comm, out=out, stream=stream, mode=args.mode)
 
@@ -325,7 +335,10 @@ def main():
             with torch.cuda.stream(stream):
                 for _ in range(k_e2e):
                     xd.copy_(pinned, non_blocking=True)
-                    rb.reduce_multi(xd, "sum", comm, out=out, stream=stream, mode=args.mode)
+                    if args.collective == "team":
+                        rb.reduce_multi_team(xd, "sum", comm, out=out, stream=stream, mode=args.mode)
+                    else:
+                        rb.reduce_multi(xd, "sum", comm, out=out, stream=stream, mode=args.mode)
                     out.item()
             dt = (time.perf_counter() - t0) / k_e2e
             t = torch.tensor([dt], dtype=torch.float64, device=dev)
@@ -334,7 +347,7 @@ def main():
         e2e = {"value": round(world * n * 4 / dt / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": n * 4,
                "d2h_bytes_per_step": 4, "ms_per_step": round(dt * 1e3, 3),
                "path": "reduce_host (C ABI, pinned host buffer, chunked H2D overlapped with the chunk reductions)"
-               if comm is None else "pinned H2D copy + reduce_multi + D2H of the result"}
+               if comm is None else f"pinned H2D copy + reduce_multi ({args.collective}) + D2H of the result"}
 
     # ---- size sweep (N = 1): device time per call from a CUDA graph of R calls
     # over disjoint, never-recently-touched regions of the resident 1 GiB input
@@ -538,14 +551,15 @@ def main():
                    "kind": "paper-style OpenMP reduce pragma (P:L469), context only"}
 
     if rank == 0:
-        launches_per_step = plan["launches"] + (0 if comm is None else 1)
+        launches_per_step = plan["launches"] + (1 if (comm is not None and args.collective == "nccl") else 0)
         line = {
             "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
             "data": "synthetic", "config": workload_config(args, world, plan, comm is not None),
             "elements_per_s": round(world * n / (ms * 1e-3), 1),
-            "launch": "cuda-graph replay of the K steps" if comm is None else "stream (K reduce_multi calls)",
+            "launch": "cuda-graph replay of the K steps" if comm is None else
+                      f"stream (K sharded calls; cross-GPU combine: {args.collective})",
             "stream_launched": None if stream_ms is None else {
                 "ms_per_step": round(stream_ms, 5), "value": round(world * n * 4 / (stream_ms * 1e-3) / 1e9, 2)},
             "frac_of_hbm_peak": round(value / world / peak, 4),
@@ -569,6 +583,8 @@ def main():
         print(json.dumps(line), flush=True)
     if comm is not None:
         torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()  # no member may unmap its team buffer while others still use it
         comm.destroy()
         dist.destroy_process_group()
 
