@@ -85,7 +85,7 @@ class ClockSampler:
     }
 
     def __init__(self, index: int):
-        self.samples, self.reasons, self.ok = [], set(), False
+        self.samples, self.mem_samples, self.reasons, self.ok = [], [], set(), False
         try:
             import pynvml
             pynvml.nvmlInit()
@@ -101,6 +101,7 @@ class ClockSampler:
         while not self._stop.is_set():
             try:
                 self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.mem_samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_MEM))
                 r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
                 for k, bit in self.REASONS.items():
                     if r & bit:
@@ -124,7 +125,8 @@ class ClockSampler:
         if not self.ok:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "error": getattr(self, "err", "")}
         return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
-                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples),
+                "mem_mhz": statistics.median(self.mem_samples) if self.mem_samples else None}
 
 
 def host_info():
