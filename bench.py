@@ -129,6 +129,20 @@ class ClockSampler:
                 "mem_mhz": statistics.median(self.mem_samples) if self.mem_samples else None}
 
 
+def gpu_identity(index: int):
+    try:
+        import pynvml
+        pynvml.nvmlInit()
+        h = pynvml.nvmlDeviceGetHandleByIndex(index)
+        name = pynvml.nvmlDeviceGetName(h)
+        serial = pynvml.nvmlDeviceGetSerial(h)
+        bus = pynvml.nvmlDeviceGetPciInfo(h).busId
+        dec = lambda v: v.decode() if isinstance(v, bytes) else v
+        return {"name": dec(name), "serial": dec(serial), "pci_bus": dec(bus)}
+    except Exception as e:
+        return {"error": repr(e)[:80]}
+
+
 def host_info():
     model = ""
     try:
@@ -308,13 +322,36 @@ def main():
     kavg = ms if (comm is None and plan["launches"] == 1) else k_event
     peak, peak_src = measured_peaks()
     achieved = n * 4 / (kavg * 1e-3) / 1e9
+    # the same copy the driver's MEASURED_PEAKS uses (b.copy_(a), 1 Gi bf16,
+    # read + write bytes, best of 10), on THIS box: B200s in the pool differ
+    copy_gbs = None
+    try:
+        ca = torch.empty(1 << 30, dtype=torch.bfloat16, device=dev)
+        cb = torch.empty_like(ca)
+        cb.copy_(ca)
+        best_ms = None
+        for _ in range(10):
+            ea, eb = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ea.record()
+            cb.copy_(ca)
+            eb.record()
+            eb.synchronize()
+            t = ea.elapsed_time(eb)
+            best_ms = t if best_ms is None else min(best_ms, t)
+        copy_gbs = round(2 * ca.numel() * 2 / (best_ms * 1e-3) / 1e9, 1)
+        del ca, cb
+        torch.cuda.empty_cache()
+    except Exception:
+        pass
     traffic, ncu_s = ncu_traffic()
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
                 "kernel": "rb::k_reduce<f32,sum,U,Vs,stage> (+ grid combine epilogue)",
                 "algorithmic_bytes_per_launch": n * 4, "avg_launch_ms": round(kavg, 5),
                 "single_launch_event_ms": round(k_event, 5),
-                "peak_source": peak_src, "frac_of_nominal_8TBps": round(achieved / 8000.0, 4)}
+                "peak_source": peak_src, "frac_of_nominal_8TBps": round(achieved / 8000.0, 4),
+                "same_box_copy_gbs": copy_gbs,
+                "frac_of_same_box_copy": None if not copy_gbs else round(achieved / copy_gbs, 4)}
     # kernel share of the step (compare with the committed ncu launch list)
     roofline["kernel_share_of_step"] = round(min(1.0, kavg / ms), 4)
 
@@ -567,6 +604,7 @@ def main():
             "frac_of_hbm_peak": round(value / world / peak, 4),
             "roofline": roofline, "e2e": e2e, "clocks": clocks.summary(),
             "gpu_launches": args.steps * launches_per_step,
+            "gpu": gpu_identity(local),
         }
         if cpu is not None:
             line["cpu_baseline"] = cpu
