@@ -63,21 +63,24 @@ __device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
   return v;
 }
 
+// Scalars by value (taking the address of a kernel-parameter struct would copy
+// it to the stack in every thread of every block -- measured: -18 % bandwidth).
 template <class T>
-__device__ __noinline__ typename T::Grid team_exchange(typename T::Grid x, const TeamArgs& t) {
+__device__ __noinline__ typename T::Grid team_exchange(typename T::Grid x, char* const* bufs, int k, int rank,
+                                                          unsigned epoch) {
   using Grid = typename T::Grid;
-  const int par = t.epoch & 1;
-  for (int j = 0; j < t.k; ++j)
-    __stcg((Grid*)(t.bufs[j] + ((size_t)par * kTeamMaxRanks + t.rank) * 16), x);  // L2 (peer: remote L2)
+  const int par = epoch & 1;
+  for (int j = 0; j < k; ++j)
+    __stcg((Grid*)(bufs[j] + ((size_t)par * kTeamMaxRanks + rank) * 16), x);  // L2 (peer: remote L2)
   __threadfence_system();
-  for (int j = 0; j < t.k; ++j)
-    st_release_sys((unsigned*)(t.bufs[j] + kTeamFlagOff + ((size_t)par * kTeamMaxRanks + t.rank) * 4), t.epoch);
-  const char* own = t.bufs[t.rank];
+  for (int j = 0; j < k; ++j)
+    st_release_sys((unsigned*)(bufs[j] + kTeamFlagOff + ((size_t)par * kTeamMaxRanks + rank) * 4), epoch);
+  const char* own = bufs[rank];
   Grid acc = T::gident();
-  for (int j = 0; j < t.k; ++j) {
+  for (int j = 0; j < k; ++j) {
     const unsigned* f = (const unsigned*)(own + kTeamFlagOff + ((size_t)par * kTeamMaxRanks + j) * 4);
     const long long t0 = clock64();
-    while (ld_acquire_sys(f) != t.epoch) {
+    while (ld_acquire_sys(f) != epoch) {
       __nanosleep(64);
       // a member that never arrives must not hang the GPU: after ~2^35 cycles
       // (> 15 s) abort the kernel -- the error surfaces at the caller's sync
@@ -90,7 +93,7 @@ __device__ __noinline__ typename T::Grid team_exchange(typename T::Grid x, const
 
 template <class T>
 __device__ __forceinline__ void store_out(typename T::Grid g, const KParams& p) {
-  if (p.team.k > 0) g = team_exchange<T>(g, p.team);
+  if (p.team.k > 0) g = team_exchange<T>(g, p.team.bufs, p.team.k, p.team.rank, p.team.epoch);
   if (p.raw_out) *(typename T::Grid*)p.out = g;
   else T::finalize(g, p.out);
 }
@@ -261,7 +264,7 @@ __global__ void __launch_bounds__(1024) k_combine(const void* vals, long long co
   pdl_wait();
   typename T::Grid x = reduce_grid_values<T>((const typename T::Grid*)vals, count);
   if (threadIdx.x == 0) {
-    if (team.k > 0) x = team_exchange<T>(x, team);
+    if (team.k > 0) x = team_exchange<T>(x, team.bufs, team.k, team.rank, team.epoch);
     if (raw_out) *(typename T::Grid*)out = x;
     else T::finalize(x, out);
   }

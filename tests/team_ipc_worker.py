@@ -44,7 +44,8 @@ def main():
     dist.barrier()
     team.destroy()
     dist.destroy_process_group()
-    print(json.dumps({"rank": rank, "checked": count, "fails": fails[:5]}), flush=True)
+    # one write(2) per line: the two workers share torchrun's stdout pipe
+    os.write(1, (json.dumps({"rank": rank, "checked": count, "fails": fails[:5]}) + "\n").encode())
 
 
 if __name__ == "__main__":

@@ -76,7 +76,12 @@ def test_team_two_processes_ipc():
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
                         "--master-addr", "127.0.0.1", "--master-port", "29551", script],
                        capture_output=True, text=True, timeout=900, cwd=ROOT)
-    lines = [json.loads(l) for l in r.stdout.splitlines() if l.startswith("{")]
+    lines, dec = [], json.JSONDecoder()
+    for l in r.stdout.splitlines():
+        while l.startswith("{"):
+            obj, end = dec.raw_decode(l)
+            lines.append(obj)
+            l = l[end:].lstrip()
     assert r.returncode == 0 and len(lines) == world, (r.returncode, r.stdout[-2000:], r.stderr[-3000:])
     for l in lines:
         assert l["checked"] > 0 and not l["fails"], l
