@@ -245,13 +245,18 @@ int reduce_comm_destroy(void* comm);
  * plain pointers.  reduce_multi_team: every member calls it (same order of
  * calls on every rank) with its local shard; the block that completes a
  * rank's local reduction stores the raw value into every member's buffer
- * (P2P), raises a flag (release, system scope), waits for all k flags and
- * combines the k values in rank order -- no collective launch, deterministic
- * for a fixed team.  Every member's *out receives the global result.
+ * (P2P), each 4-byte word paired with the call's epoch in one 8-byte access,
+ * polls its own buffer until all k values carry the epoch and combines them
+ * in rank order -- no collective launch, no fences, deterministic for a fixed
+ * team.  Every member's *out receives the global result.
  *   reduce_team_create(&t, k, rank, handle_out)  handle_out: reduce_team_ipc_handle_bytes() bytes (or NULL)
  *   reduce_team_connect(t, handles)             k handles, rank order, from every member (IPC)
  *   reduce_team_connect_local(t, bufs)          k device pointers (reduce_team_buffer of each member)
- * A member that never calls leaves the others waiting (as with any collective). */
+ * The call counter (epoch) that sequences the exchange lives in the member's
+ * device buffer and is advanced by the kernel, so team calls may be captured
+ * into CUDA graphs and replayed (each replay is one call).  A member that
+ * never calls leaves the others waiting (as with any collective); after ~2^35
+ * cycles (> 15 s) the waiting kernel traps and the caller's sync reports it. */
 int reduce_team_create(void** team_out, int nranks, int rank, void* ipc_handle_out);
 int reduce_team_ipc_handle_bytes(void);
 void* reduce_team_buffer(void* team);

@@ -43,16 +43,19 @@ constexpr int max_block_threads(int dtype, int op, int unroll, int stage = STAGE
 // 8(f) N2, the "one-shot combine fused as the epilogue of the last block").
 // Every rank owns one buffer of kTeamBufBytes; bufs[j] is rank j's buffer as
 // seen from this GPU (a CUDA-IPC / peer mapping over NVLink, or a local pointer).
-//   [0, 2*kTeamMaxRanks*16)           slots[parity][rank]   raw values (<= 16 B)
-//   [kTeamFlagOff, + 2*kTeamMaxRanks*4) flags[parity][rank]  epoch of the value
+//   [0, 2*kTeamMaxRanks*32)  slots[parity][rank]: the raw value (<= 16 B) as
+//                            4 pairs {word, epoch} (flag-in-data, one 8-byte access each)
+//   [kTeamEpochOff, + 4)     this rank's call counter (the epoch)
+// The epoch lives in device memory and is advanced by the kernel itself, so a
+// team call captured in a CUDA graph stays correct on every replay.
 struct TeamArgs {
   char* const* bufs;  // device array of k pointers (nullptr when not a team call)
   int k, rank;
-  unsigned epoch;     // 1, 2, 3, ... per call; parity = epoch & 1
 };
 constexpr int kTeamMaxRanks = 256;
-constexpr size_t kTeamFlagOff = 2 * kTeamMaxRanks * 16;
-constexpr size_t kTeamBufBytes = kTeamFlagOff + 2 * kTeamMaxRanks * 4;
+constexpr size_t kTeamSlotBytes = 32;
+constexpr size_t kTeamEpochOff = 2 * kTeamMaxRanks * kTeamSlotBytes;
+constexpr size_t kTeamBufBytes = kTeamEpochOff + 16;
 
 // One launch of the main reduction kernel (steps S2-S5), fully resolved by the
 // host dispatcher (step S0).
@@ -108,7 +111,7 @@ cudaError_t launch_reduce(const LaunchDesc& d, cudaStream_t s);
 // Reduce `count` Grid-typed values in a fixed order with one block of
 // `block` threads and write the finalised (or raw) result to `out`.
 cudaError_t launch_combine(int dtype, int op, const void* vals, long long count, void* out,
-                           int raw_out, int block, cudaStream_t s, TeamArgs team = TeamArgs{nullptr, 0, 0, 0});
+                           int raw_out, int block, cudaStream_t s, TeamArgs team = TeamArgs{nullptr, 0, 0});
 
 // Write the identity into every accumulator slot of every (dtype, op) and zero
 // the tickets.  slots_base: 9 regions of kMaxSlots*kSlotBytes; tickets: 9 words

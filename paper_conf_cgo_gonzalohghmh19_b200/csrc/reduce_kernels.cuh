@@ -46,54 +46,86 @@ struct KParams {
 };
 
 // ---- one-shot cross-GPU combine through peer memory ------
-// Executed by ONE thread of the block that owns this rank's raw result x:
-// write x into slot [parity][rank] of every team member's buffer (P2P stores
-// over NVLink), make them visible system-wide, raise flag [parity][rank] =
-// epoch in every buffer (release, system scope), then wait until all k flags
-// of the own buffer carry this epoch (acquire) and combine slots 0..k-1 in rank
-// order (deterministic for a fixed team).  Parity double-buffering: a rank can
-// reuse parity p only after every member has set its flag for the following
-// call, i.e. after everyone finished reading parity p.
-__device__ __forceinline__ void st_release_sys(unsigned* p, unsigned v) {
-  asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+// Executed by ONE thread of the block that owns this rank's raw result x.
+// Flag-in-data protocol (as NCCL's "LL"): every 4-byte word of x travels with
+// the call's epoch in the same aligned 8-byte pair {word, epoch}, written to
+// slot [parity][rank] of every member's buffer (P2P stores over NVLink).  A
+// reader polls its own buffer until every pair of every slot 0..k-1 carries
+// the epoch, then combines the k values in rank order (deterministic for a
+// fixed team).  No fences: an 8-byte pair is written and read as one access,
+// so a matching epoch implies the word beside it.  Measured on B200 (tools/
+// probes/probe_fence.cu): fence.acq_rel.sys ~1.1 us each; the release/acquire
+// version of this exchange cost ~5 us per call, this one ~1 us.
+// Parity double-buffering: a rank can reuse parity p only after every member
+// has written its pairs for the following call, i.e. after everyone finished
+// reading parity p.
+__device__ __forceinline__ void st_pairs_sys(unsigned* p, unsigned a, unsigned b, unsigned e) {
+  asm volatile("st.relaxed.sys.global.v4.u32 [%0], {%1, %2, %3, %4};" :: "l"(p), "r"(a), "r"(e), "r"(b), "r"(e)
+               : "memory");
 }
-__device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
-  unsigned v;
-  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
+__device__ __forceinline__ void ld_pairs_sys(const unsigned* p, unsigned& a, unsigned& fa, unsigned& b, unsigned& fb) {
+  asm volatile("ld.relaxed.sys.global.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(a), "=r"(fa), "=r"(b), "=r"(fb) : "l"(p)
+               : "memory");
 }
 
 // Scalars by value (taking the address of a kernel-parameter struct would copy
 // it to the stack in every thread of every block -- measured: -18 % bandwidth).
 template <class T>
-__device__ __noinline__ typename T::Grid team_exchange(typename T::Grid x, char* const* bufs, int k, int rank,
-                                                          unsigned epoch) {
+__device__ __noinline__ typename T::Grid team_exchange(typename T::Grid x, char* const* bufs, int k, int rank) {
   using Grid = typename T::Grid;
+  static_assert(sizeof(Grid) <= 16 && sizeof(Grid) % 4 == 0, "team slot holds <= 4 words");
+  constexpr int NW = sizeof(Grid) / 4;  // data words
+  constexpr int NV = (NW + 1) / 2;      // 16-byte stores of {w, e, w, e}
+  // advance this rank's call counter (every member calls in the same order, so
+  // the counters agree); 0 means "never written" and is skipped so that the
+  // parity still alternates across the wrap: ..., 2^32-1 (odd), 2 (even), 3, ...
+  volatile unsigned* ctr = (volatile unsigned*)(bufs[rank] + kTeamEpochOff);
+  unsigned epoch = *ctr + 1;
+  if (epoch == 0) epoch = 2;
+  *ctr = epoch;
   const int par = epoch & 1;
-  for (int j = 0; j < k; ++j)
-    __stcg((Grid*)(bufs[j] + ((size_t)par * kTeamMaxRanks + rank) * 16), x);  // L2 (peer: remote L2)
-  __threadfence_system();
-  for (int j = 0; j < k; ++j)
-    st_release_sys((unsigned*)(bufs[j] + kTeamFlagOff + ((size_t)par * kTeamMaxRanks + rank) * 4), epoch);
+  unsigned w[4] = {0u, 0u, 0u, 0u};
+  memcpy(w, &x, sizeof(Grid));
+  for (int j = 0; j < k; ++j) {
+    if (j == rank) continue;  // the own value never leaves the register
+    unsigned* dst = (unsigned*)(bufs[j] + ((size_t)par * kTeamMaxRanks + rank) * kTeamSlotBytes);
+#pragma unroll
+    for (int v = 0; v < NV; ++v) st_pairs_sys(dst + 4 * v, w[2 * v], w[2 * v + 1], epoch);
+  }
   const char* own = bufs[rank];
   Grid acc = T::gident();
   for (int j = 0; j < k; ++j) {
-    const unsigned* f = (const unsigned*)(own + kTeamFlagOff + ((size_t)par * kTeamMaxRanks + j) * 4);
-    const long long t0 = clock64();
-    while (ld_acquire_sys(f) != epoch) {
-      __nanosleep(64);
-      // a member that never arrives must not hang the GPU: after ~2^35 cycles
-      // (> 15 s) abort the kernel -- the error surfaces at the caller's sync
-      if (clock64() - t0 > (1ll << 35)) __trap();
+    if (j == rank) {
+      acc = T::gcomb(acc, x);
+      continue;
     }
-    acc = T::gcomb(acc, __ldcv((const Grid*)(own + ((size_t)par * kTeamMaxRanks + j) * 16)));  // no stale L1
+    const unsigned* src = (const unsigned*)(own + ((size_t)par * kTeamMaxRanks + j) * kTeamSlotBytes);
+    unsigned r[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+    for (int v = 0; v < NV; ++v) {
+      unsigned fa, fb;
+      ld_pairs_sys(src + 4 * v, r[2 * v], fa, r[2 * v + 1], fb);
+      if (fa != epoch || fb != epoch) {
+        const long long t0 = clock64();
+        do {
+          __nanosleep(32);
+          // a member that never arrives must not hang the GPU: after ~2^35
+          // cycles (> 15 s) abort the kernel -- the error surfaces at the sync
+          if (clock64() - t0 > (1ll << 35)) __trap();
+          ld_pairs_sys(src + 4 * v, r[2 * v], fa, r[2 * v + 1], fb);
+        } while (fa != epoch || fb != epoch);
+      }
+    }
+    Grid y;
+    memcpy(&y, r, sizeof(Grid));
+    acc = T::gcomb(acc, y);
   }
   return acc;
 }
 
 template <class T>
 __device__ __forceinline__ void store_out(typename T::Grid g, const KParams& p) {
-  if (p.team.k > 0) g = team_exchange<T>(g, p.team.bufs, p.team.k, p.team.rank, p.team.epoch);
+  if (p.team.k > 0) g = team_exchange<T>(g, p.team.bufs, p.team.k, p.team.rank);
   if (p.raw_out) *(typename T::Grid*)p.out = g;
   else T::finalize(g, p.out);
 }
@@ -264,7 +296,7 @@ __global__ void __launch_bounds__(1024) k_combine(const void* vals, long long co
   pdl_wait();
   typename T::Grid x = reduce_grid_values<T>((const typename T::Grid*)vals, count);
   if (threadIdx.x == 0) {
-    if (team.k > 0) x = team_exchange<T>(x, team.bufs, team.k, team.rank, team.epoch);
+    if (team.k > 0) x = team_exchange<T>(x, team.bufs, team.k, team.rank);
     if (raw_out) *(typename T::Grid*)out = x;
     else T::finalize(x, out);
   }

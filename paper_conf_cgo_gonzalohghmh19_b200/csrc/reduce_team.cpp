@@ -5,10 +5,11 @@
 // mapped into every member's address space -- CUDA IPC handles across processes
 // (P2P over NVLink / NVSwitch between GPUs, or the same GPU), or plain pointers
 // within one process -- and the block that finishes a rank's local reduction
-// writes its raw value into every member's buffer, raises a flag, waits for
-// all members' flags and combines the k values in rank order (kernel side:
-// team_exchange in reduce_kernels.cuh).  One launch per call (two for
-// TWO_PASS); the exchange is a few peer stores and one flag wait.
+// writes its raw value, each 4-byte word paired with the call's epoch, into
+// every member's buffer, polls its own buffer until all k values carry the
+// epoch and combines them in rank order (kernel side: team_exchange in
+// reduce_kernels.cuh).  One launch per call (two for TWO_PASS); the exchange is
+// a few peer stores and one poll, no fences and no collective launch.
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -25,7 +26,6 @@ struct Team {
   std::vector<char*> bufs;
   std::vector<bool> ipc_opened;
   char** d_bufs = nullptr;
-  unsigned epoch = 0;
   bool connected = false;
   std::mutex mu;
 };
@@ -56,7 +56,7 @@ int reduce_team_create(void** team_out, int nranks, int rank, void* ipc_handle_o
   t->ipc_opened.assign(nranks, false);
   cudaError_t e = cudaGetDevice(&t->device);
   if (e == cudaSuccess) e = cudaMalloc(&t->own, kTeamBufBytes);
-  if (e == cudaSuccess) e = cudaMemset(t->own, 0, kTeamBufBytes);  // flags start at epoch 0
+  if (e == cudaSuccess) e = cudaMemset(t->own, 0, kTeamBufBytes);  // flags and counter start at 0
   if (e == cudaSuccess) e = cudaMalloc(&t->d_bufs, sizeof(char*) * nranks);
   if (e == cudaSuccess && ipc_handle_out) {
     cudaIpcMemHandle_t h;
@@ -139,9 +139,7 @@ int reduce_multi_team(int dtype, int op, const void* in_local, size_t n_local, v
     std::lock_guard<std::mutex> lk(t->mu);
     P.d.team.bufs = t->d_bufs;
     P.d.team.k = t->k;
-    P.d.team.rank = t->rank;
-    P.d.team.epoch = ++t->epoch;
-    if (t->epoch == 0) P.d.team.epoch = ++t->epoch;  // 0 is the "never written" flag value
+    P.d.team.rank = t->rank;  // the epoch is advanced on the device (graph-capturable)
   }
   return launch_plan(&P, ws, out, (cudaStream_t)stream);
 }

@@ -70,6 +70,48 @@ def test_team_streams_in_process(k):
             t.destroy()
 
 
+def test_team_graph_replay():
+    """Team calls captured once per member into CUDA graphs and replayed: the
+    epoch is advanced on the device, so every replay is a fresh exchange (new
+    input values must show up in every member's result)."""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    k, n = 2, (1 << 20) + 11
+    team = rb.Team.local(k)
+    streams = [torch.cuda.Stream() for _ in range(k)]
+    try:
+        shards, outs, graphs = [], [], []
+        for r in range(k):
+            lo, hi = rb.shard_range(n, k, r)
+            shards.append(torch.zeros(hi - lo, dtype=torch.int32, device="cuda"))
+            outs.append(torch.zeros(1, dtype=torch.int32, device="cuda"))
+        torch.cuda.synchronize()
+        for r in range(k):  # warm (first call allocates the stream's workspace)
+            rb.reduce_multi_team(shards[r], "sum", team[r], out=outs[r], stream=streams[r])
+        torch.cuda.synchronize()
+        for r in range(k):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=streams[r]):
+                rb.reduce_multi_team(shards[r], "sum", team[r], out=outs[r], stream=streams[r])
+            graphs.append(g)
+        torch.cuda.synchronize()
+        for rep in range(6):
+            x = synth.make("int32", n, "int_full", 500 + rep)
+            for r in range(k):
+                lo, hi = rb.shard_range(n, k, r)
+                shards[r].copy_(torch.from_numpy(x[lo:hi]))
+            torch.cuda.synchronize()
+            for r in range(k):
+                with torch.cuda.stream(streams[r]):
+                    graphs[r].replay()
+            torch.cuda.synchronize()
+            _check_all(x, "sum", [o.cpu().numpy() for o in outs])
+    finally:
+        torch.cuda.synchronize()
+        for t in team:
+            t.destroy()
+
+
 def test_team_two_processes_ipc():
     script = os.path.join(ROOT, "tests", "team_ipc_worker.py")
     world = 2
