@@ -51,6 +51,7 @@ constexpr int max_block_threads(int dtype, int op, int unroll, int stage = STAGE
 struct TeamArgs {
   char* const* bufs;  // device array of k pointers (nullptr when not a team call)
   int k, rank;
+  int shared_gpu;     // another member runs on this GPU (no early PDL trigger)
 };
 constexpr int kTeamMaxRanks = 256;
 constexpr size_t kTeamSlotBytes = 32;
@@ -111,7 +112,7 @@ cudaError_t launch_reduce(const LaunchDesc& d, cudaStream_t s);
 // Reduce `count` Grid-typed values in a fixed order with one block of
 // `block` threads and write the finalised (or raw) result to `out`.
 cudaError_t launch_combine(int dtype, int op, const void* vals, long long count, void* out,
-                           int raw_out, int block, cudaStream_t s, TeamArgs team = TeamArgs{nullptr, 0, 0});
+                           int raw_out, int block, cudaStream_t s, TeamArgs team = TeamArgs{nullptr, 0, 0, 0});
 
 // Write the identity into every accumulator slot of every (dtype, op) and zero
 // the tickets.  slots_base: 9 regions of kMaxSlots*kSlotBytes; tickets: 9 words

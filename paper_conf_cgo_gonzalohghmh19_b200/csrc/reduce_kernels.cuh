@@ -216,8 +216,12 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
   // its start (the next grid fills SMs as this one drains); in a one-wave or
   // persistent grid every block triggers after its main loop (triggering at
   // the start would park the next grid's CTAs on the SMs for the whole run).
+  // A team call whose members share this GPU never triggers: the next grid's
+  // parked CTAs could fill the SMs a co-resident member needs to reach the
+  // exchange this grid's last block is waiting in.
   pdl_wait();
-  const bool early_trigger = gridDim.x > kPdlTriggerWindow && blockIdx.x + kPdlTriggerWindow >= gridDim.x;
+  const bool may_trigger = !p.team.shared_gpu;
+  const bool early_trigger = may_trigger && gridDim.x > kPdlTriggerWindow && blockIdx.x + kPdlTriggerWindow >= gridDim.x;
   if (early_trigger) pdl_trigger();
   if (p.gc == GC_CLUSTER) cluster_arrive_relaxed();  // phase 1: "this CTA has started"
   Part<T> a[T::NA];
@@ -275,7 +279,7 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
       }
     }
   }
-  if (!early_trigger && gridDim.x <= kPdlTriggerWindow) pdl_trigger();
+  if (may_trigger && !early_trigger && gridDim.x <= kPdlTriggerWindow) pdl_trigger();
   if (blockIdx.x == gridDim.x - 1) {
     using Elem = typename T::Elem;
     const int t = threadIdx.x;

@@ -27,11 +27,20 @@ struct Team {
   std::vector<bool> ipc_opened;
   char** d_bufs = nullptr;
   bool connected = false;
+  bool shared_gpu = false;  // some peer buffer lives on this member's GPU
   std::mutex mu;
 };
 
 int team_upload(Team* t) {
   t->bufs[t->rank] = t->own;
+  t->shared_gpu = false;
+  for (int j = 0; j < t->k; ++j) {
+    if (j == t->rank) continue;
+    cudaPointerAttributes a;
+    cudaError_t e = cudaPointerGetAttributes(&a, t->bufs[j]);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaPointerGetAttributes (team peer buffer)");
+    if (a.device == t->device) t->shared_gpu = true;
+  }
   cudaError_t e = cudaMemcpy(t->d_bufs, t->bufs.data(), sizeof(char*) * t->k, cudaMemcpyHostToDevice);
   if (e != cudaSuccess) return cuda_fail(e, "team pointer upload");
   t->connected = true;
@@ -140,6 +149,7 @@ int reduce_multi_team(int dtype, int op, const void* in_local, size_t n_local, v
     P.d.team.bufs = t->d_bufs;
     P.d.team.k = t->k;
     P.d.team.rank = t->rank;  // the epoch is advanced on the device (graph-capturable)
+    P.d.team.shared_gpu = t->shared_gpu ? 1 : 0;
   }
   return launch_plan(&P, ws, out, (cudaStream_t)stream);
 }

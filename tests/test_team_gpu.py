@@ -70,6 +70,36 @@ def test_team_streams_in_process(k):
             t.destroy()
 
 
+def test_team_same_gpu_back_to_back():
+    """Two members on one GPU, 40 calls each queued on their streams with no
+    host sync in between (large grids, so programmatic dependent launch would
+    let the next call's CTAs park on the SMs): members sharing a GPU do not
+    trigger early, so neither member can starve the other out of the exchange."""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    k, n, iters = 2, (1 << 25) + 3, 40
+    team = rb.Team.local(k)
+    streams = [torch.cuda.Stream() for _ in range(k)]
+    try:
+        x = synth.make("float32", n, "uniform_pm1", 4242)
+        shards = []
+        for r in range(k):
+            lo, hi = rb.shard_range(n, k, r)
+            shards.append(torch.from_numpy(x[lo:hi]).cuda())
+        outs = [[torch.empty(1, device="cuda") for _ in range(iters)] for _ in range(k)]
+        torch.cuda.synchronize()
+        for it in range(iters):
+            for r in range(k):
+                rb.reduce_multi_team(shards[r], "sum", team[r], out=outs[r][it], stream=streams[r])
+        torch.cuda.synchronize()
+        for it in range(iters):
+            _check_all(x, "sum", [outs[r][it].cpu().numpy() for r in range(k)])
+    finally:
+        torch.cuda.synchronize()
+        for t in team:
+            t.destroy()
+
+
 def test_team_graph_replay():
     """Team calls captured once per member into CUDA graphs and replayed: the
     epoch is advanced on the device, so every replay is a fresh exchange (new
