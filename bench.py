@@ -45,7 +45,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=300)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=N_PER_GPU, help="elements per GPU")
+    ap.add_argument("--n", "--elements", dest="n", type=int, default=N_PER_GPU,
+                    help="elements per GPU (spell it --elements under torchrun, whose parser eats --n)")
     ap.add_argument("--mode", default="fast", choices=["fast", "deterministic"])
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -55,6 +56,9 @@ def parse():
     ap.add_argument("--collective", default="team", choices=["team", "nccl"],
                     help="cross-GPU combine: 'team' = fused into the reduction kernel over peer memory "
                          "(reduce_multi_team), 'nccl' = one ncclAllReduce of the per-rank scalar")
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="TEST MODE: every rank on cuda:0, gloo control plane, team combine over CUDA IPC "
+                         "(validates the multi-rank path on a one-GPU box; timings are not scaling numbers)")
     return ap.parse_args()
 
 
@@ -224,6 +228,9 @@ def main():
     import synth
     import paper_conf_cgo_gonzalohghmh19_b200 as rb
 
+    if args.share_gpu and args.collective != "team":
+        raise SystemExit("--share-gpu needs --collective team (NCCL refuses two ranks on one GPU)")
+    local = 0 if args.share_gpu else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     sharded = world > 1 or args.sharded
@@ -232,7 +239,18 @@ def main():
         os.environ.setdefault("MASTER_PORT", "29533")
         os.environ.setdefault("RANK", str(rank))
         os.environ.setdefault("WORLD_SIZE", str(world))
-        dist.init_process_group("nccl", device_id=dev)
+        if args.share_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
+
+    def allmax(v):
+        """max over ranks of a host float (device tensor for NCCL, host for gloo)"""
+        if world == 1 and not sharded:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device="cpu" if args.share_gpu else dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
     n = args.n
     x_host = synth.make("float32", n, "uniform01", synth.seed_for(1, n, rank))
     x = torch.from_numpy(x_host).to(dev)
@@ -290,10 +308,24 @@ def main():
     sync_all()
     ms = e0.elapsed_time(e1) / args.steps
     if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = allmax(ms)
     value = world * n * 4 / (ms * 1e-3) / 1e9
+    # sharded: the same K steps without the cross-rank combine (local reduce
+    # only), so the combine's cost per step is visible
+    decomposition = None
+    if comm is not None:
+        sync_all()
+        with torch.cuda.stream(stream):
+            e0.record(stream)
+            for _ in range(args.steps):
+                rb.reduce(x, "sum", out=out, stream=stream, mode=args.mode)
+            e1.record(stream)
+        e1.synchronize()
+        local_ms = allmax(e0.elapsed_time(e1) / args.steps)
+        sync_all()
+        decomposition = {"local_reduce_ms_per_step": round(local_ms, 5),
+                         "combine_us_per_step": round((ms - local_ms) * 1e3, 3),
+                         "how": "max over ranks of K stream-launched local reduce() calls vs the K sharded calls"}
     stream_ms = None
     if graph is not None:  # the same K steps launched one by one from the host
         with torch.cuda.stream(stream):
@@ -379,10 +411,7 @@ def main():
                     else:
                         rb.reduce_multi(xd, "sum", comm, out=out, stream=stream, mode=args.mode)
                     out.item()
-            dt = (time.perf_counter() - t0) / k_e2e
-            t = torch.tensor([dt], dtype=torch.float64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            dt = float(t.item())
+            dt = allmax((time.perf_counter() - t0) / k_e2e)
         e2e = {"value": round(world * n * 4 / dt / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": n * 4,
                "d2h_bytes_per_step": 4, "ms_per_step": round(dt * 1e3, 3),
                "path": "reduce_host (C ABI, pinned host buffer, chunked H2D overlapped with the chunk reductions)"
@@ -606,6 +635,10 @@ def main():
             "gpu_launches": args.steps * launches_per_step,
             "gpu": gpu_identity(local),
         }
+        if decomposition is not None:
+            line["sharded_decomposition"] = decomposition
+        if args.share_gpu:
+            line["test_mode"] = "--share-gpu: all ranks on one GPU (code-path check, not a scaling number)"
         if cpu is not None:
             line["cpu_baseline"] = cpu
             line["cpu_openmp"] = cpu_omp
