@@ -28,7 +28,17 @@ for dt in (torch.int32, torch.float32, torch.float64):
     if dt != torch.float64:
         for nb in (7, 20000, 1 << 20):
             rb.histogram(base, 0, 4000, nb)
+# team combine (k = 1: members on one GPU cannot run concurrently under the
+# sanitizer, which serialises kernels, so k > 1 would wait for itself)
+team = rb.Team.local(1)[0]
+for dt in (torch.int32, torch.float32, torch.float64):
+    for n in (0, 33, (1 << 20) + 3):
+        x = torch.arange(n + 1, device="cuda").to(dt)[1:]
+        for op in ("sum", "min", "max"):
+            for kw in (dict(), dict(mode="deterministic"), dict(grid_combine=4, grid=8)):
+                rb.reduce_multi_team(x, op, team, **kw)
 torch.cuda.synchronize()
+team.destroy()
 print("ok")
 PY
 rc=0
