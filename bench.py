@@ -553,14 +553,19 @@ def main():
             o3 = torch.empty(4096, dtype=tdt, device=dev)
             for op in ("sum", "min", "max"):
                 row = {"dtype": dt_name, "op": op, "n": m}
-                for mode in ("fast", "deterministic"):
-                    def launch_3(t, op=op, mode=mode, o3=o3):
+                # atomic = "DT,A" (red.global per block + ticket), tree = strict
+                # deterministic (partials + k_combine), auto = the table's fast-mode pick
+                arms = (("atomic", dict(grid_combine=1)), ("tree", dict(mode="deterministic", grid_combine=2)),
+                        ("auto_fast", dict()), ("auto_deterministic", dict(mode="deterministic")))
+                for arm, kw in arms:
+                    def launch_3(t, op=op, kw=kw, o3=o3):
                         ctr[0] = (ctr[0] + 1) % 4096
-                        rb.reduce(t, op, out=o3[ctr[0]:ctr[0] + 1], stream=stream, mode=mode)
+                        rb.reduce(t, op, out=o3[ctr[0]:ctr[0] + 1], stream=stream, **kw)
                     sec = time_calls(launch_3, regs_w, regs_t, stream, repeats=2)
-                    pp = rb.query_plan(dt_name, op, m, in_ptr=regs_t[0].data_ptr(), mode=mode)
-                    row[mode] = {"us": round(sec * 1e6, 2), "GBps": round(m * es / sec / 1e9, 1),
-                                 "grid_combine": ["direct", "atomic", "two_pass", "last_block", "cluster"][pp["grid_combine"]]}
+                    pp = rb.query_plan(dt_name, op, m, in_ptr=regs_t[0].data_ptr(), **kw)
+                    row[arm] = {"us": round(sec * 1e6, 2), "GBps": round(m * es / sec / 1e9, 1),
+                                "grid_combine": ["direct", "atomic", "two_pass", "last_block", "cluster"][pp["grid_combine"]],
+                                "grid": pp["grid"], "block": pp["block"], "unroll": pp["unroll"]}
                 cfg3.append(row)
 
     # ---- BASELINE configs[4] at k = 1: one 8 GiB (2^31 fp32) array on one GPU

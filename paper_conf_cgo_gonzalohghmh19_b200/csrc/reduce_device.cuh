@@ -93,6 +93,12 @@ __device__ __forceinline__ double dmax_sel(double a, double b) {
 __device__ __forceinline__ double dmin_sel(double a, double b) {
   double r; asm("min.f64 %0, %1, %2;" : "=d"(r) : "d"(a), "d"(b)); return r;
 }
+// 1 iff a or b is NaN (one unordered compare for two elements)
+__device__ __forceinline__ uint32_t dnan2(double a, double b) {
+  uint32_t r;
+  asm("{\n\t.reg .pred p;\n\tsetp.nan.f64 p, %1, %2;\n\tselp.u32 %0, 1, 0, p;\n\t}" : "=r"(r) : "d"(a), "d"(b));
+  return r;
+}
 __device__ __forceinline__ double nan64() { return __longlong_as_double(0x7FF8000000000000ll); }
 
 // Order-preserving keys (reading R3): unsigned order of key(x) == the order
@@ -236,9 +242,27 @@ template <int OP> struct TrF64 {
   using Elem = double;
   using Acc = double;
   using Grid = typename std::conditional<OP == OP_SUM, double, unsigned long long>::type;
-  // sums: vector tree into 2 accumulators; min/max: per-lane select + NaN flag
-  static constexpr int VE = 4, NA = OP == OP_SUM ? 2 : 4, kLaneWords = 2;
-  static constexpr bool kVecTree = OP == OP_SUM;
+  // Vector tree into 2 accumulators.  min/max (kSelNaN): the streaming tree
+  // is plain compare-selects (DSETP + 2 SEL; max.f64 lowers to ~3x that with
+  // its NaN quieting and register shuffles, which made the fp64 min/max loop
+  // issue-bound), and what those selects get wrong is repaired per thread in
+  // finish(): NaN from a sticky flag (aux bit 0, one unordered compare per two
+  // elements), and the sign of a zero result from aux bit 31 -- for max "some
+  // element had its sign bit clear", for min "some element had it set".  If
+  // the max is +-0 every element is <= 0, so a sign-clear element can only be
+  // +0 (or NaN, flagged anyway); symmetrically for min.
+  static constexpr int VE = 4, NA = 2, kLaneWords = 2;
+  static constexpr bool kVecTree = true;
+  static constexpr bool kSelNaN = OP != OP_SUM;
+  __device__ static double sel(double a, double b) { return OP == OP_MIN ? (b < a ? b : a) : (b > a ? b : a); }
+  __device__ static void fold4(double& a, uint32_t& aux, const uint32_t (&r)[8]) {
+    const double x0 = __hiloint2double((int)r[1], (int)r[0]), x1 = __hiloint2double((int)r[3], (int)r[2]);
+    const double x2 = __hiloint2double((int)r[5], (int)r[4]), x3 = __hiloint2double((int)r[7], (int)r[6]);
+    aux |= dnan2(x0, x1) | dnan2(x2, x3);
+    if (OP == OP_MIN) aux |= (r[1] | r[3] | r[5] | r[7]) & 0x80000000u;
+    else aux |= ~(r[1] & r[3] & r[5] & r[7]) & 0x80000000u;
+    a = sel(a, sel(sel(x0, x1), sel(x2, x3)));
+  }
   static constexpr bool kMax = OP == OP_MAX;
   __device__ static double lift(double x) { return x; }
   __device__ static Acc ident() {
@@ -259,7 +283,9 @@ template <int OP> struct TrF64 {
   __device__ static Acc warp(Acc v) { return warp_butterfly(v, [](double x, double y) { return comb(x, y); }); }
   __device__ static Acc finish(Acc a, uint32_t aux) {
     if (OP == OP_SUM) return a;
-    return aux ? nan64() : a;
+    if (aux & 1u) return nan64();
+    if (a == 0.0 && (aux >> 31)) return OP == OP_MIN ? -0.0 : 0.0;
+    return a;
   }
   __device__ static Grid to_grid(Acc a) {
     if constexpr (OP == OP_SUM) return a; else return key64<kMax>(a);
@@ -395,10 +421,16 @@ template <class T> using Part = typename PartOf<T>::type;
 //     accumulator `slot % NA` (NA = 2: two independent chains) -- the same
 //     addition depth as one accumulator per lane, with 6 fewer live registers,
 //     which keeps the small-unroll kernels at 32 registers (full occupancy).
-//   otherwise (accurate sums, fp64 min/max): lane k folds into accumulator k.
+//   fp64 min/max: the same tree of selects, NaN in the sticky flag.
+//   otherwise (accurate sums): lane k folds into accumulator k.
+template <class T, class = void> struct HasSelNaN : std::false_type {};
+template <class T> struct HasSelNaN<T, std::enable_if_t<T::kSelNaN>> : std::true_type {};
+
 template <class T>
 __device__ __forceinline__ void fold_vec(Part<T> (&a)[T::NA], uint32_t& aux, const uint32_t (&r)[8], int slot) {
-  if constexpr (T::kVecTree) {
+  if constexpr (HasSelNaN<T>::value) {
+    T::fold4(a[slot % T::NA], aux, r);
+  } else if constexpr (T::kVecTree) {
     using Acc = typename T::Acc;
     Acc t;
     if constexpr (T::kLaneWords == 1) {

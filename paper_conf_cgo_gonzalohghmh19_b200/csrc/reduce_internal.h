@@ -29,7 +29,11 @@ constexpr int kMaxSmemTileBytes = 128 * 1024;
 // keep 33 % more bytes in flight than the 6 blocks 35-36 registers allow).
 constexpr int min_blocks_hint(int dtype, int op, int unroll, int stage, int max_threads) {
   return (stage == STAGE_REG && (unroll == 1 || (unroll == 2 && dtype != 0)) && op != 3 && !(dtype == 2 && op != 0))
-             ? 2048 / max_threads : 1;
+             ? 2048 / max_threads
+             // fp64 min/max: left alone, ptxas spends 96 registers at U = 4
+             // (2 blocks of 256 per SM, 24 % occupancy, 3.4 TB/s one tile per
+             // block); capped at 64 the loop keeps its loads in flight
+             : (stage == STAGE_REG && dtype == 2 && (op == 1 || op == 2) && unroll <= 4) ? 1024 / max_threads : 1;
 }
 
 constexpr int max_block_threads(int dtype, int op, int unroll, int stage = STAGE_REG) {
