@@ -6,9 +6,13 @@ One step = one pass of the whole hot path (steps S0-S6, plus S7 for N>1) over
 one batch of synthetic input already resident in HBM:
   N = 1 : reduce(fp32, sum) of n = 2^28 elements (1 GiB) -- the largest point
           of BASELINE configs[1] ("fp32 sum size sweep 1K-256M"), the headline.
-  N > 1 : reduce_multi(fp32, sum): every rank reduces its own 2^28-element
-          shard and the per-rank scalars are combined by one NCCL all-reduce
+  N > 1 : reduce_multi_team(fp32, sum): every rank reduces its own 2^28-element
+          shard and the per-rank scalars meet in the kernel's epilogue over
+          peer memory (--collective nccl: one NCCL all-reduce instead; the
+          team path falls back to it if the peer mapping cannot be made)
           (configs[4]: at N = 8 this is the 8 GiB array).  Weak scaling.
+          The sharded result is checked against the sum of the per-rank local
+          results once after warm-up (`cross_rank_check`).
 The 1 GiB per-GPU input is larger than the 126 MB L2, so consecutive steps
 read from HBM without an explicit flush.
 
@@ -257,8 +261,19 @@ def main():
     out = torch.empty(1, dtype=torch.float32, device=dev)
     stream = torch.cuda.Stream(dev)
     comm = None
+    collective_note = None
     if sharded:
-        comm = rb.Team() if args.collective == "team" else rb.Comm()
+        if args.collective == "team":
+            try:
+                comm = rb.Team()
+            except rb.ReduceError as e:  # e.g. no peer mapping between the GPUs: use the NCCL combine
+                if args.share_gpu:
+                    raise
+                collective_note = f"team combine unavailable ({e}); fell back to the NCCL all-reduce"
+                print(f"bench: {collective_note}", file=sys.stderr)
+                args.collective = "nccl"
+        if comm is None:
+            comm = rb.Comm()
     plan = rb.query_plan("float32", "sum", n, in_ptr=x.data_ptr(), mode=args.mode)
     rb.prepare(stream, n)
 
@@ -280,6 +295,23 @@ def main():
         for _ in range(max(3, args.warmup)):
             step()
     sync_all()
+    cross_check = None
+    if comm is not None:
+        # the sharded result against the per-rank local results summed over the
+        # torch process group (an independent path): relative gap must be at
+        # the fp32 rounding level of one final conversion
+        got = float(out.item())
+        loc = torch.empty(1, dtype=torch.float32, device=dev)
+        rb.reduce(x, "sum", out=loc, stream=stream, mode=args.mode)
+        torch.cuda.synchronize(dev)
+        t = torch.tensor([float(loc.item())], dtype=torch.float64, device="cpu" if args.share_gpu else dev)
+        dist.all_reduce(t)
+        want = float(t.item())
+        rel = abs(got - want) / max(abs(want), 1e-30)
+        cross_check = {"sharded": got, "sum_of_local": want, "rel_gap": rel, "ok": rel <= 4 * world * 2.0 ** -24}
+        if not cross_check["ok"]:
+            print(f"bench: sharded result disagrees with the sum of local results: {cross_check}", file=sys.stderr)
+        sync_all()
     # Single GPU: the K steps are captured once into a CUDA graph and replayed
     # (no host launch gaps between steps; the same kernels on the same
     # HBM-resident input).  The plain stream-launched loop is timed as well.
@@ -660,6 +692,10 @@ def main():
         }
         if decomposition is not None:
             line["sharded_decomposition"] = decomposition
+        if cross_check is not None:
+            line["cross_rank_check"] = cross_check
+        if collective_note is not None:
+            line["config"]["collective_note"] = collective_note
         if args.share_gpu:
             line["test_mode"] = "--share-gpu: all ranks on one GPU (code-path check, not a scaling number)"
         if cpu is not None:

@@ -347,12 +347,25 @@ class Team:
         nb = lib.reduce_team_ipc_handle_bytes()
         hbuf = (ctypes.c_char * nb)()
         handle = ctypes.c_void_p()
-        _check(lib.reduce_team_create(ctypes.byref(handle), world, rank, ctypes.cast(hbuf, ctypes.c_void_p)),
-               "reduce_team_create")
+        # every step is agreed over the group, so a failure on one rank raises on
+        # all of them instead of leaving the others blocked in a collective
+        st = lib.reduce_team_create(ctypes.byref(handle), world, rank, ctypes.cast(hbuf, ctypes.c_void_p))
+        err = None if st == OK else (st, last_error())
         allh = [None] * world
-        dist.all_gather_object(allh, bytes(hbuf), group=group)
-        joined = (ctypes.c_char * (nb * world)).from_buffer_copy(b"".join(allh))
-        _check(lib.reduce_team_connect(handle, ctypes.cast(joined, ctypes.c_void_p)), "reduce_team_connect")
+        dist.all_gather_object(allh, (st, bytes(hbuf)), group=group)
+        if st == OK and all(s == OK for s, _ in allh):
+            joined = (ctypes.c_char * (nb * world)).from_buffer_copy(b"".join(h for _, h in allh))
+            st = lib.reduce_team_connect(handle, ctypes.cast(joined, ctypes.c_void_p))
+            err = None if st == OK else (st, last_error())
+        else:
+            st = st if st != OK else next(s for s, _ in allh if s != OK)
+        sts = [None] * world
+        dist.all_gather_object(sts, st, group=group)
+        if any(s != OK for s in sts):
+            if handle.value:
+                lib.reduce_team_destroy(handle)
+            bad = next(r for r, s in enumerate(sts) if s != OK)
+            raise ReduceError(sts[bad], f"Team (rank {bad} failed{'' if err is None else ': ' + err[1]})")
         self.handle, self.rank, self.world = handle.value, rank, world
 
     @classmethod
