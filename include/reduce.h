@@ -130,10 +130,13 @@ typedef struct {
                          is also the table's, else one block per tile), -1 = one
                          block per tile, > 0 = at most this many blocks (persistent);
                          for REDUCE_GC_CLUSTER: the cluster size, 1..16 (0 = 16) */
-  int seg_group;      /* reduce_segmented / reduce_batched only: 0 = auto (8 lanes per
-                         segment for uniform segments <= 128 elements, one warp for
-                         <= 4096 and for offset arrays, else one block), 1 = one
-                         warp per segment, 2 = one block per segment, 3 = 8 lanes */
+  int seg_group;      /* reduce_segmented / reduce_batched only: 0 = auto (uniform
+                         rows: one thread per row up to 512 bytes, 8 lanes up to 4 KB,
+                         one warp up to 16 KB, else one block; offset arrays: 8 lanes),
+                         1 = one warp per segment, 2 = one block per segment,
+                         3 = 8 lanes, 4 = one thread.  Whatever the group, segments
+                         much longer than its first round are cut into 64 KB chunks
+                         that whole blocks reduce (two more launches; load balance) */
   int stage;          /* 0 = auto; REDUCE_STAGE_REG: 256-bit loads straight into
                          registers; REDUCE_STAGE_SMEM: cp.async 16-byte copies into a
                          shared-memory tile (block*unroll*32 <= 128 KiB), then shared
@@ -168,6 +171,8 @@ int reduce_query_plan(int dtype, int op, const void* in, size_t n, const reduce_
 
 /* Allocate (or grow) the workspace of (current device, stream) so that calls
  * with up to `max_n` elements need no allocation -- call before graph capture.
+ * Also allocates the stream's segment queue (reduce_segmented / reduce_batched;
+ * a capture without it runs those calls without load balancing).
  * Also re-initialises the atomic accumulators and tickets (recovery after an
  * aborted kernel). */
 int reduce_prepare(reduce_stream_t stream, size_t max_n);
@@ -189,11 +194,15 @@ int reduce_host(int dtype, int op, const void* host_in, size_t n, void* host_out
  * i < num_segments.  `offsets` is a DEVICE array of num_segments + 1 int64
  * element offsets (non-decreasing; a decreasing pair is treated as an empty
  * segment, which yields the identity); `out` is a DEVICE array of
- * num_segments elements of dtype.  One warp or one block per segment (the
- * paper's small-array versions assign one warp / block per partition with no
- * global atomics): one launch, no atomics, deterministic.
- * Segment starts may have any element alignment.  Options used: block
- * (32..512, default 256), seg_group.  reduce_batched is the uniform case: num_segments rows of seg_len
+ * num_segments elements of dtype.  One thread, 8 lanes, one warp or one block
+ * per segment (the paper's small-array versions assign one warp / block per
+ * partition with no global atomics); segments much longer than
+ * their group's first round are cut into 64 KB chunks that whole blocks reduce,
+ * then combined in chunk order (the stream's workspace holds the queue; two
+ * more launches; load balance for skewed lengths).  Values never touch
+ * atomics and every combine has a fixed order: deterministic.  Up to 3
+ * launches (1 for uniform rows too short to be cut).  Segment starts may have
+ * any element alignment.  Options used: block (32..512, default 256), seg_group.  reduce_batched is the uniform case: num_segments rows of seg_len
  * contiguous elements (row i at in + i*seg_len), no offsets array. */
 int reduce_segmented(int dtype, int op, const void* in, const int64_t* offsets, size_t num_segments, void* out,
                      reduce_stream_t stream, const reduce_opts_t* opts);

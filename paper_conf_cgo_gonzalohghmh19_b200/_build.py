@@ -64,6 +64,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     nvcc = _nvcc()
     inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", _nccl_include()]
     common = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-Xptxas", "-warn-spills"] + inc
+    # experiment hook (tools/probes A/B builds), e.g. REDUCE_B200_NVCC_FLAGS="-DRB_SEG_PIPE=2"
+    common += os.environ.get("REDUCE_B200_NVCC_FLAGS", "").split()
 
     def compile_one(src: str) -> str:
         obj = os.path.join(BUILD, os.path.basename(src) + ".o")

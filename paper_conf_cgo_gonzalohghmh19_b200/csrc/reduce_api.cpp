@@ -240,6 +240,7 @@ static void free_workspace(Workspace* w) {
   cudaSetDevice(w->device);
   if (w->base) cudaFree(w->base);
   if (w->partials) cudaFree(w->partials);
+  if (w->segq) cudaFree(w->segq);
   if (w->staging) cudaFree(w->staging);
   for (int i = 0; i < 2; ++i) {
     if (w->ev_copied[i]) cudaEventDestroy(w->ev_copied[i]);
@@ -306,6 +307,34 @@ int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
   return REDUCE_OK;
 }
 
+// The stream's long-segment queue (allocated and zeroed on first use, or by
+// reduce_prepare before a graph capture).
+int get_seg_queue(cudaStream_t stream, char** out) {
+  Workspace* w = nullptr;
+  int st = get_workspace(stream, 0, &w);
+  if (st != REDUCE_OK) return st;
+  std::lock_guard<std::mutex> lk(g_ws_mu);
+  if (w->segq == nullptr) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone)
+      return fail(REDUCE_ERR_NOT_PREPARED, "segment queue missing during stream capture: call reduce_prepare first");
+    char* q = nullptr;
+    cudaError_t e = cudaMalloc((void**)&q, kSegQBytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(REDUCE_ERR_NO_MEMORY, "cudaMalloc(segment queue) failed");
+    }
+    e = cudaMemsetAsync(q, 0, kSegQHdrBytes, stream);
+    if (e != cudaSuccess) {
+      cudaFree(q);
+      return cuda_fail(e, "segment queue init");
+    }
+    w->segq = q;
+  }
+  *out = w->segq;
+  return REDUCE_OK;
+}
+
 int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream) {
   LaunchDesc& d = P->d;
   const int combo = combo_index(d.dtype, d.op);
@@ -361,12 +390,16 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   if (opts) {
     if (opts->block != 0 && (opts->block < 32 || opts->block > 512 || opts->block % 32 != 0))
       return fail(REDUCE_ERR_INVALID_ARG, "segmented block must be 0 or a multiple of 32 in [32, 512]");
-    if (opts->seg_group < 0 || opts->seg_group > 3) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0..3");
+    if (opts->seg_group < 0 || opts->seg_group > 4) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0..4");
     if (opts->block) block = opts->block;
     group = opts->seg_group;
   }
-  if (group == 0) group = !uniform ? 1 : (seg_len <= 128 ? 3 : (seg_len <= 4096 ? 1 : 2));
-  const int lanes = group == 1 ? 32 : (group == 3 ? 8 : 0);
+  // auto: by row bytes for uniform batches (B200 sweep, tools/seg_bench.py);
+  // 8 lanes for offset arrays (long segments go to the queue either way)
+  const unsigned long long row_bytes = (unsigned long long)seg_len * (unsigned long long)s;
+  if (group == 0)
+    group = !uniform ? 3 : (row_bytes <= 512 ? 4 : (row_bytes <= 4096 ? 3 : (row_bytes <= 16384 ? 1 : 2)));
+  const int lanes = group == 1 ? 32 : (group == 3 ? 8 : (group == 4 ? 1 : 0));
   SegParams p;
   p.in = (const char*)in;
   p.offsets = (const long long*)offsets;
@@ -374,6 +407,21 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   p.nseg = (long long)nseg;
   p.out = out;
   p.raw_out = 0;
+  // long-segment queue: needed unless no row can be longer than the group's
+  // first round plus its long threshold (uniform rows only)
+  const long long ve = 32 / s;
+  const long long first_round = lanes > 0 ? lanes : block;
+  const long long long_vecs = lanes == 1 ? 32 : lanes == 8 ? 512 : lanes == 32 ? 2048 : 8192;
+  const bool may_long = !uniform || (long long)(seg_len / ve) > first_round + long_vecs - 1;
+  p.use_q = 0;
+  p.q = SegQueue{nullptr, nullptr, nullptr, nullptr};
+  if (may_long) {
+    char* q = nullptr;
+    if (get_seg_queue((cudaStream_t)stream, &q) == REDUCE_OK) {  // else (capture without prepare): no queue
+      p.use_q = 1;
+      p.q = seg_queue_at(q);
+    }
+  }
   cudaError_t e = launch_segmented(dtype, op, p, lanes, block, (cudaStream_t)stream);
   if (e != cudaSuccess) return cuda_fail(e, "segmented reduction launch");
   return REDUCE_OK;
@@ -399,7 +447,7 @@ int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, 
   if (counts == nullptr || ((uintptr_t)counts % 4u) != 0) return fail(REDUCE_ERR_INVALID_ARG, "counts is NULL or misaligned");
   if (n > 0 && (in == nullptr || ((uintptr_t)in % 4u) != 0))
     return fail(REDUCE_ERR_INVALID_ARG, "in is NULL or not aligned to the element size");
-  HistParams p;
+  HistParams p = {};
   p.in = (const char*)in;
   size_t head = 0;
   if (n > 0) {
@@ -418,6 +466,8 @@ int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, 
     p.hi_i = (long long)hi;
     p.range_i = (unsigned long long)(p.hi_i - p.lo_i);
     p.magic = ~0ull / p.range_i;
+    p.narrow = (unsigned long long)p.range_i * (unsigned long long)nbins < (1ull << 32) ? 1 : 0;
+    p.magic32 = p.narrow ? (unsigned)(0xFFFFFFFFull / p.range_i) : 0u;
   } else {
     p.lo_f = (float)lo;
     p.hi_f = (float)hi;
@@ -452,6 +502,9 @@ int reduce_prepare(reduce_stream_t stream, size_t max_n) {
   if (g < 1024) g = 1024;
   Workspace* ws = nullptr;
   int st = get_workspace((cudaStream_t)stream, (size_t)g * 8, &ws);
+  if (st != REDUCE_OK) return st;
+  char* q = nullptr;
+  st = get_seg_queue((cudaStream_t)stream, &q);  // so segmented calls can be captured too
   if (st != REDUCE_OK) return st;
   cudaError_t e = launch_init_workspace(ws->slots, ws->tickets, (cudaStream_t)stream);
   if (e != cudaSuccess) return cuda_fail(e, "workspace init kernel");

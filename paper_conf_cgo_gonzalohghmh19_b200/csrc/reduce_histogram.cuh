@@ -13,11 +13,13 @@
 // operations, floor(fl(fl(x - lo) * scale)) (__fsub_rn / __fmul_rn: never
 // contracted into an FMA).  The B200's FP64 pipe is far too slow for a
 // per-element fp64 rule at HBM speed (measured 2.5 TB/s).  A persistent grid (one wave) streams 32-byte
-// vectors; each block counts into a shared histogram (ATOMS.ADD) and merges
-// its non-zero bins into `counts` with global atomics at the end.  Up to 8 x
-// 16384 bins are split into bin ranges, one range per group of blocks (each
-// group re-reads the input); beyond that, elements count straight into global
-// memory.
+// vectors (two loads in flight per thread); each block counts into a shared
+// histogram (ATOMS.ADD) replicated R times across the banks -- lane l counts
+// into copy l % R, so with R = 32 a warp's 32 updates hit 32 different banks
+// whatever their bins -- and merges its non-zero bins into `counts` with global
+// atomics at the end.  Up to 8 x 16384 bins are split into bin ranges, one range
+// per group of blocks (each group re-reads the input); beyond that, elements
+// count straight into global memory.
 #pragma once
 #include "reduce_kernels.cuh"
 
@@ -25,71 +27,142 @@ namespace rb {
 
 constexpr int kHistSharedMaxBins = 16384;  // 64 KB of u32 counters per block
 
-// Count w into bins[b - b0] if its bin b lies in [b0, b1).
+// Bin of one element, or -1 if it is not counted.  Branch-free (selects and
+// predicated corrections), so the bins of a whole vector are computed with
+// instruction-level parallelism before any counter is touched.
 template <int DT>
-__device__ __forceinline__ void hist_add(uint32_t w, const HistParams& p, unsigned* bins, long long b0, long long b1) {
+__device__ __forceinline__ int hist_bin(uint32_t w, const HistParams& p) {
   if constexpr (DT == DT_I32) {
     const long long v = (long long)(int32_t)w;
-    if (v < p.lo_i || v >= p.hi_i) return;
-    const unsigned long long num = (unsigned long long)(v - p.lo_i) * (unsigned long long)p.nbins;
-    unsigned long long q = __umul64hi(num, p.magic);
-    unsigned long long r = num - q * p.range_i;
-    while (r >= p.range_i) {  // at most two steps: q underestimates by < 2
-      ++q;
-      r -= p.range_i;
+    const bool in = v >= p.lo_i && v < p.hi_i;
+    int b;
+    if (p.narrow) {  // (hi - lo) * nbins < 2^32: the quotient in 32-bit arithmetic
+      const unsigned range = (unsigned)p.range_i;
+      const unsigned num = (unsigned)(v - p.lo_i) * (unsigned)p.nbins;
+      unsigned q = __umulhi(num, p.magic32);
+      unsigned r = num - q * range;
+      // q underestimates floor(num / range) by at most 2
+      if (r >= range) { ++q; r -= range; }
+      if (r >= range) ++q;
+      b = (int)q;
+    } else {
+      const unsigned long long num = (unsigned long long)(v - p.lo_i) * (unsigned long long)p.nbins;
+      unsigned long long q = __umul64hi(num, p.magic);
+      unsigned long long r = num - q * p.range_i;
+      if (r >= p.range_i) { ++q; r -= p.range_i; }
+      if (r >= p.range_i) ++q;
+      b = (int)q;
     }
-    if ((long long)q >= b0 && (long long)q < b1) atomicAdd(bins + (q - b0), 1u);
+    return in ? b : -1;
   } else {
     const float x = __uint_as_float(w);
-    if (!(x >= p.lo_f && x < p.hi_f)) return;  // NaN fails both
+    // x >= lo makes t >= 0, so truncation is floor; t <= nbins * (1 + 2^-22) < 2^31
     const float t = __fmul_rn(__fsub_rn(x, p.lo_f), p.scale_f);
-    const long long b = (long long)floorf(t);
-    if (b >= 0 && b < p.nbins && b >= b0 && b < b1) atomicAdd(bins + (b - b0), 1u);
+    const int b = __float2int_rz(t);
+    return (x >= p.lo_f && x < p.hi_f && b < p.nbins) ? b : -1;  // NaN fails the compares
+  }
+}
+
+// Count the 8 elements of one vector: bins [b0, b1) in shared memory at byte
+// address sbase (this lane's copy; a bin's R copies are adjacent words), or
+// straight into global `counts`.
+template <int DT, bool kShared>
+__device__ __forceinline__ void hist_vec(const uint32_t (&r)[8], const HistParams& p, uint32_t sbase,
+                                         uint32_t sdummy, int rshift, int b0, int b1) {
+  int bin[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) bin[k] = hist_bin<DT>(r[k], p);
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    if constexpr (kShared) {
+      // unconditional: an element that is not counted adds 0 to this lane's
+      // own dummy word (ptxas turns any predicated shared atomic into a
+      // branch-wrapped one -- a reconvergence region per element)
+      const uint32_t ok = bin[k] >= b0 && bin[k] < b1;
+      const uint32_t a = ok ? sbase + ((uint32_t)(bin[k] - b0) << (rshift + 2)) : sdummy;
+      asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(ok) : "memory");
+    } else {
+      if (bin[k] >= 0) atomicAdd(p.counts + bin[k], 1u);
+    }
   }
 }
 
 // kShared: the grid is split into `parts` groups of blocks; group j counts only
-// bins [j*K, (j+1)*K) (K = kHistSharedMaxBins) in shared memory, reading the
-// whole input -- `parts` passes over the data instead of one global atomic per
-// element.  !kShared: every element is one global atomic (very many bins).
+// bins [j*K, (j+1)*K) (K = kHistSharedMaxBins) in shared memory, R = 2^rep_log2
+// copies per bin, reading the whole input -- `parts` passes over the data
+// instead of one global atomic per element.  !kShared: every element is one
+// global atomic (very many bins).
 template <int DT, bool kShared>
-__global__ void __launch_bounds__(512) k_histogram(const HistParams p, int parts) {
+__global__ void __launch_bounds__(256) k_histogram(const HistParams p, int parts, int rep_log2) {
   extern __shared__ unsigned sbins[];
-  long long b0 = 0, b1 = p.nbins;
+  int b0 = 0, b1 = p.nbins;
   unsigned blk = blockIdx.x, nblk = gridDim.x;
-  unsigned* bins = p.counts;
+  uint32_t sbase = 0, sdummy = 0;
   if constexpr (kShared) {
     const unsigned per = gridDim.x / parts;
     const unsigned j = blockIdx.x / per;
     blk = blockIdx.x - j * per;
     nblk = per;
-    b0 = (long long)j * kHistSharedMaxBins;
+    b0 = (int)j * kHistSharedMaxBins;
     b1 = b0 + kHistSharedMaxBins < p.nbins ? b0 + kHistSharedMaxBins : p.nbins;
-    bins = sbins;
-    for (long long i = threadIdx.x; i < b1 - b0; i += blockDim.x) sbins[i] = 0u;
+    const int R = 1 << rep_log2;
+    sbase = (uint32_t)__cvta_generic_to_shared(sbins) + 4u * (threadIdx.x & (R - 1));
+    // 32 dummy words after the bins, one per lane
+    sdummy = (uint32_t)__cvta_generic_to_shared(sbins) + 4u * ((b1 - b0) * R + (threadIdx.x & 31));
+    for (int i = threadIdx.x; i < (b1 - b0) * R; i += blockDim.x) sbins[i] = 0u;
     __syncthreads();
   }
   const unsigned long long stride = (unsigned long long)nblk * blockDim.x;
   unsigned long long v = (unsigned long long)blk * blockDim.x + threadIdx.x;
-  for (; v < p.body_vecs; v += stride) {
+  for (; v + stride < p.body_vecs; v += 2 * stride) {
+    uint32_t r0[8], r1[8];
+    ld_v8(p.body + v * kVecBytes, r0);
+    ld_v8(p.body + (v + stride) * kVecBytes, r1);
+    hist_vec<DT, kShared>(r0, p, sbase, sdummy, rep_log2, b0, b1);
+    hist_vec<DT, kShared>(r1, p, sbase, sdummy, rep_log2, b0, b1);
+  }
+  if (v < p.body_vecs) {
     uint32_t r[8];
     ld_v8(p.body + v * kVecBytes, r);
-#pragma unroll
-    for (int k = 0; k < 8; ++k) hist_add<DT>(r[k], p, bins, b0, b1);
+    hist_vec<DT, kShared>(r, p, sbase, sdummy, rep_log2, b0, b1);
   }
-  if (blk == 0) {
+  if (blk == 0) {  // head and tail elements (< 8 each), as one padded vector
     const int t = threadIdx.x;
-    if (t < p.head) hist_add<DT>(__ldg((const uint32_t*)p.in + t), p, bins, b0, b1);
-    else if (t >= 8 && t - 8 < p.tail)
-      hist_add<DT>(__ldg((const uint32_t*)(p.body + p.body_vecs * kVecBytes) + (t - 8)), p, bins, b0, b1);
+    uint32_t r[8];
+    const bool mine = t < p.head || (t >= 8 && t - 8 < p.tail);
+    r[0] = !mine ? 0u
+           : t < p.head ? __ldg((const uint32_t*)p.in + t)
+                        : __ldg((const uint32_t*)(p.body + p.body_vecs * kVecBytes) + (t - 8));
+    if (mine) {
+      const int bn = hist_bin<DT>(r[0], p);
+      if constexpr (kShared) {
+        if (bn >= b0 && bn < b1)
+          asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(sbase + ((uint32_t)(bn - b0) << (rep_log2 + 2))) : "memory");
+      } else {
+        if (bn >= 0) atomicAdd(p.counts + bn, 1u);
+      }
+    }
   }
   if constexpr (kShared) {
     __syncthreads();
-    for (long long i = threadIdx.x; i < b1 - b0; i += blockDim.x) {
-      const unsigned c = sbins[i];
-      if (c) atomicAdd(p.counts + b0 + i, c);
+    // merge: each warp reads 32 consecutive words (32 / R bins, conflict-free),
+    // sums each bin's R copies with shuffles, one global atomic per non-zero bin
+    const int R = 1 << rep_log2;
+    const int lane = threadIdx.x & 31, words = (b1 - b0) * R;
+    for (int base = (threadIdx.x & ~31); base < words; base += blockDim.x) {
+      const int i = base + lane;
+      unsigned c = i < words ? sbins[i] : 0u;
+      for (int o = R >> 1; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+      if ((lane & (R - 1)) == 0 && i < words && c) atomicAdd(p.counts + b0 + (i >> rep_log2), c);
     }
   }
+}
+
+// Copies per bin: as many as keep a block's bins within 64 KB (<= 32).
+inline int hist_rep_log2(int bins_per_block) {
+  int rl = 5;
+  while (rl > 0 && (long long)bins_per_block * (1 << rl) * 4 > 64 * 1024) --rl;
+  return rl;
 }
 
 template <int DT>
@@ -101,14 +174,19 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
   if (e != cudaSuccess) return e;
   const int parts = (p.nbins + kHistSharedMaxBins - 1) / kHistSharedMaxBins;
   const bool shared = parts <= 8;  // up to 8 passes over the data beat one global atomic per element
-  const int sbins = shared ? (parts == 1 ? p.nbins : kHistSharedMaxBins) : 0;
-  const size_t smem = (size_t)sbins * sizeof(unsigned);
-  // one wave per part group: as many blocks as fit (the shared bins limit residency)
-  int per_sm = 2048 / block;
-  if (smem > 0) {
-    const int by_smem = (int)((200 * 1024) / smem);
-    if (by_smem < per_sm) per_sm = by_smem < 1 ? 1 : by_smem;
+  const int per_block_bins = shared ? (parts == 1 ? p.nbins : kHistSharedMaxBins) : 0;
+  const int rep_log2 = shared ? hist_rep_log2(per_block_bins) : 0;
+  const size_t smem = shared ? ((size_t)per_block_bins * ((size_t)1 << rep_log2) + 32) * sizeof(unsigned) : 0;
+  auto kernel = shared ? k_histogram<DT, true> : k_histogram<DT, false>;
+  if (smem > 48 * 1024) {
+    e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
   }
+  // one wave per part group: as many blocks as fit (the shared bins limit residency)
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, block, smem);
+  if (e != cudaSuccess) return e;
+  if (per_sm < 1) per_sm = 1;
   long long per_part = (long long)sms * per_sm / (shared ? parts : 1);
   const long long need = (long long)((p.body_vecs + block - 1) / block);
   if (need < per_part) per_part = need;
@@ -120,15 +198,7 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
   cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cfg.numAttrs = 0;  // follows a memset node: ordinary stream order
-  if (shared) {
-    if (smem > 48 * 1024) {
-      e = cudaFuncSetAttribute(k_histogram<DT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               kHistSharedMaxBins * (int)sizeof(unsigned));
-      if (e != cudaSuccess) return e;
-    }
-    return cudaLaunchKernelEx(&cfg, k_histogram<DT, true>, p, parts);
-  }
-  return cudaLaunchKernelEx(&cfg, k_histogram<DT, false>, p, 1);
+  return cudaLaunchKernelEx(&cfg, kernel, p, shared ? parts : 1, rep_log2);
 }
 
 }  // namespace rb

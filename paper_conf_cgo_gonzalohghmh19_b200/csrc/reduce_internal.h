@@ -81,7 +81,30 @@ struct LaunchDesc {
   TeamArgs team;                 // team.k > 0: exchange the raw result with the team first
 };
 
-// One segmented / batched launch, see reduce_segmented.cuh.
+// Long-segment queue of a segmented call (lives in the stream's workspace):
+// segments too long for one group are cut into chunks that whole blocks reduce
+// (k_seg_chunks), then their chunk partials are combined in order (k_seg_finish).
+constexpr unsigned kSegQItems = 1u << 18;  // chunk items (and partial slots)
+constexpr unsigned kSegQLongs = 1u << 17;  // long segments (each uses >= 2 items)
+constexpr size_t kSegQHdrBytes = 256;
+constexpr size_t kSegQBytes = kSegQHdrBytes + (size_t)kSegQItems * 16 /* items */ +
+                              (size_t)kSegQItems * 16 /* partials */ + (size_t)kSegQLongs * 24 /* longs */;
+struct SegQueue {
+  unsigned* hdr;       // [0] items reserved, [1] long segments, [2] finish ticket (self-resetting)
+  long long* items;    // [2 * i]: chunk i = elements [lo, hi)
+  void* partials;      // Grid[kSegQItems]: chunk i's value
+  long long* longs;    // [3 * j]: segment, first partial, partial count
+};
+inline SegQueue seg_queue_at(char* base) {
+  SegQueue q;
+  q.hdr = (unsigned*)base;
+  q.items = (long long*)(base + kSegQHdrBytes);
+  q.partials = base + kSegQHdrBytes + (size_t)kSegQItems * 16;
+  q.longs = (long long*)(base + kSegQHdrBytes + (size_t)kSegQItems * 32);
+  return q;
+}
+
+// One segmented / batched call, see reduce_segmented.cuh.
 struct SegParams {
   const char* in;
   const long long* offsets;  // device, nseg + 1 entries; NULL: uniform segments of seg_len
@@ -89,8 +112,10 @@ struct SegParams {
   long long nseg;
   void* out;                 // T[nseg] (finalised) or Grid[nseg] (raw)
   int raw_out;
+  int use_q;                 // 1: offload long segments to q (2 more launches)
+  SegQueue q;
 };
-// group: lanes per segment (8 or 32) or 0 = one block per segment.
+// group: lanes per segment (1, 8 or 32) or 0 = one block per segment.
 cudaError_t launch_segmented(int dtype, int op, const SegParams& p, int group, int block, cudaStream_t s);
 
 // One histogram launch, see reduce_histogram.cuh.
@@ -102,6 +127,8 @@ struct HistParams {
   long long lo_i, hi_i;         // int32 input: integer bounds
   unsigned long long range_i;   //   hi_i - lo_i
   unsigned long long magic;     //   floor((2^64 - 1) / range_i): quotient by multiply-high
+  unsigned magic32;             //   floor((2^32 - 1) / range_i) when narrow
+  int narrow;                   //   range_i * nbins < 2^32: 32-bit quotient
   float lo_f, hi_f, scale_f;    // fp32 input: (float)lo, (float)hi, (float)(nbins / (hi - lo))
   int nbins;
   unsigned* counts;             // device, nbins

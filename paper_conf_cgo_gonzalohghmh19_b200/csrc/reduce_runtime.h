@@ -21,6 +21,7 @@ struct Workspace {
   char* scalars = nullptr;     // 64 x 64-byte scratch scalars (raw results, gathers)
   char* partials = nullptr;    // per-block / per-chunk Grid values
   size_t partials_bytes = 0;
+  char* segq = nullptr;        // long-segment queue of reduce_segmented / reduce_batched (kSegQBytes)
   // reduce_host staging (lazily created)
   char* staging = nullptr;     // 2 x staging_bytes
   size_t staging_bytes = 0;

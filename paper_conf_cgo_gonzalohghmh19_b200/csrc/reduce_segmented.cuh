@@ -1,38 +1,66 @@
-// reduce_segmented.cuh -- many independent reductions in one launch (SURVEY
+// reduce_segmented.cuh -- many independent reductions in one call (SURVEY
 // section 8(f) N1: batched / segmented reduction).
 //
 // Segment i is in[lo_i, hi_i) with lo_i = offsets[i], hi_i = offsets[i+1]
 // (device int64 array of num_segments + 1 entries), or lo_i = i * seg_len for
 // uniform batches (offsets == NULL); out[i] receives its result.  The paper's
 // small-array winners assign one warp or one block per
-// partition with no global atomics; here the group size is chosen from the mean
-// segment length:
-//   kGroup == 32    : one warp per segment (8 segments per 256-thread block),
-//                     warp combine only (redux / shuffles);
-//   kGroup == block : one block per segment, block combine "Vs".
+// partition with no global atomics; here the group size is chosen from the
+// segment length (host side, reduce_api.cpp):
+//   kGroup == 1     : one thread per segment (rows of a few vectors);
+//   kGroup == 8     : 8 lanes per segment (4 segments per warp), shuffles;
+//   kGroup == 32    : one warp per segment, warp combine only (redux / shuffles);
+//   kGroup == 0     : one block per segment, block combine "Vs".
 // Each segment gets its own head / 32-byte-aligned body / tail split, so any
-// element-aligned offset works.  Every step is fixed-order: deterministic.
+// element-aligned offset works.
+//
+// Load balance.  A group reduces the first round of its segment (one vector
+// per lane, plus head and tail); a segment with more than kLongVecs vectors
+// left is not finished by the group: the group's partial goes into the
+// stream's long-segment queue with the rest of the segment cut into chunks of
+// kChunkVecs vectors (k_segmented, leader thread: integer atomics reserve the
+// slots), whole blocks of a persistent grid reduce the chunks (k_seg_chunks),
+// and one warp per long segment combines its partials in chunk order
+// (k_seg_finish, which also resets the queue).  So one huge segment among
+// millions of short ones is spread over the GPU instead of one warp.  Values
+// never touch atomics and every combine is in a fixed order: deterministic.
 #pragma once
 #include "reduce_kernels.cuh"
 
 namespace rb {
 
-// Fold in[lo, hi) by `lanes` cooperating threads (this one is `lid`).
-template <class T, int U>
-__device__ __forceinline__ void fold_range(Part<T> (&a)[T::NA], uint32_t& aux, const char* base,
-                                           long long lo, long long hi, int lid, int lanes) {
-  using Elem = typename T::Elem;
-  constexpr int s = sizeof(Elem);
-  if (hi <= lo) return;
-  const char* p = base + lo * s;
-  const long long n = hi - lo;
-  const unsigned mis = (unsigned)((uintptr_t)p & 31u);
+// A segment in[lo, hi) split into a head (< 32 B, up to the first 32-byte
+// boundary), `nvec` aligned 32-byte vectors and a tail (< 32 B).
+struct SegGeo {
+  const char* p;     // first element
+  const char* body;  // first aligned vector
+  long long nvec;
+  int head, tail;    // elements
+};
+
+template <class T>
+__device__ __forceinline__ SegGeo seg_geo(const char* base, long long lo, long long hi) {
+  constexpr int s = sizeof(typename T::Elem);
+  SegGeo g;
+  const long long n = hi > lo ? hi - lo : 0;
+  g.p = base + lo * s;
+  const unsigned mis = (unsigned)((uintptr_t)g.p & 31u);
   long long head = mis ? (long long)((32u - mis) / s) : 0;
   if (head > n) head = n;
-  const char* body = p + head * s;
-  const long long nvec = (n - head) / T::VE;
-  const long long tail = (n - head) % T::VE;
-  long long v = lid;
+  g.head = (int)head;
+  g.body = g.p + head * s;
+  g.nvec = (n - head) / T::VE;
+  g.tail = (int)((n - head) % T::VE);
+  return g;
+}
+
+// Fold vectors v0, v0 + lanes, ... < nvec of a segment body, U loads in
+// flight, then the remainder one at a time.
+template <class T, int U>
+__device__ __forceinline__ void fold_body(Part<T> (&a)[T::NA], uint32_t& aux, const char* body,
+                                          long long v0, long long nvec, int lanes) {
+  long long v = v0;
+#pragma unroll 1
   for (; v + (long long)(U - 1) * lanes < nvec; v += (long long)U * lanes) {
     uint32_t r[U][8];
 #pragma unroll
@@ -40,15 +68,26 @@ __device__ __forceinline__ void fold_range(Part<T> (&a)[T::NA], uint32_t& aux, c
 #pragma unroll
     for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, r[u], u);
   }
+#pragma unroll 1
   for (; v < nvec; v += lanes) {
     uint32_t r[8];
     ld_v8(body + v * kVecBytes, r);
     fold_vec<T>(a, aux, r, 0);
   }
+}
+
+// Fold in[lo, hi) by `lanes` cooperating threads (this one is `lid`).
+template <class T, int U>
+__device__ __forceinline__ void fold_range(Part<T> (&a)[T::NA], uint32_t& aux, const char* base,
+                                           long long lo, long long hi, int lid, int lanes) {
+  using Elem = typename T::Elem;
+  if (hi <= lo) return;
+  const SegGeo g = seg_geo<T>(base, lo, hi);
+  fold_body<T, U>(a, aux, g.body, lid, g.nvec, lanes);
   // head and tail (< 8 elements each) by the first lanes, into two different
   // accumulators (groups may be only 8 lanes wide)
-  if (lid < head) fold_elem<T>(a[0], aux, __ldg((const Elem*)p + lid));
-  if (lid < tail) fold_elem<T>(a[T::NA - 1], aux, __ldg((const Elem*)(body + nvec * kVecBytes) + lid));
+  if (lid < g.head) fold_elem<T>(a[0], aux, __ldg((const Elem*)g.p + lid));
+  if (lid < g.tail) fold_elem<T>(a[T::NA - 1], aux, __ldg((const Elem*)(g.body + g.nvec * kVecBytes) + lid));
 }
 
 template <class T>
@@ -57,81 +96,289 @@ __device__ __forceinline__ void seg_store(const SegParams& p, long long seg, typ
   else T::finalize(g, (char*)p.out + seg * (long long)sizeof(typename T::Elem));
 }
 
-// kGroup = 8 or 32: that many lanes per segment (4 or 1 segments per warp in
-// flight); kGroup = 0: one block per segment.  The grid is persistent (a few
-// blocks per SM) and groups stride over the segments, so millions of tiny
-// segments do not pay one CTA launch each.
+template <class T>
+__device__ __forceinline__ void seg_bounds(const SegParams& p, long long seg, long long& lo, long long& hi) {
+  lo = hi = 0;
+  if (seg < p.nseg) {
+    if (p.offsets) {
+      lo = __ldg(p.offsets + seg);
+      hi = __ldg(p.offsets + seg + 1);
+    } else {
+      lo = seg * p.seg_len;
+      hi = lo + p.seg_len;
+    }
+  }
+}
+
+// Segments a small group keeps in flight: the first-round loads of kSegPipe
+// segments are issued before any of them is folded (B200 A/B, tools/seg_bench.py:
+// 2 beats 1 on short rows; 4 needs 128 registers and loses).
+#ifndef RB_SEG_PIPE
+#define RB_SEG_PIPE 2
+#endif
+constexpr int kSegPipe = RB_SEG_PIPE;
+
+// Vectors left after a group's first round above which a segment goes to the
+// long-segment queue.
+template <int kGroup>
+__host__ __device__ constexpr long long seg_long_vecs() {
+  return kGroup == 1 ? 32 : kGroup == 8 ? 512 : kGroup == 32 ? 2048 : 8192;
+}
+// Chunks of a queued segment: at least kChunkMinVecs vectors (16 KB, four
+// rounds of four loads for the warp that reduces one), at most kMaxChunks per
+// segment (one huge segment still spreads over thousands of warps).
+constexpr long long kChunkMinVecs = 512;
+constexpr long long kMaxChunks = 4096;
+constexpr unsigned kNoSlot = 0xFFFFFFFFu;
+
+// Leader of a group: reserve queue slots for the rest of segment `seg` --
+// elements [rem_lo, rem_hi), 32-byte aligned at both ends -- and write its
+// chunk items.  Slot `base` is left for the group's own partial (written
+// after the group combine), chunks take base+1 .. base+k.  Returns kNoSlot if
+// the queue is full: the group then finishes the segment itself.
+__device__ __forceinline__ unsigned seg_reserve(unsigned* hdr, long long* items, long long* longs, long long seg,
+                                             long long rem_lo, long long rem_hi, int ve) {
+  const long long nv = (rem_hi - rem_lo) / ve;
+  long long per_v = (nv + kMaxChunks - 1) / kMaxChunks;
+  if (per_v < kChunkMinVecs) per_v = kChunkMinVecs;
+  const long long per = per_v * ve;
+  const long long k = (nv + per_v - 1) / per_v;
+  const unsigned need = (unsigned)(k + 1);
+  const unsigned base = atomicAdd(hdr + 0, need);
+  if ((unsigned long long)base + need > kSegQItems) {
+    // reserved past the end: leave the reachable part of the range empty
+    for (unsigned long long i = base; i < kSegQItems; ++i) {
+      items[2 * i] = 0;
+      items[2 * i + 1] = 0;
+    }
+    return kNoSlot;
+  }
+  items[2 * (size_t)base] = 0;  // the group's partial: an empty item
+  items[2 * (size_t)base + 1] = 0;
+  for (long long c = 0; c < k; ++c) {
+    const long long lo = rem_lo + c * per;
+    items[2 * (base + 1 + c)] = lo;
+    items[2 * (base + 1 + c) + 1] = lo + per < rem_hi ? lo + per : rem_hi;
+  }
+  const unsigned j = atomicAdd(hdr + 1, 1u);  // < kSegQLongs: every long segment holds >= 2 items
+  longs[3 * (size_t)j] = seg;
+  longs[3 * (size_t)j + 1] = base;
+  longs[3 * (size_t)j + 2] = k + 1;
+  return base;
+}
+
+// kGroup = 1, 8 or 32 lanes per segment (32 / kGroup segments per warp at a
+// time, kSegPipe of them in flight); kGroup = 0: one block per segment.  The
+// grid is persistent (one wave) and groups stride over the segments, so
+// millions of tiny segments do not pay one CTA launch each.
 template <int DT, int OP, int kGroup>
 __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
+  using Elem = typename T::Elem;
+  using Grid = typename T::Grid;
+  constexpr long long kLong = seg_long_vecs<kGroup>();
   pdl_wait();
   const int lane = threadIdx.x & 31;
-  long long first, step;
-  int lid, lanes;
   if constexpr (kGroup > 0) {
     const long long groups_per_block = blockDim.x / kGroup;
-    first = (long long)blockIdx.x * groups_per_block + threadIdx.x / kGroup;
-    step = (long long)gridDim.x * groups_per_block;
-    lid = threadIdx.x % kGroup;
-    lanes = kGroup;
-  } else {
-    first = blockIdx.x;
-    step = gridDim.x;
-    lid = threadIdx.x;
-    lanes = blockDim.x;
-  }
-  // all groups of a warp (all threads of a block) run the same number of
-  // iterations -- the shuffles / barriers need every lane -- and a group past
-  // the last segment folds nothing
-  const long long base = kGroup > 0 ? first - lane / kGroup : first;
-  const long long iters = base < p.nseg ? (p.nseg - base + step - 1) / step : 0;
+    const long long first = (long long)blockIdx.x * groups_per_block + threadIdx.x / kGroup;
+    const long long step = (long long)gridDim.x * groups_per_block;
+    const int lid = threadIdx.x % kGroup;
+    const int leader = lane - lid;
+    // all groups of a warp run the same number of rounds (the shuffles need
+    // every lane); a group past the last segment folds nothing
+    const long long wbase = first - lane / kGroup;
+    const long long count = wbase < p.nseg ? (p.nseg - wbase + step - 1) / step : 0;
 #pragma unroll 1
-  for (long long it = 0; it < iters; ++it) {
-    const long long seg = first + it * step;
-    const bool live = seg < p.nseg;
-    long long lo = 0, hi = 0;
-    if (live) {
-      if (p.offsets) {
-        lo = __ldg(p.offsets + seg);
-        hi = __ldg(p.offsets + seg + 1);
-      } else {
-        lo = seg * p.seg_len;
-        hi = lo + p.seg_len;
+    for (long long k0 = 0; k0 < count; k0 += kSegPipe) {
+      // phase 1: the first round of every segment -- one vector, one head and
+      // one tail element per lane -- with all kSegPipe segments' loads issued
+      // before any is folded
+      uint32_t r[kSegPipe][8];
+      Elem hv[kSegPipe], tv[kSegPipe];
+      bool hasv[kSegPipe], hash[kSegPipe], hast[kSegPipe], more = false;
+      unsigned slot[kSegPipe];
+#pragma unroll
+      for (int j = 0; j < kSegPipe; ++j) {
+        long long lo, hi;
+        seg_bounds<T>(p, first + (k0 + j) * step, lo, hi);
+        const SegGeo g = seg_geo<T>(p.in, lo, hi);
+        hasv[j] = lid < g.nvec;
+        hash[j] = lid < g.head;
+        hast[j] = lid < g.tail;
+        more |= g.nvec > kGroup || (kGroup < 8 && (g.head > kGroup || g.tail > kGroup));
+        if (hasv[j]) ld_v8(g.body + (long long)lid * kVecBytes, r[j]);
+        if (hash[j]) hv[j] = __ldg((const Elem*)g.p + lid);
+        if (hast[j]) tv[j] = __ldg((const Elem*)(g.body + g.nvec * kVecBytes) + lid);
+        // a long segment: the leader queues the rest of it (every lane of the
+        // warp takes part in the broadcast)
+        slot[j] = kNoSlot;
+        if (p.use_q && lid == 0 && g.nvec - kGroup > kLong)
+          slot[j] = seg_reserve(p.q.hdr, p.q.items, p.q.longs, first + (k0 + j) * step,
+                                lo + g.head + (long long)kGroup * T::VE, lo + g.head + g.nvec * T::VE, T::VE);
+        if constexpr (kGroup > 1) slot[j] = __shfl_sync(0xffffffffu, slot[j], leader);
+      }
+      Acc v[kSegPipe];
+#pragma unroll
+      for (int j = 0; j < kSegPipe; ++j) {
+        Part<T> a[T::NA];
+        init_parts<T>(a);
+        uint32_t aux = 0;
+        if (hasv[j]) fold_vec<T>(a, aux, r[j], 1);
+        if (hash[j]) fold_elem<T>(a[0], aux, hv[j]);
+        if (hast[j]) fold_elem<T>(a[T::NA - 1], aux, tv[j]);
+        v[j] = thread_result<T>(a, aux);
+      }
+      // phase 2 (the rest of segments longer than one round that were not
+      // queued; for groups narrower than 8 lanes also the head / tail elements
+      // past the first): one code copy for all j, geometry recomputed
+      if (more) {
+#pragma unroll 1
+        for (int j = 0; j < kSegPipe; ++j) {
+          long long lo, hi;
+          seg_bounds<T>(p, first + (k0 + j) * step, lo, hi);
+          const SegGeo g = seg_geo<T>(p.in, lo, hi);
+          unsigned sj = kNoSlot;
+#pragma unroll
+          for (int q = 0; q < kSegPipe; ++q)
+            if (q == j) sj = slot[q];
+          Part<T> a[T::NA];
+          init_parts<T>(a);
+          uint32_t aux = 0;
+          bool any = false;
+          if (g.nvec > kGroup && sj == kNoSlot) {
+            fold_body<T, 4>(a, aux, g.body, lid + kGroup, g.nvec, kGroup);
+            any = true;
+          }
+          if constexpr (kGroup < 8) {
+            for (int h = lid + kGroup; h < g.head; h += kGroup) fold_elem<T>(a[0], aux, __ldg((const Elem*)g.p + h));
+            for (int t = lid + kGroup; t < g.tail; t += kGroup)
+              fold_elem<T>(a[T::NA - 1], aux, __ldg((const Elem*)(g.body + g.nvec * kVecBytes) + t));
+            any |= g.head > kGroup || g.tail > kGroup;
+          }
+          if (any) {
+            const Acc e = thread_result<T>(a, aux);
+#pragma unroll
+            for (int q = 0; q < kSegPipe; ++q)
+              if (q == j) v[q] = T::comb(v[q], e);
+          }
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < kSegPipe; ++j) {
+        const long long seg = first + (k0 + j) * step;
+        Acc w = v[j];
+        if constexpr (kGroup == 32) {
+          w = T::warp(w);
+        } else {
+#pragma unroll
+          for (int o = kGroup / 2; o > 0; o >>= 1) w = T::comb(w, shfl_xor(w, o));
+        }
+        if (lid == 0 && seg < p.nseg) {
+          if (slot[j] != kNoSlot) ((Grid*)p.q.partials)[slot[j]] = T::to_grid(w);  // k_seg_finish writes out[seg]
+          else seg_store<T>(p, seg, T::to_grid(w));
+        }
       }
     }
-    Part<T> a[T::NA];
-    init_parts<T>(a);
-    uint32_t aux = 0;
-    fold_range<T, 4>(a, aux, p.in, lo, hi, lid, lanes);
-    const Acc v = thread_result<T>(a, aux);
-    if constexpr (kGroup == 32) {
-      const Acc w = T::warp(v);
-      if (lane == 0 && live) seg_store<T>(p, seg, T::to_grid(w));
-    } else if constexpr (kGroup > 0) {
-      Acc w = v;
-#pragma unroll
-      for (int o = kGroup / 2; o > 0; o >>= 1) w = T::comb(w, shfl_xor(w, o));
-      if (lid == 0 && live) seg_store<T>(p, seg, T::to_grid(w));
-    } else {
-      const typename T::Grid g = block_combine<T, BC_SHFL>(v);
-      if (threadIdx.x == 0 && live) seg_store<T>(p, seg, g);
-      __syncthreads();  // block_combine's shared scratch is reused next iteration
+  } else {
+    __shared__ unsigned s_slot;
+#pragma unroll 1
+    for (long long seg = blockIdx.x; seg < p.nseg; seg += gridDim.x) {
+      long long lo, hi;
+      seg_bounds<T>(p, seg, lo, hi);
+      const SegGeo g = seg_geo<T>(p.in, lo, hi);
+      if (threadIdx.x == 0) {
+        s_slot = kNoSlot;
+        if (p.use_q && g.nvec - (long long)blockDim.x > kLong)
+          s_slot = seg_reserve(p.q.hdr, p.q.items, p.q.longs, seg, lo + g.head + (long long)blockDim.x * T::VE,
+                               lo + g.head + g.nvec * T::VE, T::VE);
+      }
+      __syncthreads();
+      const unsigned sl = s_slot;
+      Part<T> a[T::NA];
+      init_parts<T>(a);
+      uint32_t aux = 0;
+      // a queued segment: only the first round here
+      fold_body<T, 4>(a, aux, g.body, threadIdx.x, sl != kNoSlot ? (long long)blockDim.x : g.nvec, blockDim.x);
+      if ((int)threadIdx.x < g.head) fold_elem<T>(a[0], aux, __ldg((const Elem*)g.p + threadIdx.x));
+      if ((int)threadIdx.x < g.tail)
+        fold_elem<T>(a[T::NA - 1], aux, __ldg((const Elem*)(g.body + g.nvec * kVecBytes) + threadIdx.x));
+      const Grid gv = block_combine<T, BC_SHFL>(thread_result<T>(a, aux));
+      if (threadIdx.x == 0) {
+        if (sl != kNoSlot) ((Grid*)p.q.partials)[sl] = gv;
+        else seg_store<T>(p, seg, gv);
+      }
+      __syncthreads();  // block_combine's shared scratch and s_slot are reused next iteration
     }
   }
   pdl_trigger();  // persistent grid: let the next kernel in only as this one finishes
 }
 
+// Queued chunks -> partials, one warp per chunk (persistent grid).
 template <int DT, int OP>
-cudaError_t launch_segmented_op(const SegParams& p, int group, int block, cudaStream_t s) {
-  int dev = 0, sms = 148;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const long long per_block = group > 0 ? block / group : 1;
-  long long grid = (p.nseg + per_block - 1) / per_block;
-  const long long cap = (long long)sms * (2048 / block);  // one full wave
-  if (grid > cap) grid = cap;
-  if (grid < 1) grid = 1;
+__global__ void __launch_bounds__(256) k_seg_chunks(const SegParams p) {
+  using T = Tr<DT, OP>;
+  pdl_wait();
+  unsigned n = *(volatile unsigned*)(p.q.hdr + 0);
+  if (n > kSegQItems) n = kSegQItems;
+  const int lane = threadIdx.x & 31;
+  const unsigned warps = gridDim.x * (blockDim.x >> 5);
+#pragma unroll 1
+  for (unsigned i = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n; i += warps) {
+    const long long lo = p.q.items[2 * (size_t)i], hi = p.q.items[2 * (size_t)i + 1];
+    if (hi <= lo) continue;  // a group partial's slot, or left empty (warp-uniform)
+    Part<T> a[T::NA];
+    init_parts<T>(a);
+    uint32_t aux = 0;
+    fold_range<T, 4>(a, aux, p.in, lo, hi, lane, 32);
+    const typename T::Acc w = T::warp(thread_result<T>(a, aux));
+    if (lane == 0) ((typename T::Grid*)p.q.partials)[i] = T::to_grid(w);
+  }
+  pdl_trigger();
+}
+
+// One warp per queued segment: its partials in order (the group's first round,
+// then the chunks) -> out[seg]; the last block resets the queue for the next
+// call on this stream.
+template <int DT, int OP>
+__global__ void __launch_bounds__(256) k_seg_finish(const SegParams p) {
+  using T = Tr<DT, OP>;
+  using Grid = typename T::Grid;
+  pdl_wait();
+  unsigned nl = *(volatile unsigned*)(p.q.hdr + 1);
+  if (nl > kSegQLongs) nl = kSegQLongs;
+  const int lane = threadIdx.x & 31;
+  const unsigned warps = gridDim.x * (blockDim.x >> 5);
+#pragma unroll 1
+  for (unsigned j = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); j < nl; j += warps) {
+    const long long seg = p.q.longs[3 * (size_t)j], base = p.q.longs[3 * (size_t)j + 1];
+    const long long cnt = p.q.longs[3 * (size_t)j + 2];
+    Grid x = T::gident();
+    for (long long i = lane; i < cnt; i += 32) x = T::gcomb(x, __ldcg((const Grid*)p.q.partials + base + i));
+    x = T::gwarp(x);
+    if (lane == 0) seg_store<T>(p, seg, x);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0 && ticket_acq_rel(p.q.hdr + 2) == gridDim.x - 1) {
+    p.q.hdr[0] = 0u;
+    p.q.hdr[1] = 0u;
+    p.q.hdr[2] = 0u;
+  }
+  pdl_trigger();
+}
+
+// Resident blocks per SM of a kernel at a block size (persistent grids are one
+// full wave of them).
+template <class K>
+int seg_blocks_per_sm(K kernel, int block) {
+  int nb = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, block, 0) != cudaSuccess || nb < 1) nb = 1;
+  return nb;
+}
+
+template <class K>
+cudaError_t seg_launch(K kernel, long long grid, int block, const SegParams& p, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid, 1, 1);
   cfg.blockDim = dim3(block, 1, 1);
@@ -141,9 +388,38 @@ cudaError_t launch_segmented_op(const SegParams& p, int group, int block, cudaSt
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = pdl_enabled() ? 1 : 0;
-  if (group == 8) return cudaLaunchKernelEx(&cfg, k_segmented<DT, OP, 8>, p);
-  if (group == 32) return cudaLaunchKernelEx(&cfg, k_segmented<DT, OP, 32>, p);
-  return cudaLaunchKernelEx(&cfg, k_segmented<DT, OP, 0>, p);
+  return cudaLaunchKernelEx(&cfg, kernel, p);
+}
+
+template <int DT, int OP, int kGroup>
+cudaError_t launch_segmented_group(const SegParams& p, int block, int sms, cudaStream_t s) {
+  static int per_sm[17] = {0};  // resident blocks by block / 32 (cached)
+  const int key = block / 32;
+  if (per_sm[key] == 0) per_sm[key] = seg_blocks_per_sm(k_segmented<DT, OP, kGroup>, block);
+  const long long per_block = kGroup > 0 ? block / kGroup : 1;
+  long long grid = (p.nseg + per_block - 1) / per_block;
+  const long long cap = (long long)sms * per_sm[key];  // one full wave
+  if (grid > cap) grid = cap;
+  if (grid < 1) grid = 1;
+  return seg_launch(k_segmented<DT, OP, kGroup>, grid, block, p, s);
+}
+
+template <int DT, int OP>
+cudaError_t launch_segmented_op(const SegParams& p, int group, int block, cudaStream_t s) {
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaError_t e;
+  if (group == 1) e = launch_segmented_group<DT, OP, 1>(p, block, sms, s);
+  else if (group == 8) e = launch_segmented_group<DT, OP, 8>(p, block, sms, s);
+  else if (group == 32) e = launch_segmented_group<DT, OP, 32>(p, block, sms, s);
+  else e = launch_segmented_group<DT, OP, 0>(p, block, sms, s);
+  if (e != cudaSuccess || !p.use_q) return e;
+  static int chunk_per_sm = 0;
+  if (chunk_per_sm == 0) chunk_per_sm = seg_blocks_per_sm(k_seg_chunks<DT, OP>, 256);
+  e = seg_launch(k_seg_chunks<DT, OP>, (long long)sms * chunk_per_sm, 256, p, s);
+  if (e != cudaSuccess) return e;
+  return seg_launch(k_seg_finish<DT, OP>, sms, 256, p, s);
 }
 
 template <int DT>

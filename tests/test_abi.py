@@ -133,7 +133,7 @@ def test_query_plan_staging():
 
 def test_segmented_argument_validation():
     L = rb.lib
-    o = rb.make_opts(seg_group=4)
+    o = rb.make_opts(seg_group=5)
     assert L.reduce_segmented(1, 0, 4096, None, 10, 8192, None, None) == 1        # offsets NULL
     assert L.reduce_segmented(1, 0, 4096, 4096, 10, None, None, None) == 1        # out NULL
     assert L.reduce_segmented(5, 0, 4096, 4096, 10, 8192, None, None) == 1        # dtype

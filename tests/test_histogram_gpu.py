@@ -44,3 +44,36 @@ def test_histogram_special_values_and_big():
         want = oracle.histogram(x, 0.0, 1.0, nbins)
         assert (got == want).all()
         assert int(got.sum()) == int(((x >= 0) & (x < 1)).sum())
+
+
+@pytest.mark.parametrize("lo,hi,nbins", [
+    (-2.0 ** 31, 2.0 ** 31, 1000),        # range * nbins >= 2^32: 64-bit quotient path
+    (-2.0 ** 32, 2.0 ** 32, 1 << 20),     # widest accepted range, many bins (bin-range passes)
+    (-65536.0, 65537.0, 65535),           # range * nbins just above 2^32
+    (-65536.0, 0.0, 65535),               # range * nbins just below 2^32: 32-bit path
+    (0.0, 3.0, 3),                        # one bin per value
+])
+def test_histogram_int32_wide_ranges(lo, hi, nbins):
+    rb = _rb()
+    x = synth.make("int32", (1 << 20) + 11, "int_full", 77)
+    x[:6] = [np.iinfo(np.int32).min, np.iinfo(np.int32).max, 0, -1, 1, 2]
+    if hi - lo < 2 ** 20:
+        x[7::3] = (x[7::3] % int(2 * (hi - lo))) + int(lo) - int((hi - lo) // 2)
+    t = to_device(x, 5)
+    got = rb.histogram(t, lo, hi, nbins).cpu().numpy().view(np.uint32)
+    want = oracle.histogram(x, lo, hi, nbins)
+    assert (got == want).all(), np.nonzero(got != want)[0][:5]
+
+
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+def test_histogram_replication_boundaries(dtype):
+    """bins per block at the shared-copy boundaries (32, 16, ... copies per bin)"""
+    rb = _rb()
+    n = (1 << 19) + 5
+    x = synth.make(dtype, n, "int_small" if dtype == "int32" else "uniform01", 91)
+    lo, hi = (-1000.0, 1001.0) if dtype == "int32" else (0.0, 1.0)
+    for nbins in (2, 31, 32, 33, 511, 512, 513, 1023, 1024, 2048, 4095, 4096, 8192, 16383):
+        t = to_device(x, nbins % 8)
+        got = rb.histogram(t, lo, hi, nbins).cpu().numpy().view(np.uint32)
+        want = oracle.histogram(x, lo, hi, nbins)
+        assert (got == want).all(), (nbins, np.nonzero(got != want)[0][:5])

@@ -9,7 +9,7 @@ import pytest
 
 import oracle
 import synth
-from tests._util import NP, BITS
+from tests._util import NP, BITS, to_device
 
 pytestmark = pytest.mark.gpu
 DTYPES = ["int32", "float32", "float64"]
@@ -51,7 +51,7 @@ def _segments(rng, nseg, max_len, skew=False):
 
 
 @pytest.mark.parametrize("dtype", DTYPES)
-@pytest.mark.parametrize("group", [0, 1, 2, 3])
+@pytest.mark.parametrize("group", [0, 1, 2, 3, 4])
 @pytest.mark.parametrize("skew", [False, True])
 def test_segmented_matches_oracle_per_segment(dtype, group, skew):
     import torch
@@ -63,7 +63,7 @@ def test_segmented_matches_oracle_per_segment(dtype, group, skew):
     xt = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     ot = torch.from_numpy(offs).cuda()
     bounds = list(zip(offs[:-1].tolist(), offs[1:].tolist()))
-    lanes = {0: 32, 1: 32, 2: 256, 3: 8}[group]
+    lanes = {0: 8, 1: 32, 2: 256, 3: 8, 4: 1}[group]
     for op in OPS:
         got = rb.reduce_segmented(xt, ot, op, seg_group=group).cpu().numpy()
         _check_segments(x, bounds, op, got, lanes)
@@ -78,9 +78,11 @@ def test_batched_rows(dtype, rows, cols):
     x = synth.make(dtype, rows * cols, "int_full" if dtype == "int32" else "uniform01", rows + cols)
     xt = torch.from_numpy(x).cuda().view(rows, cols)
     bounds = [(r * cols, (r + 1) * cols) for r in range(rows)]
-    for group in (0, 1, 2, 3):
-        auto = 8 if cols <= 128 else (32 if cols <= 4096 else 256)
-        lanes = {0: auto, 1: 32, 2: 256, 3: 8}[group]
+    s = x.dtype.itemsize
+    for group in (0, 1, 2, 3, 4):
+        rb_ = cols * s
+        auto = 1 if rb_ <= 512 else (8 if rb_ <= 4096 else (32 if rb_ <= 16384 else 256))
+        lanes = {0: auto, 1: 32, 2: 256, 3: 8, 4: 1}[group]
         for op in OPS:
             got = rb.reduce_batched(xt, op, seg_group=group).cpu().numpy()
             _check_segments(x, bounds, op, got, lanes)
@@ -102,3 +104,99 @@ def test_segmented_special_values_and_determinism():
             _check_segments(x, bounds, op, got, {1: 32, 2: 256, 3: 8}[group])
     outs = {rb.reduce_segmented(xt, ot, "sum").cpu().numpy().tobytes() for _ in range(20)}
     assert len(outs) == 1
+
+
+def _skewed(rng, nseg, huge):
+    """many short segments (0..40 elements) with a few huge ones (up to `huge`
+    elements) at seeded positions: the long-segment queue's workload"""
+    lens = rng.integers(0, 41, nseg)
+    pos = rng.choice(nseg, 6, replace=False)
+    lens[pos] = [huge, huge // 3, 70000, 16385, 4099, 300]
+    offs = np.zeros(nseg + 1, np.int64)
+    offs[1:] = np.cumsum(lens)
+    return offs
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("group", [0, 1, 2, 3, 4])
+def test_segmented_long_segments_load_balanced(dtype, group):
+    """segments far longer than a group's first round go through the chunk
+    queue (k_seg_chunks / k_seg_finish); results per segment vs the oracle,
+    and bitwise identical over repeated calls (fixed chunk order)"""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    rng = np.random.Generator(np.random.PCG64(101 + group))
+    offs = _skewed(rng, 20000, 3_000_001)
+    total = int(offs[-1])
+    x = synth.make(dtype, total + 5, "int_full" if dtype == "int32" else "uniform_pm1", 12)[5:]
+    xt = to_device(x, 3)
+    ot = torch.from_numpy(offs).cuda()
+    bounds = list(zip(offs[:-1].tolist(), offs[1:].tolist()))
+    lanes = {0: 8, 1: 32, 2: 256, 3: 8, 4: 1}[group]
+    for op in OPS + (["sum_accurate"] if dtype != "int32" else []):
+        got = rb.reduce_segmented(xt, ot, op, seg_group=group)
+        if op == "sum_accurate":
+            g = got.cpu().numpy()
+            for i in np.nonzero(np.diff(offs) > 1000)[0]:
+                lo, hi = bounds[i]
+                exact = math.fsum(x[lo:hi].astype(np.float64))
+                a = float(np.abs(x[lo:hi].astype(np.float64)).sum())
+                assert abs(float(g[i]) - exact) <= 2.0 ** -23 * abs(exact) + 1e-9 * a, (i, g[i], exact)
+            continue
+        _check_segments(x, bounds, op, got.cpu().numpy(), lanes)
+        again = rb.reduce_segmented(xt, ot, op, seg_group=group)
+        assert got.cpu().numpy().tobytes() == again.cpu().numpy().tobytes()
+
+
+def test_segmented_queue_overflow_falls_back():
+    """more queued chunks than the queue holds (kSegQItems = 2^18): the
+    segments that do not fit are finished by their own group, results exact"""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    nseg = 150000
+    lens = np.full(nseg, 8 * 40, np.int64)  # 40 vectors: queued by 1-lane groups (2 items each)
+    lens[::1000] = 70000                     # a few multi-chunk ones
+    offs = np.zeros(nseg + 1, np.int64)
+    offs[1:] = np.cumsum(lens)
+    x = synth.make("int32", int(offs[-1]), "int_full", 13)
+    xt, ot = torch.from_numpy(x).cuda(), torch.from_numpy(offs).cuda()
+    got = rb.reduce_segmented(xt, ot, "sum", seg_group=4).cpu().numpy()
+    want = np.add.reduceat(x.astype(np.int64), offs[:-1]).astype(np.int64)
+    want = ((want + 2 ** 31) % 2 ** 32 - 2 ** 31).astype(np.int32)
+    assert (got == want).all(), np.nonzero(got != want)[0][:5]
+    gmax = rb.reduce_segmented(xt, ot, "max", seg_group=4).cpu().numpy()
+    assert (gmax == np.maximum.reduceat(x, offs[:-1])).all()
+
+
+def test_batched_long_rows_chunked():
+    """a few rows of millions of elements: every row is cut into chunks"""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    rows, cols = 3, 5_000_003
+    x = synth.make("float64", rows * cols, "intvalued", 14)
+    xt = torch.from_numpy(x).cuda().view(rows, cols)
+    for group in (0, 1, 2, 3, 4):
+        got = rb.reduce_batched(xt, "sum", seg_group=group).cpu().numpy()
+        want = x.reshape(rows, cols).astype(np.float64).sum(axis=1)  # integer-valued: exact in any order
+        assert (got == want).all(), (group, got, want)
+
+
+def test_segmented_graph_capture_with_queue():
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    rng = np.random.Generator(np.random.PCG64(5))
+    offs = _skewed(rng, 5000, 1_000_000)
+    x = synth.make("float32", int(offs[-1]), "uniform01", 15)
+    xt, ot = torch.from_numpy(x).cuda(), torch.from_numpy(offs).cuda()
+    ref = rb.reduce_segmented(xt, ot, "sum").cpu().numpy()
+    s = torch.cuda.Stream()
+    rb.prepare(s, 1 << 20)
+    out = torch.empty(len(offs) - 1, dtype=torch.float32, device="cuda")
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        rb.reduce_segmented(xt, ot, "sum", out=out, stream=s)
+    for _ in range(4):
+        out.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert out.cpu().numpy().tobytes() == ref.tobytes()
