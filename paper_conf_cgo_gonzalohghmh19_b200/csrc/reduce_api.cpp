@@ -413,6 +413,11 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   const long long first_round = lanes > 0 ? lanes : block;
   const long long long_vecs = lanes == 1 ? 32 : lanes == 8 ? 512 : lanes == 32 ? 2048 : 8192;
   const bool may_long = !uniform || (long long)(seg_len / ve) > first_round + long_vecs - 1;
+  // predicated tail round (B200 A/B, tools/probes/seg_tail_ab.sh): accurate
+  // sums and 2-8 KB fp rows with sub-block groups; never for one block per row
+  p.tail = lanes == 0 ? 0
+           : op == REDUCE_SUM_ACCURATE ? 1
+           : (uniform && dtype != REDUCE_INT32 && row_bytes >= 2048 && row_bytes <= 8192) ? 1 : 0;
   p.use_q = 0;
   p.q = SegQueue{nullptr, nullptr, nullptr, nullptr};
   if (may_long) {

@@ -113,6 +113,7 @@ struct SegParams {
   void* out;                 // T[nseg] (finalised) or Grid[nseg] (raw)
   int raw_out;
   int use_q;                 // 1: offload long segments to q (2 more launches)
+  int tail;                  // 1: fold a segment's last vectors in one predicated round
   SegQueue q;
 };
 // group: lanes per segment (1, 8 or 32) or 0 = one block per segment.

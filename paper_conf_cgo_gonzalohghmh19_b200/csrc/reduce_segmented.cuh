@@ -54,9 +54,12 @@ __device__ __forceinline__ SegGeo seg_geo(const char* base, long long lo, long l
   return g;
 }
 
-// Fold vectors v0, v0 + lanes, ... < nvec of a segment body, U loads in
-// flight, then the remainder one at a time.
-template <class T, int U>
+// Fold vectors v0, v0 + lanes, ... < nvec of a segment body: full rounds of U
+// loads in flight, then the last (< U) vectors either in one predicated round
+// (kTail: more loads in flight, more registers) or one at a time.  B200
+// (tools/probes/seg_tail_ab.sh): the predicated round wins for rows >= 2 KB
+// and for accurate sums, one at a time (64 registers) for short rows.
+template <class T, int U, bool kTail = false>
 __device__ __forceinline__ void fold_body(Part<T> (&a)[T::NA], uint32_t& aux, const char* body,
                                           long long v0, long long nvec, int lanes) {
   long long v = v0;
@@ -68,11 +71,23 @@ __device__ __forceinline__ void fold_body(Part<T> (&a)[T::NA], uint32_t& aux, co
 #pragma unroll
     for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, r[u], u);
   }
+  if constexpr (kTail) {
+    if (v < nvec) {
+      uint32_t r[U - 1][8];
+#pragma unroll
+      for (int u = 0; u < U - 1; ++u)
+        if (v + (long long)u * lanes < nvec) ld_v8(body + (v + (long long)u * lanes) * kVecBytes, r[u]);
+#pragma unroll
+      for (int u = 0; u < U - 1; ++u)
+        if (v + (long long)u * lanes < nvec) fold_vec<T>(a, aux, r[u], u);
+    }
+  } else {
 #pragma unroll 1
-  for (; v < nvec; v += lanes) {
-    uint32_t r[8];
-    ld_v8(body + v * kVecBytes, r);
-    fold_vec<T>(a, aux, r, 0);
+    for (; v < nvec; v += lanes) {
+      uint32_t r[8];
+      ld_v8(body + v * kVecBytes, r);
+      fold_vec<T>(a, aux, r, 0);
+    }
   }
 }
 
@@ -171,7 +186,7 @@ __device__ __forceinline__ unsigned seg_reserve(unsigned* hdr, long long* items,
 // time, kSegPipe of them in flight); kGroup = 0: one block per segment.  The
 // grid is persistent (one wave) and groups stride over the segments, so
 // millions of tiny segments do not pay one CTA launch each.
-template <int DT, int OP, int kGroup>
+template <int DT, int OP, int kGroup, bool kTail>
 __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
@@ -248,7 +263,7 @@ __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
           uint32_t aux = 0;
           bool any = false;
           if (g.nvec > kGroup && sj == kNoSlot) {
-            fold_body<T, 4>(a, aux, g.body, lid + kGroup, g.nvec, kGroup);
+            fold_body<T, 4, kTail>(a, aux, g.body, lid + kGroup, g.nvec, kGroup);
             any = true;
           }
           if constexpr (kGroup < 8) {
@@ -300,7 +315,7 @@ __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
       init_parts<T>(a);
       uint32_t aux = 0;
       // a queued segment: only the first round here
-      fold_body<T, 4>(a, aux, g.body, threadIdx.x, sl != kNoSlot ? (long long)blockDim.x : g.nvec, blockDim.x);
+      fold_body<T, 4, kTail>(a, aux, g.body, threadIdx.x, sl != kNoSlot ? (long long)blockDim.x : g.nvec, blockDim.x);
       if ((int)threadIdx.x < g.head) fold_elem<T>(a[0], aux, __ldg((const Elem*)g.p + threadIdx.x));
       if ((int)threadIdx.x < g.tail)
         fold_elem<T>(a[T::NA - 1], aux, __ldg((const Elem*)(g.body + g.nvec * kVecBytes) + threadIdx.x));
@@ -391,17 +406,25 @@ cudaError_t seg_launch(K kernel, long long grid, int block, const SegParams& p, 
   return cudaLaunchKernelEx(&cfg, kernel, p);
 }
 
-template <int DT, int OP, int kGroup>
+template <int DT, int OP, int kGroup, bool kTail>
 cudaError_t launch_segmented_group(const SegParams& p, int block, int sms, cudaStream_t s) {
   static int per_sm[17] = {0};  // resident blocks by block / 32 (cached)
   const int key = block / 32;
-  if (per_sm[key] == 0) per_sm[key] = seg_blocks_per_sm(k_segmented<DT, OP, kGroup>, block);
+  if (per_sm[key] == 0) per_sm[key] = seg_blocks_per_sm(k_segmented<DT, OP, kGroup, kTail>, block);
   const long long per_block = kGroup > 0 ? block / kGroup : 1;
   long long grid = (p.nseg + per_block - 1) / per_block;
   const long long cap = (long long)sms * per_sm[key];  // one full wave
   if (grid > cap) grid = cap;
   if (grid < 1) grid = 1;
-  return seg_launch(k_segmented<DT, OP, kGroup>, grid, block, p, s);
+  return seg_launch(k_segmented<DT, OP, kGroup, kTail>, grid, block, p, s);
+}
+
+template <int DT, int OP, bool kTail>
+cudaError_t launch_segmented_groups(const SegParams& p, int group, int block, int sms, cudaStream_t s) {
+  if (group == 1) return launch_segmented_group<DT, OP, 1, kTail>(p, block, sms, s);
+  if (group == 8) return launch_segmented_group<DT, OP, 8, kTail>(p, block, sms, s);
+  if (group == 32) return launch_segmented_group<DT, OP, 32, kTail>(p, block, sms, s);
+  return launch_segmented_group<DT, OP, 0, kTail>(p, block, sms, s);
 }
 
 template <int DT, int OP>
@@ -409,11 +432,8 @@ cudaError_t launch_segmented_op(const SegParams& p, int group, int block, cudaSt
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  cudaError_t e;
-  if (group == 1) e = launch_segmented_group<DT, OP, 1>(p, block, sms, s);
-  else if (group == 8) e = launch_segmented_group<DT, OP, 8>(p, block, sms, s);
-  else if (group == 32) e = launch_segmented_group<DT, OP, 32>(p, block, sms, s);
-  else e = launch_segmented_group<DT, OP, 0>(p, block, sms, s);
+  cudaError_t e = p.tail ? launch_segmented_groups<DT, OP, true>(p, group, block, sms, s)
+                         : launch_segmented_groups<DT, OP, false>(p, group, block, sms, s);
   if (e != cudaSuccess || !p.use_q) return e;
   static int chunk_per_sm = 0;
   if (chunk_per_sm == 0) chunk_per_sm = seg_blocks_per_sm(k_seg_chunks<DT, OP>, 256);
