@@ -146,6 +146,13 @@ constexpr long long kChunkMinVecs = 512;
 constexpr long long kMaxChunks = 4096;
 constexpr unsigned kNoSlot = 0xFFFFFFFFu;
 
+// Chunk geometry of a queued remainder of nv vectors: chunk size and count.
+__device__ __forceinline__ void seg_chunks(long long nv, long long& per_v, long long& k) {
+  per_v = (nv + kMaxChunks - 1) / kMaxChunks;
+  if (per_v < kChunkMinVecs) per_v = kChunkMinVecs;
+  k = (nv + per_v - 1) / per_v;
+}
+
 // Leader of a group: reserve queue slots for the rest of segment `seg` --
 // elements [rem_lo, rem_hi), 32-byte aligned at both ends -- and write its
 // chunk items.  Slot `base` is left for the group's own partial (written
@@ -153,11 +160,9 @@ constexpr unsigned kNoSlot = 0xFFFFFFFFu;
 // the queue is full: the group then finishes the segment itself.
 __device__ __forceinline__ unsigned seg_reserve(unsigned* hdr, long long* items, long long* longs, long long seg,
                                              long long rem_lo, long long rem_hi, int ve) {
-  const long long nv = (rem_hi - rem_lo) / ve;
-  long long per_v = (nv + kMaxChunks - 1) / kMaxChunks;
-  if (per_v < kChunkMinVecs) per_v = kChunkMinVecs;
+  long long per_v, k;
+  seg_chunks((rem_hi - rem_lo) / ve, per_v, k);
   const long long per = per_v * ve;
-  const long long k = (nv + per_v - 1) / per_v;
   const unsigned need = (unsigned)(k + 1);
   const unsigned base = atomicAdd(hdr + 0, need);
   if ((unsigned long long)base + need > kSegQItems) {
@@ -180,6 +185,57 @@ __device__ __forceinline__ unsigned seg_reserve(unsigned* hdr, long long* items,
   longs[3 * (size_t)j + 1] = base;
   longs[3 * (size_t)j + 2] = k + 1;
   return base;
+}
+
+// Warp-collective seg_reserve (every lane of the warp calls it; `want` lanes
+// queue their segment): one atomic per warp on each queue counter instead of
+// one per segment -- with many long segments the two same-address counters
+// were the bottleneck.
+__device__ __forceinline__ unsigned seg_reserve_warp(const SegParams& p, bool want, long long seg, long long rem_lo,
+                                                     long long rem_hi, int ve, int lane) {
+  long long per_v = 0, k = 0;
+  unsigned need = 0;
+  if (want) {
+    seg_chunks((rem_hi - rem_lo) / ve, per_v, k);
+    need = (unsigned)(k + 1);
+  }
+  unsigned incl = need;  // inclusive prefix of the warp's needs
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned t = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += t;
+  }
+  const unsigned total = __shfl_sync(0xffffffffu, incl, 31);
+  if (total == 0) return kNoSlot;
+  unsigned wbase = 0;
+  if (lane == 0) wbase = atomicAdd(p.q.hdr + 0, total);
+  wbase = __shfl_sync(0xffffffffu, wbase, 0);
+  const unsigned long long base = (unsigned long long)wbase + incl - need;
+  const bool fits = want && base + need <= kSegQItems;
+  if (want && !fits) {  // past the end: leave the reachable part of the range empty
+    for (unsigned long long i = base; i < kSegQItems && i < base + need; ++i) {
+      p.q.items[2 * i] = 0;
+      p.q.items[2 * i + 1] = 0;
+    }
+  }
+  const unsigned fit_mask = __ballot_sync(0xffffffffu, fits);
+  unsigned lbase = 0;
+  if (lane == 0 && fit_mask) lbase = atomicAdd(p.q.hdr + 1, (unsigned)__popc(fit_mask));
+  lbase = __shfl_sync(0xffffffffu, lbase, 0);
+  if (!fits) return kNoSlot;
+  const long long per = per_v * ve;
+  p.q.items[2 * base] = 0;  // the group's partial: an empty item
+  p.q.items[2 * base + 1] = 0;
+  for (long long c = 0; c < k; ++c) {
+    const long long lo = rem_lo + c * per;
+    p.q.items[2 * (base + 1 + c)] = lo;
+    p.q.items[2 * (base + 1 + c) + 1] = lo + per < rem_hi ? lo + per : rem_hi;
+  }
+  const unsigned j = lbase + __popc(fit_mask & ((1u << lane) - 1u));
+  p.q.longs[3 * (size_t)j] = seg;
+  p.q.longs[3 * (size_t)j + 1] = (long long)base;
+  p.q.longs[3 * (size_t)j + 2] = k + 1;
+  return (unsigned)base;
 }
 
 // kGroup = 1, 8 or 32 lanes per segment (32 / kGroup segments per warp at a
@@ -229,10 +285,12 @@ __global__ void __launch_bounds__(512) k_segmented(const SegParams p) {
         // a long segment: the leader queues the rest of it (every lane of the
         // warp takes part in the broadcast)
         slot[j] = kNoSlot;
-        if (p.use_q && lid == 0 && g.nvec - kGroup > kLong)
-          slot[j] = seg_reserve(p.q.hdr, p.q.items, p.q.longs, first + (k0 + j) * step,
-                                lo + g.head + (long long)kGroup * T::VE, lo + g.head + g.nvec * T::VE, T::VE);
-        if constexpr (kGroup > 1) slot[j] = __shfl_sync(0xffffffffu, slot[j], leader);
+        if (p.use_q) {  // warp-uniform
+          slot[j] = seg_reserve_warp(p, lid == 0 && g.nvec - kGroup > kLong, first + (k0 + j) * step,
+                                     lo + g.head + (long long)kGroup * T::VE, lo + g.head + g.nvec * T::VE, T::VE,
+                                     lane);
+          if constexpr (kGroup > 1) slot[j] = __shfl_sync(0xffffffffu, slot[j], leader);
+        }
       }
       Acc v[kSegPipe];
 #pragma unroll
