@@ -134,9 +134,10 @@ typedef struct {
                          rows: one thread per row up to 512 bytes, 8 lanes up to 4 KB,
                          one warp up to 16 KB, else one block; offset arrays: 8 lanes),
                          1 = one warp per segment, 2 = one block per segment,
-                         3 = 8 lanes, 4 = one thread.  Whatever the group, segments
-                         much longer than its first round are cut into 64 KB chunks
-                         that whole blocks reduce (two more launches; load balance) */
+                         3 = 8 lanes, 4 = one thread.  Segments much longer than
+                         their group's first round (offset arrays; or fewer than 4096
+                         uniform rows of > 64 KB) are cut into chunks of >= 16 KB that
+                         warps reduce (two more launches; load balance) */
   int stage;          /* 0 = auto; REDUCE_STAGE_REG: 256-bit loads straight into
                          registers; REDUCE_STAGE_SMEM: cp.async 16-byte copies into a
                          shared-memory tile (block*unroll*32 <= 128 KiB), then shared
@@ -197,9 +198,9 @@ int reduce_host(int dtype, int op, const void* host_in, size_t n, void* host_out
  * num_segments elements of dtype.  One thread, 8 lanes, one warp or one block
  * per segment (the paper's small-array versions assign one warp / block per
  * partition with no global atomics); segments much longer than
- * their group's first round are cut into 64 KB chunks that whole blocks reduce,
- * then combined in chunk order (the stream's workspace holds the queue; two
- * more launches; load balance for skewed lengths).  Values never touch
+ * their group's first round are cut into chunks of >= 16 KB that warps
+ * reduce, then combined in chunk order (the stream's workspace holds the
+ * queue; two more launches; load balance for skewed lengths).  Values never touch
  * atomics and every combine has a fixed order: deterministic.  Up to 3
  * launches (1 for uniform rows too short to be cut).  Segment starts may have
  * any element alignment.  Options used: block (32..512, default 256), seg_group.  reduce_batched is the uniform case: num_segments rows of seg_len

@@ -407,17 +407,17 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   p.nseg = (long long)nseg;
   p.out = out;
   p.raw_out = 0;
-  // long-segment queue: needed unless no row can be longer than the group's
-  // first round plus its long threshold (uniform rows only)
+  // long-segment queue.  Offset arrays: always (lengths unknown here; a few
+  // long segments would otherwise keep a few groups busy after the rest of
+  // the GPU is done: power-law lengths 0.3 -> 1.5 TB/s on B200).  The
+  // thresholds stay high -- queueing segments of a few KB (tried: 2 KB for 8
+  // lanes) costs more than it balances.  Uniform rows are balanced by
+  // construction: only when there are too few rows to fill the GPU.
   const long long ve = 32 / s;
   const long long first_round = lanes > 0 ? lanes : block;
   const long long long_vecs = lanes == 1 ? 32 : lanes == 8 ? 512 : lanes == 32 ? 2048 : 8192;
-  const bool may_long = !uniform || (long long)(seg_len / ve) > first_round + long_vecs - 1;
-  // predicated tail round (B200 A/B, tools/probes/seg_tail_ab.sh): accurate
-  // sums and 2-8 KB fp rows with sub-block groups; never for one block per row
-  p.tail = lanes == 0 ? 0
-           : op == REDUCE_SUM_ACCURATE ? 1
-           : (uniform && dtype != REDUCE_INT32 && row_bytes >= 2048 && row_bytes <= 8192) ? 1 : 0;
+  const bool may_long = !uniform || ((long long)(seg_len / ve) > first_round + long_vecs - 1 && nseg < 4096 &&
+                                     row_bytes > (64u << 10));
   p.use_q = 0;
   p.q = SegQueue{nullptr, nullptr, nullptr, nullptr};
   if (may_long) {
