@@ -1,4 +1,6 @@
 #!/usr/bin/env bash
+# (The split path was reverted after this A/B -- see profiles/r01_tail_split_ab.json;
+#  the script is kept as the record of how the numbers were taken.)
 # A/B of the drain split of k_reduce's last tiles: (a) kernels built without
 # the split path, (b) built with it but disabled (REDUCE_TAIL_SPLIT=0), (c) on.
 # Default bench line + ops table each.  GPU box, repo root; restores the build.
