@@ -20,7 +20,8 @@ Extra keys: roofline (dominant kernel vs the measured HBM peak), cpu_baseline
 (the oracle on the host cores), e2e (the same metric through the C-ABI host
 entry with H2D/D2H copies in the timed region), clocks (NVML, sampled during
 the timed region), gpu_launches, and `sweep` (fp32 sum GB/s vs size, each
-call after an L2 flush).
+call on a cold input region, with CUB's DeviceReduce and the CPU baseline --
+oracle and OpenMP loop -- at the same n).
 
 `--impl reference` times the CPU oracle (this tier's reference arm) on the
 same config.  Launch: python bench.py --gpus N --steps K --warmup W
@@ -161,6 +162,22 @@ def host_info():
     except Exception:
         pass
     return model, len(os.sched_getaffinity(0))
+
+
+def host_times(xh):
+    """Median host time (us) of the oracle and of the OpenMP loop on xh (rank 0 context data)."""
+    import oracle
+    reps = 5 if xh.size <= (1 << 22) else 2
+    outs = []
+    for f in (lambda: oracle.reduce(xh, "sum"), lambda: oracle.omp_sum_f32(xh)):
+        f()
+        ts = []
+        for _ in range(reps):
+            t0 = time.perf_counter()
+            f()
+            ts.append(time.perf_counter() - t0)
+        outs.append(round(statistics.median(ts) * 1e6, 2))
+    return outs
 
 
 # --------------------------------------------------------------- reference arm
@@ -502,7 +519,11 @@ def main():
                 cubref.reduce(1, 0, timed[0].data_ptr(), m, outs.data_ptr(), stream.cuda_stream)  # size temp storage
                 torch.cuda.synchronize(dev)
                 cub_sec = time_calls(launch_cub, warm, timed, stream, repeats=3)
+            # the CPU beside it at the same n (the paper's CPU
+            # crossover): the oracle (1 thread) and the OpenMP pragma loop
+            cpu_o, cpu_p = host_times(x_host[:m])
             sweep.append({"n": m, "us": round(sec * 1e6, 3), "GBps": round(gbs, 1),
+                          "cpu_oracle_us": cpu_o, "cpu_omp_us": cpu_p,
                           "cub_us": None if cub_sec is None else round(cub_sec * 1e6, 3),
                           "speedup_vs_cub": None if cub_sec is None else round(cub_sec / sec, 3),
                           "elements_per_s": round(m / sec, 1), "frac_of_peak": round(gbs / peak, 4),
@@ -598,6 +619,15 @@ def main():
                     row[arm] = {"us": round(sec * 1e6, 2), "GBps": round(m * es / sec / 1e9, 1),
                                 "grid_combine": ["direct", "atomic", "two_pass", "last_block", "cluster"][pp["grid_combine"]],
                                 "grid": pp["grid"], "block": pp["block"], "unroll": pp["unroll"]}
+                if dt_name == "float64" and op == "sum":
+                    # distinct results over 20 runs on the same input
+                    for arm, kw in (("atomic", dict(grid_combine=1)), ("tree", dict(mode="deterministic", grid_combine=2))):
+                        outs20 = torch.empty(20, dtype=tdt, device=dev)
+                        for i in range(20):
+                            rb.reduce(regs_t[0], op, out=outs20[i:i + 1], stream=stream, **kw)
+                        torch.cuda.synchronize(dev)
+                        row[arm]["distinct_results_20_runs"] = len(set(outs20.cpu().numpy().tobytes()[8 * i:8 * i + 8]
+                                                                        for i in range(20)))
                 cfg3.append(row)
 
     # ---- BASELINE configs[4] at k = 1: one 8 GiB (2^31 fp32) array on one GPU

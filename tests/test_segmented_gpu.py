@@ -200,3 +200,21 @@ def test_segmented_graph_capture_with_queue():
         g.replay()
         torch.cuda.synchronize()
         assert out.cpu().numpy().tobytes() == ref.tobytes()
+
+
+@pytest.mark.parametrize("group", [0, 1, 2, 3, 4])
+def test_segmented_decreasing_pairs_are_empty(group):
+    """include/reduce.h: a decreasing offsets pair is an empty segment (the
+    identity), including next to long (queued) segments and overlapping ranges"""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    x = synth.make("int32", 300_000, "int_full", 21)
+    offs = np.array([0, 100, 50, 200_000, 150_000, 150_001, 299_999, 10, 300_000], np.int64)
+    xt, ot = torch.from_numpy(x).cuda(), torch.from_numpy(offs).cuda()
+    ident = {"sum": 0, "min": np.iinfo(np.int32).max, "max": np.iinfo(np.int32).min}
+    for op in OPS:
+        got = rb.reduce_segmented(xt, ot, op, seg_group=group).cpu().numpy()
+        for i in range(len(offs) - 1):
+            lo, hi = int(offs[i]), int(offs[i + 1])
+            want = oracle.reduce(x[lo:hi], op).value if hi > lo else ident[op]
+            assert int(got[i]) == int(want), (op, i, lo, hi, got[i], want)
