@@ -511,7 +511,10 @@ int reduce_prepare(reduce_stream_t stream, size_t max_n) {
   char* q = nullptr;
   st = get_seg_queue((cudaStream_t)stream, &q);  // so segmented calls can be captured too
   if (st != REDUCE_OK) return st;
-  cudaError_t e = launch_init_workspace(ws->slots, ws->tickets, (cudaStream_t)stream);
+  // queue counters back to zero too (recovery after an aborted segmented call)
+  cudaError_t e = cudaMemsetAsync(q, 0, kSegQHdrBytes, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "segment queue reset");
+  e = launch_init_workspace(ws->slots, ws->tickets, (cudaStream_t)stream);
   if (e != cudaSuccess) return cuda_fail(e, "workspace init kernel");
   return REDUCE_OK;
 }
