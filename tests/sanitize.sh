@@ -1,7 +1,9 @@
 #!/usr/bin/env bash
 # compute-sanitizer pass over every kernel family (SURVEY section 4 "Sanitizers"):
 # memcheck, racecheck, synccheck and initcheck on small ragged sizes, every grid
-# combine (DIRECT, ATOMIC, TWO_PASS, LAST_BLOCK, CLUSTER), both staging modes.
+# combine (DIRECT, ATOMIC, TWO_PASS, LAST_BLOCK, CLUSTER), both staging modes,
+# every segmented group with and without the long-segment queue, the histogram
+# bin-replication and quotient paths, and the team combine.
 # Usage (GPU box): bash tests/sanitize.sh  -> exit 0 iff every tool reports 0 errors.
 set -u
 cd "$(dirname "$0")/.."
@@ -22,12 +24,22 @@ for dt in (torch.int32, torch.float32, torch.float64):
             rb.reduce(x, "sum_accurate", mode="deterministic")
     offs = torch.tensor([0, 0, 1, 33, 100, 4097], dtype=torch.int64, device="cuda")
     base = torch.arange(5000, device="cuda").to(dt)[1:]
-    for g in (0, 1, 2, 3):
+    # long segments (queued: k_seg_chunks / k_seg_finish) among short ones,
+    # a decreasing pair, and few long uniform rows (queued too)
+    loffs = torch.tensor([0, 5, 70005, 70006, 60000, 150003, 150040], dtype=torch.int64, device="cuda")
+    lbase = torch.arange(150050, device="cuda").to(dt)[3:]
+    for g in (0, 1, 2, 3, 4):
         rb.reduce_segmented(base, offs, "sum", seg_group=g)
         rb.reduce_batched(base[:4096].view(64, 64), "max", seg_group=g)
+        rb.reduce_segmented(lbase, loffs, "sum", seg_group=g)
+        rb.reduce_batched(lbase[:3 * 40001].view(3, 40001), "min", seg_group=g)
+        if dt != torch.int32:
+            rb.reduce_segmented(lbase, loffs, "sum_accurate", seg_group=g)
     if dt != torch.float64:
-        for nb in (7, 20000, 1 << 20):
+        for nb in (7, 256, 4096, 20000, 1 << 20):
             rb.histogram(base, 0, 4000, nb)
+        if dt == torch.int32:
+            rb.histogram(base, -2.0 ** 31, 2.0 ** 31, 1000)  # 64-bit quotient path
 # team combine (k = 1: members on one GPU cannot run concurrently under the
 # sanitizer, which serialises kernels, so k > 1 would wait for itself)
 team = rb.Team.local(1)[0]
