@@ -241,6 +241,7 @@ static void free_workspace(Workspace* w) {
   if (w->base) cudaFree(w->base);
   if (w->partials) cudaFree(w->partials);
   if (w->segq) cudaFree(w->segq);
+  if (w->segbal) cudaFree(w->segbal);
   if (w->staging) cudaFree(w->staging);
   for (int i = 0; i < 2; ++i) {
     if (w->ev_copied[i]) cudaEventDestroy(w->ev_copied[i]);
@@ -335,6 +336,34 @@ int get_seg_queue(cudaStream_t stream, char** out) {
   return REDUCE_OK;
 }
 
+// The stream's chunk arrays of the element-balanced segmented path (allocated
+// and its header zeroed on first use, or by reduce_prepare before a capture).
+int get_seg_bal(cudaStream_t stream, char** out) {
+  Workspace* w = nullptr;
+  int st = get_workspace(stream, 0, &w);
+  if (st != REDUCE_OK) return st;
+  std::lock_guard<std::mutex> lk(g_ws_mu);
+  if (w->segbal == nullptr) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone)
+      return fail(REDUCE_ERR_NOT_PREPARED, "segment chunk arrays missing during stream capture: call reduce_prepare first");
+    char* b = nullptr;
+    cudaError_t e = cudaMalloc((void**)&b, kBalBytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(REDUCE_ERR_NO_MEMORY, "cudaMalloc(segment chunk arrays) failed");
+    }
+    e = cudaMemsetAsync(b, 0, kBalHdrBytes, stream);
+    if (e != cudaSuccess) {
+      cudaFree(b);
+      return cuda_fail(e, "segment chunk arrays init");
+    }
+    w->segbal = b;
+  }
+  *out = w->segbal;
+  return REDUCE_OK;
+}
+
 int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream) {
   LaunchDesc& d = P->d;
   const int combo = combo_index(d.dtype, d.op);
@@ -390,17 +419,36 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   if (opts) {
     if (opts->block != 0 && (opts->block < 32 || opts->block > 512 || opts->block % 32 != 0))
       return fail(REDUCE_ERR_INVALID_ARG, "segmented block must be 0 or a multiple of 32 in [32, 512]");
-    if (opts->seg_group < 0 || opts->seg_group > 4) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0..4");
+    if (opts->seg_group < 0 || opts->seg_group > 5) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0..5");
+    if (opts->seg_group == 5 && uniform) return fail(REDUCE_ERR_INVALID_ARG, "seg_group 5 (balanced) needs an offsets array");
     if (opts->block) block = opts->block;
     group = opts->seg_group;
   }
   // auto: by row bytes for uniform batches (B200 sweep, tools/seg_bench.py);
-  // 8 lanes for offset arrays (long segments go to the queue either way)
+  // element-balanced chunks for offset arrays (reduce_segbal.cuh), else 8
+  // lanes (long segments go to the queue either way)
+  const bool want_bal = !uniform && (group == 0 || group == 5) && nseg < 0xFFFFFFFFull;
+  if (want_bal) {
+    char* b = nullptr;
+    if (get_seg_bal((cudaStream_t)stream, &b) == REDUCE_OK) {  // else (capture without prepare): group kernels
+      SegParams p{};
+      p.in = (const char*)in;
+      p.offsets = (const long long*)offsets;
+      p.nseg = (long long)nseg;
+      p.out = out;
+      p.balanced = 1;
+      p.b = seg_bal_at(b);
+      cudaError_t e = launch_segmented(dtype, op, p, 0, 0, (cudaStream_t)stream);
+      if (e != cudaSuccess) return cuda_fail(e, "segmented reduction launch");
+      return REDUCE_OK;
+    }
+  }
+  if (group == 5) group = 3;
   const unsigned long long row_bytes = (unsigned long long)seg_len * (unsigned long long)s;
   if (group == 0)
     group = !uniform ? 3 : (row_bytes <= 512 ? 4 : (row_bytes <= 4096 ? 3 : (row_bytes <= 16384 ? 1 : 2)));
   const int lanes = group == 1 ? 32 : (group == 3 ? 8 : (group == 4 ? 1 : 0));
-  SegParams p;
+  SegParams p{};
   p.in = (const char*)in;
   p.offsets = (const long long*)offsets;
   p.seg_len = (long long)seg_len;
@@ -511,6 +559,10 @@ int reduce_prepare(reduce_stream_t stream, size_t max_n) {
   char* q = nullptr;
   st = get_seg_queue((cudaStream_t)stream, &q);  // so segmented calls can be captured too
   if (st != REDUCE_OK) return st;
+  char* b = nullptr;
+  st = get_seg_bal((cudaStream_t)stream, &b);
+  if (st != REDUCE_OK) return st;
+  if (cudaMemsetAsync(b, 0, kBalHdrBytes, (cudaStream_t)stream) != cudaSuccess) return cuda_fail(cudaGetLastError(), "segment chunk arrays reset");
   // queue counters back to zero too (recovery after an aborted segmented call)
   cudaError_t e = cudaMemsetAsync(q, 0, kSegQHdrBytes, (cudaStream_t)stream);
   if (e != cudaSuccess) return cuda_fail(e, "segment queue reset");

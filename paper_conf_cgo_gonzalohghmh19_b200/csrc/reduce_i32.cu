@@ -1,7 +1,7 @@
 // reduce_i32.cu -- instantiates the reduction kernels for one dtype (split per
 // dtype so the 48 kernel instantiations per dtype compile in parallel).
 #include "reduce_kernels.cuh"
-#include "reduce_segmented.cuh"
+#include "reduce_segbal.cuh"
 #include "reduce_histogram.cuh"
 
 namespace rb {
@@ -11,6 +11,7 @@ cudaError_t combine_i32(int op, const void* v, long long c, void* out, int raw, 
 }
 cudaError_t init_i32(char* slots, char* tickets, cudaStream_t s) { return init_dt<DT_I32>(slots, tickets, s); }
 cudaError_t segmented_i32(int op, const SegParams& p, int group, int block, cudaStream_t s) {
+  if (p.balanced) return launch_segbal_dt<DT_I32>(op, p, s);
   return launch_segmented_dt<DT_I32>(op, p, group, block, s);
 }
 cudaError_t histogram_i32(const HistParams& p, int block, cudaStream_t s) {

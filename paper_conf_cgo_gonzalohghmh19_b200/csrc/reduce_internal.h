@@ -104,6 +104,33 @@ inline SegQueue seg_queue_at(char* base) {
   return q;
 }
 
+// Element-balanced segmented reduction of an offsets array (reduce_segbal.cuh):
+// the elements are cut into fixed 8 KB chunks, one warp per chunk whatever the
+// segment lengths; per-chunk boundary pieces are joined by a fix-up pass.
+constexpr unsigned kBalChunks = 1u << 20;  // chunks per call (8 GiB of input)
+constexpr size_t kBalHdrBytes = 256;
+constexpr size_t kBalBytes = kBalHdrBytes + (size_t)kBalChunks * (4 /* start_seg */ + 16 /* first */ +
+                                                                   16 /* last */ + 4 /* last_seg */ + 4 /* flags */);
+struct SegBal {
+  unsigned* hdr;         // [0] non-monotone offsets seen, [1] fix-up ticket (both self-resetting)
+  unsigned* start_seg;   // [c]: the segment holding chunk c's first element
+  void* first_val;       // Grid[c]: chunk c's piece of the segment it starts inside
+  void* last_val;        // Grid[c]: chunk c's piece of the segment still open at its end
+  unsigned* last_seg;    // [c]: that open segment
+  unsigned* flags;       // [c]: 1 if a segment boundary lies inside chunk c
+};
+inline SegBal seg_bal_at(char* base) {
+  SegBal b;
+  char* p = base + kBalHdrBytes;
+  b.hdr = (unsigned*)base;
+  b.first_val = p;  p += (size_t)kBalChunks * 16;
+  b.last_val = p;   p += (size_t)kBalChunks * 16;
+  b.start_seg = (unsigned*)p;  p += (size_t)kBalChunks * 4;
+  b.last_seg = (unsigned*)p;   p += (size_t)kBalChunks * 4;
+  b.flags = (unsigned*)p;
+  return b;
+}
+
 // One segmented / batched call, see reduce_segmented.cuh.
 struct SegParams {
   const char* in;
@@ -115,6 +142,8 @@ struct SegParams {
   int use_q;                 // 1: offload long segments to q (2 more launches)
   int tail;                  // 1: fold a segment's last vectors in one predicated round
   SegQueue q;
+  int balanced;              // 1: element-balanced chunks (offsets arrays, reduce_segbal.cuh)
+  SegBal b;
 };
 // group: lanes per segment (1, 8 or 32) or 0 = one block per segment.
 cudaError_t launch_segmented(int dtype, int op, const SegParams& p, int group, int block, cudaStream_t s);

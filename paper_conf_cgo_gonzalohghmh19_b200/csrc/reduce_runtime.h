@@ -22,6 +22,7 @@ struct Workspace {
   char* partials = nullptr;    // per-block / per-chunk Grid values
   size_t partials_bytes = 0;
   char* segq = nullptr;        // long-segment queue of reduce_segmented / reduce_batched (kSegQBytes)
+  char* segbal = nullptr;      // chunk arrays of the element-balanced reduce_segmented (kBalBytes)
   // reduce_host staging (lazily created)
   char* staging = nullptr;     // 2 x staging_bytes
   size_t staging_bytes = 0;

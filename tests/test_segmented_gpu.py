@@ -20,6 +20,9 @@ def _chain(length, dtype, lanes):
     # per-thread: m vectors through a lane tree (depth log2 VE) into 2 accumulators
     # (or one accumulator per lane), + head/tail, + merge; then group / block combines
     ve = 4 if dtype == "float64" else 8
+    if lanes < 0:  # element-balanced chunks: <= 8*VE elements in order per lane, lane scan,
+        el = 8 * ve  # then the chunk pieces joined 32 at a time by warp butterflies
+        return min(length, el) + 1 + 5 + 1 + math.ceil(math.ceil(length / (32 * el) + 1) / 32) * 6 + 2
     m = math.ceil(length / (ve * lanes))
     return m + int(math.log2(ve)) + 3 + 5 + (5 if lanes > 32 else 0)
 
@@ -63,7 +66,7 @@ def test_segmented_matches_oracle_per_segment(dtype, group, skew):
     xt = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     ot = torch.from_numpy(offs).cuda()
     bounds = list(zip(offs[:-1].tolist(), offs[1:].tolist()))
-    lanes = {0: 8, 1: 32, 2: 256, 3: 8, 4: 1}[group]
+    lanes = {0: -1, 1: 32, 2: 256, 3: 8, 4: 1}[group]
     for op in OPS:
         got = rb.reduce_segmented(xt, ot, op, seg_group=group).cpu().numpy()
         _check_segments(x, bounds, op, got, lanes)
@@ -98,10 +101,10 @@ def test_segmented_special_values_and_determinism():
     offs = np.array([0, 10, 10, 50001, 70000, 70001, 100000], np.int64)
     xt, ot = torch.from_numpy(x).cuda(), torch.from_numpy(offs).cuda()
     bounds = list(zip(offs[:-1].tolist(), offs[1:].tolist()))
-    for group in (1, 2, 3):
+    for group in (1, 2, 3, 5):
         for op in OPS:
             got = rb.reduce_segmented(xt, ot, op, seg_group=group).cpu().numpy()
-            _check_segments(x, bounds, op, got, {1: 32, 2: 256, 3: 8}[group])
+            _check_segments(x, bounds, op, got, {1: 32, 2: 256, 3: 8, 5: -1}[group])
     outs = {rb.reduce_segmented(xt, ot, "sum").cpu().numpy().tobytes() for _ in range(20)}
     assert len(outs) == 1
 
@@ -132,7 +135,7 @@ def test_segmented_long_segments_load_balanced(dtype, group):
     xt = to_device(x, 3)
     ot = torch.from_numpy(offs).cuda()
     bounds = list(zip(offs[:-1].tolist(), offs[1:].tolist()))
-    lanes = {0: 8, 1: 32, 2: 256, 3: 8, 4: 1}[group]
+    lanes = {0: -1, 1: 32, 2: 256, 3: 8, 4: 1}[group]
     for op in OPS + (["sum_accurate"] if dtype != "int32" else []):
         got = rb.reduce_segmented(xt, ot, op, seg_group=group)
         if op == "sum_accurate":
