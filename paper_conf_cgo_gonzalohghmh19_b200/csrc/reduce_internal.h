@@ -105,29 +105,32 @@ inline SegQueue seg_queue_at(char* base) {
 }
 
 // Element-balanced segmented reduction of an offsets array (reduce_segbal.cuh):
-// the elements are cut into fixed 8 KB chunks, one warp per chunk whatever the
-// segment lengths; per-chunk boundary pieces are joined by a fix-up pass.
-constexpr unsigned kBalChunks = 1u << 20;  // chunks per call (8 GiB of input)
+// the elements are cut into fixed 8 KB chunks and every warp of a one-wave
+// grid reduces one contiguous range of chunks whatever the segment lengths;
+// the pieces of segments that cross ranges are joined by a fix-up pass.
+constexpr unsigned kBalRanges = 1u << 16;  // capacity of the per-range arrays (ranges = chunk-kernel warps)
 constexpr size_t kBalHdrBytes = 256;
-constexpr size_t kBalBytes = kBalHdrBytes + (size_t)kBalChunks * (4 /* start_seg */ + 16 /* first */ +
+constexpr size_t kBalBytes = kBalHdrBytes + (size_t)kBalRanges * (4 /* start_seg */ + 16 /* first */ +
                                                                    16 /* last */ + 4 /* last_seg */ + 4 /* flags */);
 struct SegBal {
   unsigned* hdr;         // [0] non-monotone offsets seen, [1] fix-up ticket (both self-resetting)
-  unsigned* start_seg;   // [c]: the segment holding chunk c's first element
-  void* first_val;       // Grid[c]: chunk c's piece of the segment it starts inside
-  void* last_val;        // Grid[c]: chunk c's piece of the segment still open at its end
-  unsigned* last_seg;    // [c]: that open segment
-  unsigned* flags;       // [c]: 1 if a segment boundary lies inside chunk c
+  unsigned* start_seg;   // [w]: the segment holding range w's first element
+  void* first_val;       // Grid[w]: range w's piece of the segment open at its start
+  void* last_val;        // Grid[w]: range w's piece of the segment still open at its end
+  unsigned* last_seg;    // [w]: that open segment (0xFFFFFFFF: none)
+  unsigned* flags;       // [w]: 1 if a segment boundary lies inside range w
+  long long nranges;     // ranges = warps of the chunk kernel's grid (set by the launcher)
 };
 inline SegBal seg_bal_at(char* base) {
   SegBal b;
   char* p = base + kBalHdrBytes;
   b.hdr = (unsigned*)base;
-  b.first_val = p;  p += (size_t)kBalChunks * 16;
-  b.last_val = p;   p += (size_t)kBalChunks * 16;
-  b.start_seg = (unsigned*)p;  p += (size_t)kBalChunks * 4;
-  b.last_seg = (unsigned*)p;   p += (size_t)kBalChunks * 4;
+  b.first_val = p;  p += (size_t)kBalRanges * 16;
+  b.last_val = p;   p += (size_t)kBalRanges * 16;
+  b.start_seg = (unsigned*)p;  p += (size_t)kBalRanges * 4;
+  b.last_seg = (unsigned*)p;   p += (size_t)kBalRanges * 4;
   b.flags = (unsigned*)p;
+  b.nranges = 0;
   return b;
 }
 

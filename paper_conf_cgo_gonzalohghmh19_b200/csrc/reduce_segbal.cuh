@@ -37,6 +37,7 @@
 // offsets: deterministic.  Chunk geometry depends only on the input address
 // modulo 32 and offsets[0].
 #pragma once
+#include <climits>
 #include "reduce_segmented.cuh"
 
 namespace rb {
@@ -112,6 +113,20 @@ __device__ __forceinline__ typename T::Acc bal_warp_range(const SegParams& p, lo
   return T::warp(thread_result<T>(a, aux));
 }
 
+// The chunks are split into contiguous ranges, one per warp of k_segbal's
+// grid: range w = [cb(w), cb(w + 1)), cb(w) = w*per + min(w, rem).
+struct BalRanges {
+  long long per, rem;
+  __device__ BalRanges(long long nchunks, long long nranges) : per(nchunks / nranges), rem(nchunks % nranges) {}
+  __device__ long long begin(long long w) const { return w * per + (w < rem ? w : rem); }
+  // the first range starting at or after chunk c
+  __device__ long long first_at(long long c) const {
+    if (per == 0) return c;
+    const long long t = rem * (per + 1);
+    return c <= t ? (c + per) / (per + 1) : rem + (c - t + per - 1) / per;
+  }
+};
+
 template <int DT, int OP>
 __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
   using T = Tr<DT, OP>;
@@ -119,44 +134,60 @@ __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
   pdl_wait();
   const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < p.nseg) {
-    const long long E0 = __ldg(p.offsets), lo = __ldg(p.offsets + i), hi = __ldg(p.offsets + i + 1);
+    const long long E0 = __ldg(p.offsets), E1 = __ldg(p.offsets + p.nseg);
+    const long long lo = __ldg(p.offsets + i), hi = __ldg(p.offsets + i + 1);
     if (hi < lo) atomicOr(p.b.hdr, 1u);
     if (hi <= lo) {
       seg_store<T>(p, i, T::gident());
-    } else {
+    } else if (E1 > E0) {
+      // start_seg[w] = i for the ranges whose first chunk starts in [lo, hi)
+      // (chunk 0 starts at E0, chunk c > 0 at P0 + c*C)
       const long long P0 = bal_origin<B::s>(p.in, E0);
-      long long c0 = lo <= E0 ? 0 : (lo - P0 + B::C - 1) / B::C;  // chunks starting in [lo, hi)
+      const long long nchunks = (E1 - P0 + B::C - 1) / B::C;
+      const long long c0 = lo <= E0 ? 0 : (lo - P0 + B::C - 1) / B::C;
       long long c1 = (hi - P0 + B::C - 1) / B::C;
-      if (c1 > (long long)kBalChunks) c1 = kBalChunks;
-      for (long long c = c0; c < c1; ++c) p.b.start_seg[c] = (unsigned)i;
+      if (c1 > nchunks) c1 = nchunks;
+      const BalRanges R(nchunks, p.b.nranges);
+      for (long long w = R.first_at(c0); w < p.b.nranges && R.begin(w) < c1; ++w) p.b.start_seg[w] = (unsigned)i;
     }
   }
   pdl_trigger();
 }
 
+// What one chunk leaves for the range it belongs to (warp-uniform).
+template <class T>
+struct BalChunk {
+  typename T::Grid first;  // piece of the segment open at the chunk's start (whole chunk if !has_b)
+  typename T::Grid last;   // piece of the segment open at its end (if has_b)
+  unsigned last_seg;       // that segment (0xFFFFFFFF: none, past the last offset)
+  bool has_b;              // a segment boundary lies in the chunk
+  long long s_next;        // the segment holding the chunk's last element (next chunk's list start)
+};
+
 // The slow path of one chunk (its offsets slice does not fit the shared list:
 // thousands of empty segments): walk the segments in global memory, one warp
 // fold per piece.  Same outputs as the fast path.
 template <class T>
-__device__ __forceinline__ void bal_chunk_walk(const SegParams& p, long long c, long long clo, long long chi,
-                                            long long E0, long long E1, unsigned s0, int lane) {
-  using Grid = typename T::Grid;
+__device__ __forceinline__ BalChunk<T> bal_chunk_walk(const SegParams& p, long long clo, long long chi,
+                                                      long long E0, long long E1, long long s0, int lane) {
   const long long nseg = p.nseg;
   const long long vlo = clo > E0 ? clo : E0, vhi = chi < E1 ? chi : E1;
+  BalChunk<T> r;
+  r.first = r.last = T::gident();
+  r.last_seg = 0xFFFFFFFFu;
   long long j = s0;
   bool incoming = __ldg(p.offsets + j) < clo;
-  unsigned has_b = incoming ? 0u : 1u;
-  Grid first = T::gident(), last = T::gident();
-  unsigned lseg = 0xFFFFFFFFu;
+  r.has_b = !incoming;
+  r.s_next = s0;
   long long pos = vlo;
   while (true) {
     const long long end = __ldg(p.offsets + j + 1);
     const typename T::Acc v = bal_warp_range<T>(p, pos, end < vhi ? end : vhi, lane);
     if (end < chi) {  // segment j closes inside the chunk
       if (incoming) {
-        first = T::to_grid(v);
+        r.first = T::to_grid(v);
         incoming = false;
-        has_b = 1u;
+        r.has_b = true;
       } else if (lane == 0) {
         bal_store<T>(p, j, T::to_grid(v));
       }
@@ -166,25 +197,63 @@ __device__ __forceinline__ void bal_chunk_walk(const SegParams& p, long long c, 
       pos = end;
       if (j >= nseg) break;
     } else {
-      if (incoming) first = last = T::to_grid(v);
-      else { last = T::to_grid(v); lseg = (unsigned)j; }
+      if (incoming) r.first = T::to_grid(v);
+      else { r.last = T::to_grid(v); r.last_seg = (unsigned)j; }
+      r.s_next = j;
       break;
     }
   }
-  if (lane == 0) {
-    ((Grid*)p.b.first_val)[c] = first;
-    ((Grid*)p.b.last_val)[c] = last;
-    p.b.flags[c] = has_b;
-    p.b.last_seg[c] = lseg;
+  return r;
+}
+
+template <class V>
+__device__ __forceinline__ V shfl_idx_v(V v, int src) { return __shfl_sync(0xffffffffu, v, src); }
+__device__ __forceinline__ double2 shfl_idx_v(double2 v, int src) {
+  return make_double2(__shfl_sync(0xffffffffu, v.x, src), __shfl_sync(0xffffffffu, v.y, src));
+}
+
+// 8 x 32-byte loads of lane `lane` of an interior chunk (all in flight)
+template <class T>
+__device__ __forceinline__ void bal_load(const char* in, long long clo, int lane, uint32_t (&r)[kBalVecsPerLane][8]) {
+  const char* lp = in + (clo + (long long)lane * Bal<T>::EL) * Bal<T>::s;
+#pragma unroll
+  for (int j = 0; j < kBalVecsPerLane; ++j) ld_v8(lp + j * kVecBytes, r[j]);
+}
+
+// the same for the first / last chunk: partial vectors element by element,
+// positions outside [E0, E1) hold the identity
+template <class T>
+__device__ __forceinline__ void bal_load_edge(const char* in, long long clo, long long E0, long long E1, int lane,
+                                              uint32_t (&r)[kBalVecsPerLane][8]) {
+  using Elem = typename T::Elem;
+  const Elem eid = elem_ident<T>();
+  const long long e_lane = clo + (long long)lane * Bal<T>::EL;
+  const char* lp = in + e_lane * Bal<T>::s;
+#pragma unroll
+  for (int j = 0; j < kBalVecsPerLane; ++j) {
+    const long long v0 = e_lane + (long long)j * T::VE;
+    if (v0 >= E0 && v0 + T::VE <= E1) {
+      ld_v8(lp + j * kVecBytes, r[j]);
+    } else {
+#pragma unroll
+      for (int e = 0; e < T::VE; ++e) {
+        const Elem x = (v0 + e >= E0 && v0 + e < E1) ? __ldg((const Elem*)lp + j * T::VE + e) : eid;
+        if constexpr (sizeof(Elem) == 4) {
+          r[j][e] = *reinterpret_cast<const uint32_t*>(&x);
+        } else {
+          r[j][2 * e] = (uint32_t)__double2loint(x);
+          r[j][2 * e + 1] = (uint32_t)__double2hiint(x);
+        }
+      }
+    }
   }
 }
 
 template <int DT, int OP>
-__global__ void __launch_bounds__(kBalWarps * 32) k_segbal(const SegParams p) {
+__global__ void __launch_bounds__(kBalWarps * 32, 4) k_segbal(const SegParams p) {
   using T = Tr<DT, OP>;
   using B = Bal<T>;
   using Acc = typename T::Acc;
-  using Elem = typename T::Elem;
   using Grid = typename T::Grid;
   extern __shared__ __align__(16) unsigned char bal_smem[];
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -196,10 +265,9 @@ __global__ void __launch_bounds__(kBalWarps * 32) k_segbal(const SegParams p) {
   const unsigned nonmono = *(volatile unsigned*)p.b.hdr;
   const long long P0 = bal_origin<B::s>(p.in, E0);
   const long long nchunks = E1 > E0 ? (E1 - P0 + B::C - 1) / B::C : 0;
-  const long long gw = (long long)blockIdx.x * kBalWarps + wib, nw = (long long)gridDim.x * kBalWarps;
-  if (nonmono || nchunks > (long long)kBalChunks) {
-    // offsets not monotone (overlapping segments) or more chunks than the
-    // workspace holds: one warp per segment
+  const long long gw = (long long)blockIdx.x * kBalWarps + wib, nw = p.b.nranges;
+  if (nonmono) {
+    // offsets not monotone (overlapping segments): one warp per segment
 #pragma unroll 1
     for (long long seg = gw; seg < nseg; seg += nw) {
       const long long lo = __ldg(p.offsets + seg), hi = __ldg(p.offsets + seg + 1);
@@ -210,46 +278,50 @@ __global__ void __launch_bounds__(kBalWarps * 32) k_segbal(const SegParams p) {
     pdl_trigger();
     return;
   }
-  const Elem eid = elem_ident<T>();
-#pragma unroll 1
-  for (long long c = gw; c < nchunks; c += nw) {
-    const long long clo = P0 + c * B::C, chi = clo + B::C;
-    const unsigned s0 = __ldcg(p.b.start_seg + c);
-    // 1. the lane's 256 bytes, all loads in flight
-    uint32_t r[kBalVecsPerLane][8];
-    const long long e_lane = clo + (long long)lane * B::EL;
-    const char* lp = p.in + e_lane * B::s;
-    if (clo >= E0 && chi <= E1) {
-#pragma unroll
-      for (int j = 0; j < kBalVecsPerLane; ++j) ld_v8(lp + j * kVecBytes, r[j]);
-    } else {  // first / last chunk: partial vectors element by element, outside [E0, E1) the identity
-#pragma unroll
-      for (int j = 0; j < kBalVecsPerLane; ++j) {
-        const long long v0 = e_lane + (long long)j * T::VE;
-        if (v0 >= E0 && v0 + T::VE <= E1) {
-          ld_v8(lp + j * kVecBytes, r[j]);
-        } else {
-#pragma unroll
-          for (int e = 0; e < T::VE; ++e) {
-            const Elem x = (v0 + e >= E0 && v0 + e < E1) ? __ldg((const Elem*)lp + j * T::VE + e) : eid;
-            if constexpr (sizeof(Elem) == 4) {
-              r[j][e] = *reinterpret_cast<const uint32_t*>(&x);
-            } else {
-              r[j][2 * e] = (uint32_t)__double2loint(x);
-              r[j][2 * e + 1] = (uint32_t)__double2hiint(x);
-            }
-          }
-        }
+  const BalRanges R(nchunks, nw);
+  const long long cb = R.begin(gw), ce = R.begin(gw + 1);
+  // the range's carry: the piece of the segment open at the range's start
+  // (until the range's first boundary), then the segment opened last
+  Grid rfirst = T::gident(), carry = T::gident();
+  bool seen = false;
+  unsigned carry_seg = 0xFFFFFFFFu;
+  auto absorb = [&](const BalChunk<T>& k) {
+    if (!k.has_b) {
+      if (seen) carry = T::gcomb(carry, k.first); else rfirst = T::gcomb(rfirst, k.first);
+    } else {
+      if (seen) {
+        if (lane == 0 && carry_seg != 0xFFFFFFFFu) seg_store<T>(p, carry_seg, T::gcomb(carry, k.first));
+      } else {
+        rfirst = T::gcomb(rfirst, k.first);
+        seen = true;
       }
+      carry = k.last;
+      carry_seg = k.last_seg;
     }
-    // 2. the chunk's offsets slice as chunk-local positions: -1 before the
+  };
+  auto interior = [&](long long c) {
+    const long long clo = P0 + c * B::C;
+    return clo >= E0 && clo + B::C <= E1;
+  };
+  // list start of the current chunk and its first two batches of offsets
+  // (prefetched while the previous chunk is folded)
+  long long s0 = 0, vfirst = 0, vsecond = 0;
+  auto prefetch_list = [&](long long s) {
+    vfirst = s + lane <= nseg ? __ldg(p.offsets + s + lane) : LLONG_MAX;
+    vsecond = s + 32 + lane <= nseg ? __ldg(p.offsets + s + 32 + lane) : LLONG_MAX;
+  };
+  auto body = [&](long long c) {
+    const long long clo = P0 + c * B::C, chi = clo + B::C;
+    uint32_t cur[kBalVecsPerLane][8];
+    if (interior(c)) bal_load<T>(p.in, clo, lane, cur);
+    else bal_load_edge<T>(p.in, clo, E0, E1, lane, cur);
+    // the chunk's offsets slice as chunk-local positions: -1 before the
     // chunk, C at / after its end (the first such entry ends the list)
     int m = 0;
     bool ovf = false;
+    long long v = vfirst;
 #pragma unroll 1
-    for (long long base = s0;; base += 32) {
-      const long long idx = base + lane;
-      const long long v = idx <= nseg ? __ldg(p.offsets + idx) : chi;
+    for (long long base = s0;;) {
       const int loc = v < clo ? -1 : (v >= chi ? (int)B::C : (int)(v - clo));
       const unsigned stop = __ballot_sync(0xffffffffu, loc == (int)B::C);
       const int cnt = stop ? __ffs(stop) : 32;
@@ -260,119 +332,131 @@ __global__ void __launch_bounds__(kBalWarps * 32) k_segbal(const SegParams p) {
       if (lane < cnt) list[m + lane] = (short)loc;
       m += cnt;
       if (stop) break;
+      base += 32;
+      v = base == s0 + 32 ? vsecond : (base + lane <= nseg ? __ldg(p.offsets + base + lane) : LLONG_MAX);
     }
     __syncwarp();
+    BalChunk<T> k;
     if (ovf) {
-      bal_chunk_walk<T>(p, c, clo, chi, E0, E1, s0, lane);
-      __syncwarp();
-      continue;
+      k = bal_chunk_walk<T>(p, clo, chi, E0, E1, s0, lane);
+    } else {
+      k.s_next = s0 + m - 2;
     }
-    // 3. the lane's boundaries as a bit mask (bit e: a segment starts at element e)
-    const int a0 = lane * B::EL;
-    int i0 = 0;
-    {
-      int hi_i = m - 1;  // list[m - 1] == C > a0
-      while (i0 < hi_i) {
-        const int mid = (i0 + hi_i) >> 1;
-        if (list[mid] < a0) i0 = mid + 1; else hi_i = mid;
+    if (c + 1 < ce) prefetch_list(k.s_next);  // the next chunk's offsets, while this one folds
+    if (!ovf) {
+      // the lane's boundaries as a bit mask (bit e: a segment starts at element e)
+      const int a0 = lane * B::EL;
+      int i0 = 0;
+      {
+        int hi_i = m - 1;  // list[m - 1] == C > a0
+        while (i0 < hi_i) {
+          const int mid = (i0 + hi_i) >> 1;
+          if (list[mid] < a0) i0 = mid + 1; else hi_i = mid;
+        }
       }
-    }
-    unsigned long long mask = 0;
+      unsigned long long mask = 0;
 #pragma unroll 1
-    for (int j = i0; list[j] < a0 + B::EL; ++j) mask |= 1ull << (list[j] - a0);
-    const unsigned fb = __ballot_sync(0xffffffffu, mask != 0ull);
-    if (fb == 0u) {  // no boundary in the chunk: plain vector-tree fold
-      Part<T> acc[T::NA];
-      init_parts<T>(acc);
-      uint32_t aux = 0;
+      for (int j = i0; list[j] < a0 + B::EL; ++j) mask |= 1ull << (list[j] - a0);
+      const unsigned fb = __ballot_sync(0xffffffffu, mask != 0ull);
+      if (fb == 0u) {  // no boundary in the chunk: plain vector-tree fold
+        Part<T> acc[T::NA];
+        init_parts<T>(acc);
+        uint32_t aux = 0;
 #pragma unroll
-      for (int j = 0; j < kBalVecsPerLane; ++j) fold_vec<T>(acc, aux, r[j], j);
-      const Acc w = T::warp(thread_result<T>(acc, aux));
-      if (lane == 0) {
-        ((Grid*)p.b.first_val)[c] = T::to_grid(w);
-        ((Grid*)p.b.last_val)[c] = T::to_grid(w);
-        p.b.flags[c] = 0u;
-        p.b.last_seg[c] = 0xFFFFFFFFu;
-      }
-      __syncwarp();
-      continue;
-    }
-    // 4. fold element by element, closing a piece at every boundary
-    Part<T> a = PartOf<T>::ident();
-    uint32_t aux = 0;
-    int np = 0;
+        for (int j = 0; j < kBalVecsPerLane; ++j) fold_vec<T>(acc, aux, cur[j], j);
+        k.first = T::to_grid(T::warp(thread_result<T>(acc, aux)));
+        k.has_b = false;
+      } else {
+        // fold element by element, closing a piece at every boundary
+        Part<T> a = PartOf<T>::ident();
+        uint32_t aux = 0;
+        int np = 0;
 #pragma unroll
-    for (int e = 0; e < B::EL; ++e) {  // fully unrolled: constant register indices and shifts
-      if ((mask >> e) & 1ull) {
-        pieces[np * 32 + lane] = T::finish(PartOf<T>::to_acc(a), aux);
-        ++np;
-        a = PartOf<T>::ident();
-        aux = 0;
-      }
-      bal_fold1<T>(a, aux, bal_elem<T>(r, e));
-    }
-    const Acc tail = T::finish(PartOf<T>::to_acc(a), aux);
-    // 5. segmented inclusive scan over the lanes: a lane with a boundary
-    // restarts the running value with its last piece
-    const bool f = mask != 0ull;
-    Acc x = tail;
-    bool ff = f;
+        for (int e = 0; e < B::EL; ++e) {  // fully unrolled: constant register indices and shifts
+          if ((mask >> e) & 1ull) {
+            pieces[np * 32 + lane] = T::finish(PartOf<T>::to_acc(a), aux);
+            ++np;
+            a = PartOf<T>::ident();
+            aux = 0;
+          }
+          bal_fold1<T>(a, aux, bal_elem<T>(cur, e));
+        }
+        const Acc tail = T::finish(PartOf<T>::to_acc(a), aux);
+        // segmented inclusive scan over the lanes: a lane with a boundary
+        // restarts the running value with its last piece
+        const bool f = mask != 0ull;
+        Acc x = tail;
+        bool ff = f;
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const Acc y = shfl_up_v(x, d);
-      const bool fy = __shfl_up_sync(0xffffffffu, ff, d);
-      if (lane >= d) {
-        if (!ff) x = T::comb(y, x);
-        ff = ff || fy;
-      }
-    }
-    const Acc carry = shfl_up_v(x, 1);
-    __syncwarp();
-    if (f) {
-      const Acc head = pieces[lane];
-      const Acc close = lane > 0 ? T::comb(carry, head) : head;
-      if (fb & ((1u << lane) - 1u)) {  // the segment holding element a0 - 1 closes here
-        bal_store<T>(p, (long long)s0 + i0 - 1, T::to_grid(close));
-      } else {                          // the chunk's first boundary: the incoming segment's piece
-        ((Grid*)p.b.first_val)[c] = T::to_grid(close);
-      }
-      int j = i0;
+        for (int d = 1; d < 32; d <<= 1) {
+          const Acc y = shfl_up_v(x, d);
+          const bool fy = __shfl_up_sync(0xffffffffu, ff, d);
+          if (lane >= d) {
+            if (!ff) x = T::comb(y, x);
+            ff = ff || fy;
+          }
+        }
+        const Acc carry_in = shfl_up_v(x, 1);
+        Grid firstv = T::gident();
+        if (f) {
+          const Acc head = pieces[lane];
+          const Acc close = lane > 0 ? T::comb(carry_in, head) : head;
+          if (fb & ((1u << lane) - 1u)) {  // the segment holding element a0 - 1 closes here
+            bal_store<T>(p, (long long)s0 + i0 - 1, T::to_grid(close));
+          } else {                          // the chunk's first boundary: the incoming segment's piece
+            firstv = T::to_grid(close);
+          }
+          int j = i0;
 #pragma unroll 1
-      for (int k = 1; k < np; ++k) {  // segments that start and end in this lane
-        const int o = list[j];
-        while (list[j + 1] == o) ++j;
-        bal_store<T>(p, (long long)s0 + j, T::to_grid(pieces[k * 32 + lane]));
-        ++j;
+          for (int q = 1; q < np; ++q) {  // segments that start and end in this lane
+            const int o = list[j];
+            while (list[j + 1] == o) ++j;
+            bal_store<T>(p, (long long)s0 + j, T::to_grid(pieces[q * 32 + lane]));
+            ++j;
+          }
+        }
+        k.first = shfl_idx_v(firstv, __ffs(fb) - 1);
+        k.last = shfl_idx_v(T::to_grid(x), 31);
+        const long long ls = (long long)s0 + m - 2;  // the segment open at the chunk's end
+        k.last_seg = ls < nseg ? (unsigned)ls : 0xFFFFFFFFu;
+        k.has_b = true;
       }
-    }
-    if (lane == 31) {
-      const long long ls = (long long)s0 + m - 2;  // the segment open at the chunk's end
-      ((Grid*)p.b.last_val)[c] = T::to_grid(x);
-      p.b.flags[c] = 1u;
-      p.b.last_seg[c] = ls < nseg ? (unsigned)ls : 0xFFFFFFFFu;
     }
     __syncwarp();  // pieces / list are rewritten for the next chunk
+    absorb(k);
+    s0 = k.s_next;
+  };
+  if (cb < ce) {
+    s0 = __ldcg(p.b.start_seg + gw);
+    prefetch_list(s0);
+#pragma unroll 1
+    for (long long c = cb; c < ce; ++c) body(c);
+  }
+  if (lane == 0) {  // the range's pieces for the fix-up
+    ((Grid*)p.b.first_val)[gw] = rfirst;
+    ((Grid*)p.b.last_val)[gw] = seen ? carry : rfirst;
+    p.b.flags[gw] = seen ? 1u : 0u;
+    p.b.last_seg[gw] = seen ? carry_seg : 0xFFFFFFFFu;
   }
   pdl_trigger();
 }
 
+// One warp per range whose last piece opens a segment: joins it with the
+// first pieces of the following ranges up to the one where the segment closes
+// (32 ranges per step, fixed order).  The last block resets the call's flags.
 template <int DT, int OP>
 __global__ void __launch_bounds__(256) k_segbal_fix(const SegParams p) {
   using T = Tr<DT, OP>;
-  using B = Bal<T>;
   using Grid = typename T::Grid;
   pdl_wait();
-  const long long nseg = p.nseg;
-  const long long E0 = __ldg(p.offsets), E1 = __ldg(p.offsets + nseg);
   const unsigned nonmono = *(volatile unsigned*)p.b.hdr;
-  const long long P0 = bal_origin<B::s>(p.in, E0);
-  const long long nchunks = E1 > E0 ? (E1 - P0 + B::C - 1) / B::C : 0;
+  const long long nr = p.b.nranges;
   const int lane = threadIdx.x & 31;
-  if (!nonmono && nchunks <= (long long)kBalChunks) {
+  if (!nonmono) {
     const long long nw = (long long)gridDim.x * (blockDim.x >> 5);
     const Grid* fv = (const Grid*)p.b.first_val;
 #pragma unroll 1
-    for (long long c = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); c < nchunks; c += nw) {
+    for (long long c = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); c < nr; c += nw) {
       const unsigned ls = __ldcg(p.b.last_seg + c);
       if (!__ldcg(p.b.flags + c) || ls == 0xFFFFFFFFu) continue;  // warp-uniform
       Grid x = __ldcg((const Grid*)p.b.last_val + c);
@@ -381,7 +465,7 @@ __global__ void __launch_bounds__(256) k_segbal_fix(const SegParams p) {
         const long long k = b0 + lane;
         Grid v = T::gident();
         unsigned kf = 1u;
-        if (k < nchunks) {
+        if (k < nr) {
           v = __ldcg(fv + k);
           kf = __ldcg(p.b.flags + k);
         }
@@ -418,7 +502,7 @@ cudaError_t bal_launch(K kernel, long long grid, int block, size_t smem, const S
 }
 
 template <int DT, int OP>
-cudaError_t launch_segbal_op(const SegParams& p, int sms, cudaStream_t s) {
+cudaError_t launch_segbal_op(const SegParams& p0, int sms, cudaStream_t s) {
   using B = Bal<Tr<DT, OP>>;
   constexpr size_t smem = (size_t)kBalWarps * B::kWarpSmem;
   static int per_sm = 0;
@@ -431,11 +515,15 @@ cudaError_t launch_segbal_op(const SegParams& p, int sms, cudaStream_t s) {
       nb = 1;
     per_sm = nb;
   }
+  SegParams p = p0;
+  long long grid = (long long)sms * per_sm;  // one wave: every warp owns one contiguous chunk range
+  if (grid * kBalWarps > (long long)kBalRanges) grid = kBalRanges / kBalWarps;
+  p.b.nranges = grid * kBalWarps;
   cudaError_t e = bal_launch(k_segbal_scan<DT, OP>, (p.nseg + 255) / 256, 256, 0, p, s);
   if (e != cudaSuccess) return e;
-  e = bal_launch(k_segbal<DT, OP>, (long long)sms * per_sm, kBalWarps * 32, smem, p, s);
+  e = bal_launch(k_segbal<DT, OP>, grid, kBalWarps * 32, smem, p, s);
   if (e != cudaSuccess) return e;
-  return bal_launch(k_segbal_fix<DT, OP>, (long long)sms * 4, 256, 0, p, s);
+  return bal_launch(k_segbal_fix<DT, OP>, (p.b.nranges + 7) / 8, 256, 0, p, s);
 }
 
 template <int DT>

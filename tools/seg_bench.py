@@ -25,6 +25,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--tag", default="")
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--only", default="", help="batched | segmented | histogram (default: all)")
     args = ap.parse_args()
     import numpy as np
     import torch
@@ -40,6 +41,8 @@ def main():
     cols_list = (8, 32, 64, 100, 256, 1024, 16384) if not args.quick else (64, 1024)
     for dtype, op in (("float32", "sum"), ("int32", "sum"), ("float64", "sum"), ("float32", "max"),
                       ("float32", "sum_accurate")):
+        if args.only and args.only != "batched":
+            break
         if args.quick and dtype != "float32":
             continue
         tdt = getattr(torch, dtype)
@@ -57,6 +60,8 @@ def main():
                               "GBps": round(rows * cols * s / sec / 1e9, 1)})
     rng = np.random.Generator(np.random.PCG64(7))
     for dist, mean in (("uniform", 64), ("uniform", 1024), ("powerlaw", 64)):
+        if args.only and args.only != "segmented":
+            break
         nseg = total_bytes // 4 // mean
         if dist == "uniform":
             lens = rng.integers(0, 2 * mean + 1, nseg)
@@ -79,6 +84,8 @@ def main():
     xh = torch.rand(1 << 28, device=dev)
     xi = (xh * 2000 - 1000).to(torch.int32)
     for dtype, t, lo, hi in (("float32", xh, 0.0, 1.0), ("int32", xi, -1000.0, 1001.0)):
+        if args.only and args.only != "histogram":
+            break
         for nbins in (16, 256, 1024, 4096, 16384, 65536):
             if args.quick and nbins not in (256, 65536):
                 continue
