@@ -249,6 +249,19 @@ __device__ __forceinline__ void bal_load_edge(const char* in, long long clo, lon
   }
 }
 
+// The segment holding element chi - 1 (next chunk's list start) when the
+// chunk's offsets slice overflowed the shared list: scan on from `from`.
+__device__ __forceinline__ long long bal_walk_next(const long long* offsets, long long nseg, long long from,
+                                                   long long chi, int lane) {
+#pragma unroll 1
+  for (long long base = from;; base += 32) {
+    const long long idx = base + lane;
+    const long long v = idx <= nseg ? __ldg(offsets + idx) : LLONG_MAX;
+    const unsigned b = __ballot_sync(0xffffffffu, v >= chi);
+    if (b) return base + __ffs(b) - 2;
+  }
+}
+
 template <int DT, int OP>
 __global__ void __launch_bounds__(kBalWarps * 32, 4) k_segbal(const SegParams p) {
   using T = Tr<DT, OP>;
@@ -310,11 +323,18 @@ __global__ void __launch_bounds__(kBalWarps * 32, 4) k_segbal(const SegParams p)
     vfirst = s + lane <= nseg ? __ldg(p.offsets + s + lane) : LLONG_MAX;
     vsecond = s + 32 + lane <= nseg ? __ldg(p.offsets + s + 32 + lane) : LLONG_MAX;
   };
-  auto body = [&](long long c) {
-    const long long clo = P0 + c * B::C, chi = clo + B::C;
-    uint32_t cur[kBalVecsPerLane][8];
+  // the chunk's data: loaded into `cur` as soon as the previous chunk's fold
+  // has consumed it, so the loads fly during that chunk's scan / emission and
+  // this chunk's offsets processing
+  uint32_t cur[kBalVecsPerLane][8];
+  auto load_data = [&](long long c) {
+    if (c >= ce) return;
+    const long long clo = P0 + c * B::C;
     if (interior(c)) bal_load<T>(p.in, clo, lane, cur);
     else bal_load_edge<T>(p.in, clo, E0, E1, lane, cur);
+  };
+  auto body = [&](long long c) {
+    const long long clo = P0 + c * B::C, chi = clo + B::C;
     // the chunk's offsets slice as chunk-local positions: -1 before the
     // chunk, C at / after its end (the first such entry ends the list)
     int m = 0;
@@ -337,16 +357,16 @@ __global__ void __launch_bounds__(kBalWarps * 32, 4) k_segbal(const SegParams p)
     }
     __syncwarp();
     BalChunk<T> k;
-    if (ovf) {
-      k = bal_chunk_walk<T>(p, clo, chi, E0, E1, s0, lane);
-    } else {
-      k.s_next = s0 + m - 2;
-    }
+    k.s_next = s0 + m - 2;
+    if (ovf) k.s_next = bal_walk_next(p.offsets, nseg, s0 + m, chi, lane);
     if (c + 1 < ce) prefetch_list(k.s_next);  // the next chunk's offsets, while this one folds
+    int i0 = 0, np = 0;
+    unsigned long long mask = 0;
+    unsigned fb = 0;
+    Acc tv = T::ident();  // the lane's value (no boundary in the chunk) or its last piece
     if (!ovf) {
       // the lane's boundaries as a bit mask (bit e: a segment starts at element e)
       const int a0 = lane * B::EL;
-      int i0 = 0;
       {
         int hi_i = m - 1;  // list[m - 1] == C > a0
         while (i0 < hi_i) {
@@ -354,23 +374,20 @@ __global__ void __launch_bounds__(kBalWarps * 32, 4) k_segbal(const SegParams p)
           if (list[mid] < a0) i0 = mid + 1; else hi_i = mid;
         }
       }
-      unsigned long long mask = 0;
 #pragma unroll 1
       for (int j = i0; list[j] < a0 + B::EL; ++j) mask |= 1ull << (list[j] - a0);
-      const unsigned fb = __ballot_sync(0xffffffffu, mask != 0ull);
+      fb = __ballot_sync(0xffffffffu, mask != 0ull);
       if (fb == 0u) {  // no boundary in the chunk: plain vector-tree fold
         Part<T> acc[T::NA];
         init_parts<T>(acc);
         uint32_t aux = 0;
 #pragma unroll
         for (int j = 0; j < kBalVecsPerLane; ++j) fold_vec<T>(acc, aux, cur[j], j);
-        k.first = T::to_grid(T::warp(thread_result<T>(acc, aux)));
-        k.has_b = false;
+        tv = thread_result<T>(acc, aux);
       } else {
         // fold element by element, closing a piece at every boundary
         Part<T> a = PartOf<T>::ident();
         uint32_t aux = 0;
-        int np = 0;
 #pragma unroll
         for (int e = 0; e < B::EL; ++e) {  // fully unrolled: constant register indices and shifts
           if ((mask >> e) & 1ull) {
@@ -381,11 +398,23 @@ __global__ void __launch_bounds__(kBalWarps * 32, 4) k_segbal(const SegParams p)
           }
           bal_fold1<T>(a, aux, bal_elem<T>(cur, e));
         }
-        const Acc tail = T::finish(PartOf<T>::to_acc(a), aux);
+        tv = T::finish(PartOf<T>::to_acc(a), aux);
+      }
+    }
+    load_data(c + 1);  // `cur` is consumed: the next chunk's loads fly from here
+    if (ovf) {
+      const long long sn = k.s_next;
+      k = bal_chunk_walk<T>(p, clo, chi, E0, E1, s0, lane);
+      k.s_next = sn;
+    } else if (fb == 0u) {
+      k.first = T::to_grid(T::warp(tv));
+      k.has_b = false;
+    } else {
+      {
         // segmented inclusive scan over the lanes: a lane with a boundary
         // restarts the running value with its last piece
         const bool f = mask != 0ull;
-        Acc x = tail;
+        Acc x = tv;
         bool ff = f;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
@@ -429,6 +458,7 @@ __global__ void __launch_bounds__(kBalWarps * 32, 4) k_segbal(const SegParams p)
   if (cb < ce) {
     s0 = __ldcg(p.b.start_seg + gw);
     prefetch_list(s0);
+    load_data(cb);
 #pragma unroll 1
     for (long long c = cb; c < ce; ++c) body(c);
   }
