@@ -682,6 +682,32 @@ def main():
                             "arrays_per_s": round(rows / sec, 1),
                             "speedup_vs_one_reduce_per_array": None if one is None else round(one * 1e-6 * rows / sec, 1)})
 
+    # ---- variable-length segments through an offsets array (N1, the
+    # element-balanced chunk kernels): 256 MB of the resident input cut into
+    # power-law (mean 64) and uniform (0..128, 0..2048) lengths, seeded
+    segmented = None
+    if not args.no_sweep and world == 1:
+        segmented = []
+        rng_s = np.random.Generator(np.random.PCG64(2019 + 1000 * 6))
+        total = (256 << 20) // 4
+        for dist_s, mean in (("powerlaw", 64), ("uniform", 64), ("uniform", 1024)):
+            nseg = total // mean
+            if dist_s == "uniform":
+                lens = rng_s.integers(0, 2 * mean + 1, nseg)
+            else:
+                lens = np.minimum((rng_s.pareto(1.2, nseg) * mean * 0.2).astype(np.int64) + 1, 1 << 20)
+            offs = np.minimum(np.concatenate([[0], np.cumsum(lens)]), total)
+            ot = torch.from_numpy(offs).to(dev)
+            xs = x[: int(offs[-1])]
+            ob = torch.empty(nseg, dtype=torch.float32, device=dev)
+
+            def launch_s(t, ob=ob, xs=xs, ot=ot):
+                rb.reduce_segmented(xs, ot, "sum", out=ob, stream=stream)
+            sec = time_calls(launch_s, [xs] * 3, [xs] * 10, stream, repeats=2)
+            segmented.append({"lengths": f"{dist_s} mean {mean}", "segments": nseg, "elements": int(offs[-1]),
+                              "us": round(sec * 1e6, 2), "GBps": round(int(offs[-1]) * 4 / sec / 1e9, 1),
+                              "segments_per_s": round(nseg / sec, 1)})
+
     # ---- CPU baseline: the oracle on the host cores (rank 0, N = 1)
     cpu = None
     if not args.no_cpu and world == 1 and rank == 0:
@@ -735,6 +761,7 @@ def main():
             line["sweep"] = sweep
             line["small_array_latency"] = latency
             line["batched"] = batched
+            line["segmented"] = segmented
             line["ops_1GiB"] = ops_1gib
             line["histogram"] = hist
             line["config5_8GiB_one_gpu"] = big

@@ -132,12 +132,18 @@ typedef struct {
                          for REDUCE_GC_CLUSTER: the cluster size, 1..16 (0 = 16) */
   int seg_group;      /* reduce_segmented / reduce_batched only: 0 = auto (uniform
                          rows: one thread per row up to 512 bytes, 8 lanes up to 4 KB,
-                         one warp up to 16 KB, else one block; offset arrays: 8 lanes),
-                         1 = one warp per segment, 2 = one block per segment,
-                         3 = 8 lanes, 4 = one thread.  Segments much longer than
-                         their group's first round (offset arrays; or fewer than 4096
-                         uniform rows of > 64 KB) are cut into chunks of >= 16 KB that
-                         warps reduce (two more launches; load balance) */
+                         one warp up to 16 KB, else one block; offset arrays: the
+                         element-balanced chunks of 5), 1 = one warp per segment,
+                         2 = one block per segment, 3 = 8 lanes, 4 = one thread,
+                         5 = element-balanced (offset arrays only): the elements are
+                         cut into 8 KB chunks, each warp of a one-wave grid reduces a
+                         contiguous range of chunks whatever the segment lengths, and
+                         the segments crossing ranges are joined by a fix-up kernel
+                         (3 launches; non-monotone offsets fall back to one warp per
+                         segment inside the same launches).  For groups 1-4, segments
+                         much longer than their group's first round (offset arrays; or
+                         fewer than 4096 uniform rows of > 64 KB) are cut into chunks
+                         of >= 16 KB that warps reduce (two more launches) */
   int stage;          /* 0 = auto; REDUCE_STAGE_REG: 256-bit loads straight into
                          registers; REDUCE_STAGE_SMEM: cp.async 16-byte copies into a
                          shared-memory tile (block*unroll*32 <= 128 KiB), then shared
@@ -195,14 +201,20 @@ int reduce_host(int dtype, int op, const void* host_in, size_t n, void* host_out
  * i < num_segments.  `offsets` is a DEVICE array of num_segments + 1 int64
  * element offsets (non-decreasing; a decreasing pair is treated as an empty
  * segment, which yields the identity); `out` is a DEVICE array of
- * num_segments elements of dtype.  One thread, 8 lanes, one warp or one block
- * per segment (the paper's small-array versions assign one warp / block per
- * partition with no global atomics); segments much longer than
- * their group's first round are cut into chunks of >= 16 KB that warps
- * reduce, then combined in chunk order (the stream's workspace holds the
- * queue; two more launches; load balance for skewed lengths).  Values never touch
- * atomics and every combine has a fixed order: deterministic.  Up to 3
- * launches (1 for uniform rows too short to be cut).  Segment starts may have
+ * num_segments elements of dtype.  Offset arrays are reduced element-balanced
+ * by default (seg_group 5: fixed 8 KB chunks of the flat element range, the
+ * tiled partition of Fig. 1(b), with the segment boundaries carried
+ * through it -- the time no longer depends on the length distribution);
+ * the other groups give one thread, 8 lanes, one warp or one block per
+ * segment (the paper's small-array versions assign one warp / block per
+ * partition with no global atomics), and there segments much
+ * longer than their group's first round are cut into chunks of >= 16 KB that
+ * warps reduce, then combined in chunk order (the stream's workspace holds the
+ * queue; two more launches).  Values never touch atomics and every combine
+ * has a fixed order: deterministic.  Up to 3 launches (1 for uniform rows too
+ * short to be cut).  num_segments must be < 2^32 - 1 for the balanced path
+ * (else 8 lanes).  A graph capture needs reduce_prepare on the stream first
+ * (the chunk arrays; without it the capture runs the group kernels).  Segment starts may have
  * any element alignment.  Options used: block (32..512, default 256), seg_group.  reduce_batched is the uniform case: num_segments rows of seg_len
  * contiguous elements (row i at in + i*seg_len), no offsets array. */
 int reduce_segmented(int dtype, int op, const void* in, const int64_t* offsets, size_t num_segments, void* out,

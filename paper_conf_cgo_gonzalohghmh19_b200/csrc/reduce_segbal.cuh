@@ -147,8 +147,10 @@ __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
       const long long c0 = lo <= E0 ? 0 : (lo - P0 + B::C - 1) / B::C;
       long long c1 = (hi - P0 + B::C - 1) / B::C;
       if (c1 > nchunks) c1 = nchunks;
-      const BalRanges R(nchunks, p.b.nranges);
-      for (long long w = R.first_at(c0); w < p.b.nranges && R.begin(w) < c1; ++w) p.b.start_seg[w] = (unsigned)i;
+      if (c0 < c1) {  // only segments holding a chunk start (the range arithmetic divides)
+        const BalRanges R(nchunks, p.b.nranges);
+        for (long long w = R.first_at(c0); w < p.b.nranges && R.begin(w) < c1; ++w) p.b.start_seg[w] = (unsigned)i;
+      }
     }
   }
   pdl_trigger();
