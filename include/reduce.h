@@ -136,7 +136,7 @@ typedef struct {
                          element-balanced chunks of 5), 1 = one warp per segment,
                          2 = one block per segment, 3 = 8 lanes, 4 = one thread,
                          5 = element-balanced (offset arrays only): the elements are
-                         cut into 8 KB chunks, each warp of a one-wave grid reduces a
+                         cut into 4 KB chunks, each warp of a one-wave grid reduces a
                          contiguous range of chunks whatever the segment lengths, and
                          the segments crossing ranges are joined by a fix-up kernel
                          (3 launches; non-monotone offsets fall back to one warp per
@@ -202,7 +202,7 @@ int reduce_host(int dtype, int op, const void* host_in, size_t n, void* host_out
  * element offsets (non-decreasing; a decreasing pair is treated as an empty
  * segment, which yields the identity); `out` is a DEVICE array of
  * num_segments elements of dtype.  Offset arrays are reduced element-balanced
- * by default (seg_group 5: fixed 8 KB chunks of the flat element range, the
+ * by default (seg_group 5: fixed 4 KB chunks of the flat element range, the
  * tiled partition of Fig. 1(b), with the segment boundaries carried
  * through it -- the time no longer depends on the length distribution);
  * the other groups give one thread, 8 lanes, one warp or one block per

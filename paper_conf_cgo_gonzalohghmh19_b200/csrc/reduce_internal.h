@@ -105,7 +105,7 @@ inline SegQueue seg_queue_at(char* base) {
 }
 
 // Element-balanced segmented reduction of an offsets array (reduce_segbal.cuh):
-// the elements are cut into fixed 8 KB chunks and every warp of a one-wave
+// the elements are cut into fixed 4 KB chunks and every warp of a one-wave
 // grid reduces one contiguous range of chunks whatever the segment lengths;
 // the pieces of segments that cross ranges are joined by a fix-up pass.
 constexpr unsigned kBalRanges = 1u << 16;  // capacity of the per-range arrays (ranges = chunk-kernel warps)

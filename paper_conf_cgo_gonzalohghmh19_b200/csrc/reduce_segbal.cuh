@@ -6,33 +6,41 @@
 // the grid waits for the few groups that drew long segments, and each short
 // segment costs a chain of dependent loads (offsets -> data -> store).  Here
 // the ELEMENTS are split evenly instead: the flat range [offsets[0],
-// offsets[nseg]) is cut into 8 KB chunks on 32-byte boundaries and one warp
+// offsets[nseg]) is cut into 4 KB chunks on 32-byte boundaries and one warp
 // reduces one chunk whatever the segments inside it look like -- the
 // partition is by data, as the paper's tiled distribution of a single array
 // (Fig. 1(b)), with segment boundaries carried inside it.
 //
 //   k_segbal_scan : one thread per segment: the identity for empty segments,
-//                   start_seg[c] = the segment holding chunk c's first element,
-//                   and a flag if the offsets are not monotone (then the chunk
-//                   kernel falls back to one warp per segment).
-//   k_segbal      : one warp per chunk.  Lane l owns the chunk's 256 bytes
-//                   [256 l, 256 l + 256) (eight 32-byte loads in flight).  The
-//                   chunk's slice of the offsets array is copied into shared
-//                   memory as chunk-local positions; each lane turns the
-//                   boundaries in its range into a 64-bit mask, folds its
-//                   elements in order, closing a piece at every set bit
-//                   (pieces go to shared memory).  A segmented scan over the
-//                   32 lanes (5 shuffle steps, fixed order) joins the pieces of
-//                   segments that cross lanes.  Segments that start and end in
-//                   the chunk are written directly; the chunk leaves its first
-//                   piece (the segment that began before it) and its last piece
-//                   (the segment still open at its end) for the fix-up.  A chunk
-//                   without boundaries folds with the plain vector tree.
-//   k_segbal_fix  : one warp per chunk whose last piece opens a segment: joins
-//                   it with the first pieces of the following chunks up to the
-//                   chunk where the segment closes (32 chunks per step, fixed
+//                   a flag if the offsets are not monotone (then the chunk
+//                   kernel falls back to one warp per segment), and for every
+//                   chunk range the segment holding its first element.
+//   k_segbal      : a one-wave grid; warp w owns a contiguous range of chunks
+//                   and carries the segment still open from one chunk to the
+//                   next.  Per chunk, lane l owns the chunk's 128 bytes
+//                   [128 l, 128 l + 128) (four 32-byte loads, issued as soon
+//                   as the previous chunk's fold has consumed its data).  The
+//                   chunk's slice of the offsets array (its first 64 entries
+//                   prefetched) is copied into shared memory as chunk-local
+//                   positions; each lane turns the boundaries in its range
+//                   into a bit mask, folds its elements in order, closing a
+//                   piece at every set bit (pieces go to shared memory).  A
+//                   segmented scan over the 32 lanes (5 shuffle steps, fixed
+//                   order) joins the pieces of segments that cross lanes.
+//                   Segments that start and end in the chunk are written
+//                   directly.  A chunk without boundaries folds with the plain
+//                   vector tree.  The range leaves its first piece (the
+//                   segment open at its start) and its last (the segment
+//                   open at its end) for the fix-up.
+//   k_segbal_fix  : one warp per range whose last piece opens a segment: joins
+//                   it with the first pieces of the following ranges up to the
+//                   range where the segment closes (32 ranges per step, fixed
 //                   order), writes out[segment], and the last block resets the
 //                   call's flags.
+// Chunk size: 4 KB (4 vectors per lane, 96 registers, 20 resident warps per
+// SM) measured 15-17 % faster than 8 KB (128 registers, 16 warps): the chunk
+// kernel is bound by its per-chunk instruction chain, so resident warps beat
+// bytes per warp (profiles/r01_segbal_ab.txt).
 // Values never touch atomics and every combine order depends only on the
 // offsets: deterministic.  Chunk geometry depends only on the input address
 // modulo 32 and offsets[0].
@@ -42,15 +50,25 @@
 
 namespace rb {
 
-constexpr int kBalWarps = 4;        // warps per block of k_segbal
-constexpr int kBalVecsPerLane = 8;  // 32-byte vectors per lane per chunk (256 contiguous bytes)
+// Launch shape (A/B hooks: REDUCE_B200_NVCC_FLAGS="-DRB_SEGBAL_VPL=4 ...").
+#ifndef RB_SEGBAL_VPL
+#define RB_SEGBAL_VPL 4
+#endif
+#ifndef RB_SEGBAL_MINB
+#define RB_SEGBAL_MINB 5
+#endif
+constexpr int kBalWarps = 4;                    // warps per block of k_segbal
+// resident blocks asked of ptxas: 5 (96 registers, 20 warps per SM) for the
+// 4-byte plain ops; fp64 and accurate sums need more registers (4 blocks)
+constexpr int bal_min_blocks(int dt, int op) { return (dt != 2 && op != 3) ? RB_SEGBAL_MINB : 4; }
+constexpr int kBalVecsPerLane = RB_SEGBAL_VPL;  // 32-byte vectors per lane per chunk (256 contiguous bytes)
 
 template <class T>
 struct Bal {
   using Acc = typename T::Acc;
   static constexpr int s = sizeof(typename T::Elem);
   static constexpr int EL = kBalVecsPerLane * T::VE;  // elements per lane (64 or 32)
-  static constexpr long long C = 32LL * EL;           // elements per chunk (8 KB)
+  static constexpr long long C = 32LL * EL;           // elements per chunk (32 lanes x kBalVecsPerLane x 32 B = 4 KB)
   static constexpr int kList = (int)C + 64;           // offsets entries kept in shared memory
   static constexpr size_t kPieceBytes = (size_t)EL * 32 * sizeof(Acc);
   static constexpr size_t kListBytes = ((size_t)kList * 2 + 15) / 16 * 16;
@@ -265,7 +283,7 @@ __device__ __forceinline__ long long bal_walk_next(const long long* offsets, lon
 }
 
 template <int DT, int OP>
-__global__ void __launch_bounds__(kBalWarps * 32, 4) k_segbal(const SegParams p) {
+__global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segbal(const SegParams p) {
   using T = Tr<DT, OP>;
   using B = Bal<T>;
   using Acc = typename T::Acc;

@@ -3,7 +3,7 @@ csrc/reduce_segbal.cuh) against the oracle applied to every
 segment: bit-exact for int32 and min/max, G1 + G2 for fp sums.
 
 The cases aim at the chunk machinery: segments shorter than a lane, longer
-than a chunk (8 KB) and spanning hundreds of chunks, boundaries exactly on
+than a chunk (4 KB) and spanning hundreds of chunks, boundaries exactly on
 lane / chunk edges, runs of empty segments (including more than a chunk's
 offsets list holds: the walk path), offsets[0] > 0 and offsets[-1] < len(x),
 every input misalignment, non-monotone offsets (the per-segment fallback) and
@@ -101,7 +101,7 @@ def test_length_regimes(dtype, kind):
     """lengths around the lane (8 vectors) and chunk (8 KB) sizes, so
     boundaries fall on lane and chunk edges and pieces cross both"""
     rng = np.random.Generator(np.random.PCG64(KINDS.index(kind)))
-    el = 32 if dtype == "float64" else 64
+    el = 16 if dtype == "float64" else 32  # elements per lane (4 x 32 bytes); chunk = 32 lanes = 4 KB
     c = 32 * el
     if kind == "ones":
         lens = np.ones(30000, np.int64)

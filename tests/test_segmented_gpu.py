@@ -20,8 +20,8 @@ def _chain(length, dtype, lanes):
     # per-thread: m vectors through a lane tree (depth log2 VE) into 2 accumulators
     # (or one accumulator per lane), + head/tail, + merge; then group / block combines
     ve = 4 if dtype == "float64" else 8
-    if lanes < 0:  # element-balanced chunks: <= 8*VE elements in order per lane, lane scan,
-        el = 8 * ve  # then the chunk pieces joined 32 at a time by warp butterflies
+    if lanes < 0:  # element-balanced chunks: <= 4*VE elements in order per lane, lane scan,
+        el = 4 * ve  # then the chunk pieces joined 32 at a time by warp butterflies
         return min(length, el) + 1 + 5 + 1 + math.ceil(math.ceil(length / (32 * el) + 1) / 32) * 6 + 2
     m = math.ceil(length / (ve * lanes))
     return m + int(math.log2(ve)) + 3 + 5 + (5 if lanes > 32 else 0)
