@@ -150,18 +150,20 @@ __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
   using T = Tr<DT, OP>;
   using B = Bal<T>;
   pdl_wait();
-  const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < p.nseg) {
-    const long long E0 = __ldg(p.offsets), E1 = __ldg(p.offsets + p.nseg);
+  // one-wave grid striding over the segments (the per-call geometry once per thread)
+  const long long E0 = __ldg(p.offsets), E1 = __ldg(p.offsets + p.nseg);
+  const long long P0 = bal_origin<B::s>(p.in, E0);
+  const long long nchunks = E1 > E0 ? (E1 - P0 + B::C - 1) / B::C : 0;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+#pragma unroll 1
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < p.nseg; i += stride) {
     const long long lo = __ldg(p.offsets + i), hi = __ldg(p.offsets + i + 1);
     if (hi < lo) atomicOr(p.b.hdr, 1u);
     if (hi <= lo) {
       seg_store<T>(p, i, T::gident());
-    } else if (E1 > E0) {
+    } else if (nchunks > 0) {
       // start_seg[w] = i for the ranges whose first chunk starts in [lo, hi)
       // (chunk 0 starts at E0, chunk c > 0 at P0 + c*C)
-      const long long P0 = bal_origin<B::s>(p.in, E0);
-      const long long nchunks = (E1 - P0 + B::C - 1) / B::C;
       const long long c0 = lo <= E0 ? 0 : (lo - P0 + B::C - 1) / B::C;
       long long c1 = (hi - P0 + B::C - 1) / B::C;
       if (c1 > nchunks) c1 = nchunks;
@@ -507,17 +509,28 @@ __global__ void __launch_bounds__(256) k_segbal_fix(const SegParams p) {
     const Grid* fv = (const Grid*)p.b.first_val;
 #pragma unroll 1
     for (long long c = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); c < nr; c += nw) {
-      const unsigned ls = __ldcg(p.b.last_seg + c);
-      if (!__ldcg(p.b.flags + c) || ls == 0xFFFFFFFFu) continue;  // warp-uniform
+      // this range's words and the first batch of the following ranges' in
+      // one round of loads (most segments close in the next range)
+      const unsigned ls = __ldcg(p.b.last_seg + c), fc = __ldcg(p.b.flags + c);
       Grid x = __ldcg((const Grid*)p.b.last_val + c);
+      long long k = c + 1 + lane;
+      Grid v = T::gident();
+      unsigned kf = 1u;
+      if (k < nr) {
+        v = __ldcg(fv + k);
+        kf = __ldcg(p.b.flags + k);
+      }
+      if (!fc || ls == 0xFFFFFFFFu) continue;  // warp-uniform
 #pragma unroll 1
       for (long long b0 = c + 1;; b0 += 32) {
-        const long long k = b0 + lane;
-        Grid v = T::gident();
-        unsigned kf = 1u;
-        if (k < nr) {
-          v = __ldcg(fv + k);
-          kf = __ldcg(p.b.flags + k);
+        if (b0 != c + 1) {
+          k = b0 + lane;
+          v = T::gident();
+          kf = 1u;
+          if (k < nr) {
+            v = __ldcg(fv + k);
+            kf = __ldcg(p.b.flags + k);
+          }
         }
         const unsigned bal = __ballot_sync(0xffffffffu, kf != 0u);
         const int stop = bal ? __ffs(bal) - 1 : 32;
@@ -569,7 +582,9 @@ cudaError_t launch_segbal_op(const SegParams& p0, int sms, cudaStream_t s) {
   long long grid = (long long)sms * per_sm;  // one wave: every warp owns one contiguous chunk range
   if (grid * kBalWarps > (long long)kBalRanges) grid = kBalRanges / kBalWarps;
   p.b.nranges = grid * kBalWarps;
-  cudaError_t e = bal_launch(k_segbal_scan<DT, OP>, (p.nseg + 255) / 256, 256, 0, p, s);
+  long long sgrid = (p.nseg + 255) / 256;
+  if (sgrid > (long long)sms * 8) sgrid = (long long)sms * 8;
+  cudaError_t e = bal_launch(k_segbal_scan<DT, OP>, sgrid, 256, 0, p, s);
   if (e != cudaSuccess) return e;
   e = bal_launch(k_segbal<DT, OP>, grid, kBalWarps * 32, smem, p, s);
   if (e != cudaSuccess) return e;
