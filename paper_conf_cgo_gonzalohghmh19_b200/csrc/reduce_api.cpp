@@ -3,6 +3,7 @@
 // Every step of the reduction itself runs in the CUDA kernels; there is no
 // host or CPU fallback anywhere in this library.
 #include <atomic>
+#include <climits>
 #include <cmath>
 #include <cstring>
 #include <map>
@@ -519,8 +520,25 @@ int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, 
     p.hi_i = (long long)hi;
     p.range_i = (unsigned long long)(p.hi_i - p.lo_i);
     p.magic = ~0ull / p.range_i;
-    p.narrow = (unsigned long long)p.range_i * (unsigned long long)nbins < (1ull << 32) ? 1 : 0;
-    p.magic32 = p.narrow ? (unsigned)(0xFFFFFFFFull / p.range_i) : 0u;
+    const long long lo_c = p.lo_i > (long long)INT32_MIN ? p.lo_i : (long long)INT32_MIN;
+    const long long hi_c = p.hi_i < (long long)INT32_MAX + 1 ? p.hi_i : (long long)INT32_MAX + 1;
+    p.narrow = ((unsigned long long)p.range_i * (unsigned long long)nbins < (1ull << 32) && hi_c > lo_c) ? 1 : 0;
+    // q = (t + ((n - t) >> 1)) >> shift32, t = umulhi(n, magic32): with
+    // l = ceil(log2 d), magic32 = floor(2^32 (2^l - d) / d) + 1, shift32 = l - 1
+    // (Granlund & Montgomery 1994, fig. 4.1).  d = 1: every counted element
+    // has n = 0, which the zero multiplier maps to 0.
+    p.magic32 = 0u;
+    p.shift32 = 0;
+    if (p.narrow && p.range_i > 1) {
+      int l = 0;
+      while ((1ull << l) < p.range_i) ++l;
+      const unsigned __int128 num = ((unsigned __int128)1 << 32) * ((1ull << l) - p.range_i);
+      p.magic32 = (unsigned)(num / p.range_i + 1);
+      p.shift32 = l - 1;
+    }
+    p.lo_c32 = (unsigned)(long long)lo_c;
+    p.lim32 = p.narrow ? (unsigned)(hi_c - 1 - lo_c) : 0u;
+    p.lo32 = (unsigned)p.lo_i;
   } else {
     p.lo_f = (float)lo;
     p.hi_f = (float)hi;

@@ -7,9 +7,11 @@
 //   counts[b] = #{ i : lo <= x_i < hi, b = floor((x_i - lo) * nbins / (hi - lo)) }
 //
 // Bins are decided in the input's own arithmetic -- the same rule as the oracle
-// (reading R13): int32 exactly, with a 64-bit numerator divided by
-// multiply-high with a precomputed reciprocal plus a correction step (no
-// integer division instruction); fp32 with two correctly rounded fp32
+// (reading R13): int32 exactly -- when (hi - lo) * nbins < 2^32 a
+// 32-bit range check and numerator divided by the Granlund-Montgomery
+// multiply-high sequence (exact, no correction), else a 64-bit numerator
+// divided by multiply-high plus a correction step (no integer division
+// instruction either way); fp32 with two correctly rounded fp32
 // operations, floor(fl(fl(x - lo) * scale)) (__fsub_rn / __fmul_rn: never
 // contracted into an FMA).  The B200's FP64 pipe is far too slow for a
 // per-element fp64 rule at HBM speed (measured 2.5 TB/s).  A persistent grid (one wave) streams 32-byte
@@ -33,19 +35,18 @@ constexpr int kHistSharedMaxBins = 16384;  // 64 KB of u32 counters per block
 template <int DT>
 __device__ __forceinline__ int hist_bin(uint32_t w, const HistParams& p) {
   if constexpr (DT == DT_I32) {
+    if (p.narrow) {  // (hi - lo) * nbins < 2^32: range check and quotient in 32-bit arithmetic
+      // int32 range check against the clamped bounds: one subtract, one unsigned compare
+      const bool in = w - p.lo_c32 <= p.lim32;
+      const unsigned num = (w - p.lo32) * (unsigned)p.nbins;  // x - lo is exact mod 2^32 when counted
+      const unsigned t = __umulhi(num, p.magic32);            // exact floor(num / range): no correction
+      const unsigned q = (t + ((num - t) >> 1)) >> p.shift32;
+      return in ? (int)q : -1;
+    }
     const long long v = (long long)(int32_t)w;
     const bool in = v >= p.lo_i && v < p.hi_i;
     int b;
-    if (p.narrow) {  // (hi - lo) * nbins < 2^32: the quotient in 32-bit arithmetic
-      const unsigned range = (unsigned)p.range_i;
-      const unsigned num = (unsigned)(v - p.lo_i) * (unsigned)p.nbins;
-      unsigned q = __umulhi(num, p.magic32);
-      unsigned r = num - q * range;
-      // q underestimates floor(num / range) by at most 2
-      if (r >= range) { ++q; r -= range; }
-      if (r >= range) ++q;
-      b = (int)q;
-    } else {
+    {
       const unsigned long long num = (unsigned long long)(v - p.lo_i) * (unsigned long long)p.nbins;
       unsigned long long q = __umul64hi(num, p.magic);
       unsigned long long r = num - q * p.range_i;

@@ -160,8 +160,13 @@ struct HistParams {
   long long lo_i, hi_i;         // int32 input: integer bounds
   unsigned long long range_i;   //   hi_i - lo_i
   unsigned long long magic;     //   floor((2^64 - 1) / range_i): quotient by multiply-high
-  unsigned magic32;             //   floor((2^32 - 1) / range_i) when narrow
-  int narrow;                   //   range_i * nbins < 2^32: 32-bit quotient
+  unsigned magic32;             //   narrow: Granlund-Montgomery multiplier of range_i (exact
+  int shift32;                  //   floor(n / range_i) for every 32-bit n, no correction step)
+  int narrow;                   //   range_i * nbins < 2^32 (and [lo, hi) meets the int32 range):
+                                //   32-bit range check and quotient
+  unsigned lo_c32, lim32;       //   narrow: counted iff (uint32)(x - lo_c32) <= lim32, with [lo_c, hi_c)
+                                //   = [lo, hi) clamped to the int32 range, lim32 = hi_c - 1 - lo_c
+  unsigned lo32;                //   narrow: (uint32)lo_i (x - lo mod 2^32 is exact for counted x)
   float lo_f, hi_f, scale_f;    // fp32 input: (float)lo, (float)hi, (float)(nbins / (hi - lo))
   int nbins;
   unsigned* counts;             // device, nbins

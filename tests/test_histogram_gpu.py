@@ -52,13 +52,27 @@ def test_histogram_special_values_and_big():
     (-65536.0, 65537.0, 65535),           # range * nbins just above 2^32
     (-65536.0, 0.0, 65535),               # range * nbins just below 2^32: 32-bit path
     (0.0, 3.0, 3),                        # one bin per value
+    (5.0, 6.0, 1),                        # range 1 (the zero multiplier)
+    (5.0, 6.0, 3),                        # range 1, more bins than values
+    (-512.0, 512.0, 64),                  # power-of-two range (multiplier 1)
+    (-513.0, 512.0, 64),                  # 2^k + 1
+    (-511.0, 512.0, 1000),                # 2^k - 1, range * nbins near 2^20
+    (-40000.0, 67000.0, 40000),           # range * nbins just below 2^32, odd divisor
+    (2.0 ** 31 - 10, 2.0 ** 31 + 10, 4),  # narrow, hi above INT32_MAX: clamped 32-bit range check
+    (-2.0 ** 31 - 10, -2.0 ** 31 + 10, 3),  # narrow, lo below INT32_MIN
+    (2.0 ** 31 + 5, 2.0 ** 31 + 100, 7),  # entirely above the int32 range: nothing counted
+    (-2.0 ** 32, -2.0 ** 31 - 1, 2),      # entirely below
 ])
 def test_histogram_int32_wide_ranges(lo, hi, nbins):
     rb = _rb()
     x = synth.make("int32", (1 << 20) + 11, "int_full", 77)
     x[:6] = [np.iinfo(np.int32).min, np.iinfo(np.int32).max, 0, -1, 1, 2]
+    edge = np.arange(-12, 12, dtype=np.int64)  # values next to both ends of the int32 range
+    x[1000:1024] = (edge + 2 ** 31).astype(np.int64).clip(-2 ** 31, 2 ** 31 - 1).astype(np.int32)
+    x[2000:2024] = (edge - 2 ** 31).clip(-2 ** 31, 2 ** 31 - 1).astype(np.int32)
     if hi - lo < 2 ** 20:
-        x[7::3] = (x[7::3] % int(2 * (hi - lo))) + int(lo) - int((hi - lo) // 2)
+        y = (x[7::3].astype(np.int64) % int(2 * (hi - lo))) + int(lo) - int((hi - lo) // 2)
+        x[7::3] = y.clip(-2 ** 31, 2 ** 31 - 1).astype(np.int32)
     t = to_device(x, 5)
     got = rb.histogram(t, lo, hi, nbins).cpu().numpy().view(np.uint32)
     want = oracle.histogram(x, lo, hi, nbins)
