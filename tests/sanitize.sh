@@ -28,6 +28,16 @@ for dt in (torch.int32, torch.float32, torch.float64):
     # a decreasing pair, and few long uniform rows (queued too)
     loffs = torch.tensor([0, 5, 70005, 70006, 60000, 150003, 150040], dtype=torch.int64, device="cuda")
     lbase = torch.arange(150050, device="cuda").to(dt)[3:]
+    # element-balanced path (seg_group 0 / 5): monotone offsets with segments
+    # crossing lanes, chunks and warp ranges, a run of 3000 empty segments (the
+    # per-piece walk) and a window not starting at element 0
+    rng = np.random.Generator(np.random.PCG64(3))
+    lens = np.minimum((rng.pareto(1.2, 6000) * 8).astype(np.int64) + 1, 60000)
+    lens[2000:5000] = 0
+    moffs = torch.from_numpy(np.concatenate([[7], 7 + np.cumsum(lens)])).to("cuda")
+    mbase = torch.arange(int(moffs[-1]) + 16, device="cuda").to(dt)[1:]
+    for op in ("sum", "min", "max") + (("sum_accurate",) if dt != torch.int32 else ()):
+        rb.reduce_segmented(mbase, moffs, op, seg_group=5)
     for g in (0, 1, 2, 3, 4):
         rb.reduce_segmented(base, offs, "sum", seg_group=g)
         rb.reduce_batched(base[:4096].view(64, 64), "max", seg_group=g)
@@ -38,6 +48,10 @@ for dt in (torch.int32, torch.float32, torch.float64):
     if dt != torch.float64:
         for nb in (7, 256, 4096, 20000, 1 << 20):
             rb.histogram(base, 0, 4000, nb)
+        if dt == torch.int32:  # both int32 quotient paths and clamped bounds
+            rb.histogram(base, -2.0 ** 31, 2.0 ** 31, 1000)
+            rb.histogram(base, 2.0 ** 31 - 10, 2.0 ** 31 + 10, 4)
+            rb.histogram(base, 5, 6, 3)
         if dt == torch.int32:
             rb.histogram(base, -2.0 ** 31, 2.0 ** 31, 1000)  # 64-bit quotient path
 # team combine (k = 1: members on one GPU cannot run concurrently under the
