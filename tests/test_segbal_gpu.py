@@ -213,3 +213,54 @@ def test_matches_group_kernels_exactly_for_ints():
     for op in ("sum", "min", "max"):
         outs = {rb.reduce_segmented(xt, ot, op, seg_group=g).cpu().numpy().tobytes() for g in (0, 1, 2, 3, 4, 5)}
         assert len(outs) == 1, op
+
+
+def _reduceat(x, offs, op):
+    """numpy reference per segment (vectorised; empty segments -> identity)."""
+    lo = offs[:-1]
+    empty = offs[1:] <= lo
+    idx = np.minimum(lo, max(x.size - 1, 0))
+    if op == "sum":
+        r = np.add.reduceat(x.astype(np.int64 if x.dtype == np.int32 else np.float64), idx)
+        r[empty] = 0
+        return r
+    f = np.minimum if op == "min" else np.maximum
+    r = f.reduceat(x, idx)
+    ident = {"min": np.iinfo(np.int32).max, "max": np.iinfo(np.int32).min} if x.dtype == np.int32 else \
+        {"min": np.inf, "max": -np.inf}
+    r[empty] = ident[op]
+    return r
+
+
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+def test_bench_workload_full_size(dtype):
+    """bench.py's `segmented` workload at full size (1 M power-law segments over
+    ~60 M elements, the launch the bench times): int32 sums (mod 2^32), int32 /
+    fp32 min and max bit-exact against numpy reduceat; fp32 sums within the
+    G2 gate per segment ((L + 1) u sum|x|, L the balanced chain)."""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    rng = np.random.Generator(np.random.PCG64(2019 + 1000 * 6))
+    total = (256 << 20) // 4
+    nseg = total // 64
+    lens = np.minimum((rng.pareto(1.2, nseg) * 64 * 0.2).astype(np.int64) + 1, 1 << 20)
+    offs = np.minimum(np.concatenate([[0], np.cumsum(lens)]), total)
+    n = int(offs[-1])
+    x = synth.make(dtype, n, "int_full" if dtype == "int32" else "uniform01", 66)
+    xt, ot = torch.from_numpy(x).cuda(), torch.from_numpy(offs).cuda()
+    for op in ("sum", "min", "max"):
+        got = rb.reduce_segmented(xt, ot, op).cpu().numpy()
+        want = _reduceat(x, offs, op)
+        if dtype == "int32" and op == "sum":
+            want = ((want + 2 ** 31) % 2 ** 32 - 2 ** 31).astype(np.int32)
+            assert (got == want).all(), np.nonzero(got != want)[0][:5]
+        elif op == "sum":
+            lens_ = np.diff(offs)
+            absum = np.abs(want)  # uniform01: all terms >= 0, sum|x| = sum
+            el = 32
+            chain = np.minimum(lens_, el) + 8 + 6 * (np.ceil(np.ceil(lens_ / (32 * el) + 1) / 32)) + 2
+            gate = (chain + 1) * 2.0 ** -24 * absum + 2.0 ** -24 * absum  # + the final fp32 rounding
+            err = np.abs(got.astype(np.float64) - want)
+            assert (err <= gate).all(), (np.nonzero(err > gate)[0][:5], err.max())
+        else:
+            assert (got.view(np.uint32) == want.astype(x.dtype).view(np.uint32)).all(), op
