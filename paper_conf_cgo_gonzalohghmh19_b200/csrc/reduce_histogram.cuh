@@ -159,6 +159,76 @@ __global__ void __launch_bounds__(256) k_histogram(const HistParams p, int parts
   }
 }
 
+// Many bins in one pass (16384 < nbins <= ~116 K): one block per SM holds the
+// whole histogram as 16-bit counters, two bins per shared word, so 65536 bins
+// take 128 KB instead of needing four passes over the input with 32-bit bins.
+// A counter is kept below 2^16 by its carry: the update that takes a half from
+// 0x7FFF to 0x8000 (seen in the atomic's return value) moves 0x8000 to the
+// global count and subtracts it from the half -- exact, and since at most a
+// block's in-flight updates (<< 0x8000) can land in between, a half never
+// wraps into its neighbour.  The final merge adds both halves of every
+// non-zero word to `counts`.
+template <int DT>
+__global__ void __launch_bounds__(1024) k_histogram16(const HistParams p) {
+  extern __shared__ unsigned sw[];
+  const int words = (p.nbins + 1) >> 1;
+  for (int i = threadIdx.x; i < words + 32; i += blockDim.x) sw[i] = 0u;
+  __syncthreads();
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sw);
+  const uint32_t sdummy = sbase + 4u * (uint32_t)(words + (threadIdx.x & 31));
+  auto count8 = [&](const uint32_t (&r)[8]) {
+    int bin[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) bin[k] = hist_bin<DT>(r[k], p);
+    uint32_t old[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {  // unconditional (uncounted elements add 0 to the lane's dummy word)
+      const bool ok = bin[k] >= 0;
+      const uint32_t a = ok ? sbase + 4u * (uint32_t)(bin[k] >> 1) : sdummy;
+      const uint32_t inc = ok ? 1u << ((bin[k] & 1) << 4) : 0u;
+      asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(old[k]) : "r"(a), "r"(inc) : "memory");
+    }
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int sh = (bin[k] & 1) << 4;
+      if (bin[k] >= 0 && ((old[k] >> sh) & 0xFFFFu) == 0x7FFFu) {  // this update reached 0x8000: carry
+        atomicSub(&sw[bin[k] >> 1], 0x8000u << sh);
+        atomicAdd(p.counts + bin[k], 0x8000u);
+      }
+    }
+  };
+  const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+  unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
+  for (; v + stride < p.body_vecs; v += 2 * stride) {
+    uint32_t r0[8], r1[8];
+    ld_v8(p.body + v * kVecBytes, r0);
+    ld_v8(p.body + (v + stride) * kVecBytes, r1);
+    count8(r0);
+    count8(r1);
+  }
+  if (v < p.body_vecs) {
+    uint32_t r[8];
+    ld_v8(p.body + v * kVecBytes, r);
+    count8(r);
+  }
+  if (blockIdx.x == 0 && threadIdx.x < 16) {  // head and tail elements (< 8 each)
+    const int t = threadIdx.x;
+    const bool mine = t < p.head || (t >= 8 && t - 8 < p.tail);
+    if (mine) {
+      const uint32_t w = t < p.head ? __ldg((const uint32_t*)p.in + t)
+                                    : __ldg((const uint32_t*)(p.body + p.body_vecs * kVecBytes) + (t - 8));
+      const int bn = hist_bin<DT>(w, p);
+      if (bn >= 0) atomicAdd(p.counts + bn, 1u);
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < words; i += blockDim.x) {
+    const unsigned w = sw[i];
+    if (w & 0xFFFFu) atomicAdd(p.counts + 2 * i, w & 0xFFFFu);
+    if (w >> 16) atomicAdd(p.counts + 2 * i + 1, w >> 16);
+  }
+}
+
 // Copies per bin: as many as keep a block's bins within 64 KB (<= 32).
 inline int hist_rep_log2(int bins_per_block) {
   int rl = 5;
@@ -173,6 +243,29 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   cudaError_t e = cudaMemsetAsync(p.counts, 0, (size_t)p.nbins * sizeof(unsigned), s);
   if (e != cudaSuccess) return e;
+  if (p.nbins > kHistSharedMaxBins) {  // one pass with 16-bit shared counters if the histogram fits
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    const size_t smem16 = ((size_t)(p.nbins + 1) / 2 + 32) * sizeof(unsigned);
+    if (smem16 <= (size_t)optin) {
+      e = cudaFuncSetAttribute(k_histogram16<DT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem16);
+      if (e != cudaSuccess) return e;
+      int per_sm = 0;
+      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_histogram16<DT>, 1024, smem16);
+      if (e != cudaSuccess) return e;
+      if (per_sm < 1) per_sm = 1;
+      long long grid = (long long)sms * per_sm;
+      const long long need = (long long)((p.body_vecs + 1023) / 1024);
+      if (need < grid) grid = need < 1 ? 1 : need;
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3((unsigned)grid, 1, 1);
+      cfg.blockDim = dim3(1024, 1, 1);
+      cfg.dynamicSmemBytes = smem16;
+      cfg.stream = s;
+      cfg.numAttrs = 0;
+      return cudaLaunchKernelEx(&cfg, k_histogram16<DT>, p);
+    }
+  }
   const int parts = (p.nbins + kHistSharedMaxBins - 1) / kHistSharedMaxBins;
   const bool shared = parts <= 8;  // up to 8 passes over the data beat one global atomic per element
   const int per_block_bins = shared ? (parts == 1 ? p.nbins : kHistSharedMaxBins) : 0;

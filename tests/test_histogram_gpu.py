@@ -91,3 +91,29 @@ def test_histogram_replication_boundaries(dtype):
         got = rb.histogram(t, lo, hi, nbins).cpu().numpy().view(np.uint32)
         want = oracle.histogram(x, lo, hi, nbins)
         assert (got == want).all(), (nbins, np.nonzero(got != want)[0][:5])
+
+
+@pytest.mark.parametrize("dtype", ["int32", "float32"])
+@pytest.mark.parametrize("nbins", [16385, 65536, 100003])
+def test_histogram_16bit_counters_carry(dtype, nbins):
+    """16384 < nbins: one pass with 16-bit shared counters.  A few bins get far
+    more than 2^15 elements per block (every 0x8000 moves to the global count),
+    neighbours of those bins (same shared word) stay exact, and the rest is
+    spread over every bin."""
+    rb = _rb()
+    n = (1 << 25) + 13
+    if dtype == "int32":
+        x = synth.make("int32", n, "int_full", 5) % nbins
+        x[: n // 2] = 7            # bin 7 (word 3, high half) and
+        x[n // 2: n // 2 + n // 4] = 6  # bin 6, the low half of the same word
+        lo, hi = 0.0, float(nbins)
+    else:
+        x = synth.make("float32", n, "uniform01", 5)
+        x[: n // 2] = np.float32(0.5)
+        x[n // 2: n // 2 + n // 4] = np.float32(0.5) - np.float32(1.0 / nbins)
+        lo, hi = 0.0, 1.0
+    t = to_device(x, 1)
+    got = rb.histogram(t, lo, hi, nbins).cpu().numpy().view(np.uint32)
+    want = oracle.histogram(x, lo, hi, nbins)
+    assert (got == want).all(), np.nonzero(got != want)[0][:5]
+    assert int(got.sum()) == int(want.sum())
