@@ -137,7 +137,9 @@ def test_segmented_argument_validation():
     assert L.reduce_segmented(1, 0, 4096, None, 10, 8192, None, None) == 1        # offsets NULL
     assert L.reduce_segmented(1, 0, 4096, 4096, 10, None, None, None) == 1        # out NULL
     assert L.reduce_segmented(5, 0, 4096, 4096, 10, 8192, None, None) == 1        # dtype
-    assert L.reduce_batched(1, 0, 4096, 10, 10, 8192, None, ctypes.byref(o)) == 1  # seg_group
+    assert L.reduce_batched(1, 0, 4096, 10, 10, 8192, None, ctypes.byref(o)) == 1  # seg_group 5 needs offsets
+    o6 = rb.make_opts(seg_group=6)
+    assert L.reduce_segmented(1, 0, 4096, 4096, 10, 8192, None, ctypes.byref(o6)) == 1  # seg_group range
     assert L.reduce_batched(2, 0, 4100, 10, 10, 8192, None, None) == 1            # misaligned fp64
     assert L.reduce_batched(1, 0, None, 10, 0, None, None, None) == 0             # no segments: no-op
 
