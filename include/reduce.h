@@ -232,8 +232,11 @@ int reduce_batched(int dtype, int op, const void* in, size_t seg_len, size_t num
  * when that is in [0, nbins).  NaN is never counted.  `counts` is a DEVICE array of nbins uint32, overwritten (a memset
  * node precedes the kernel).  Per-block shared-memory histograms with
  * shared atomics (the paper's "VA1" codelet per bin), merged with global
- * atomics; nbins > 16384 counts in global memory directly.  Counts are exact
- * (integer atomics commute). */
+ * atomics: up to 16384 bins as replicated 32-bit counters; up to what one
+ * block's shared memory holds at 16 bits per bin (~116 K bins) in one pass
+ * with 16-bit counters whose every 0x8000 is carried to `counts`; beyond that
+ * in 16384-bin passes (up to 8), else straight into global memory.  Counts
+ * are exact (integer atomics commute). */
 int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, int nbins, uint32_t* counts,
                      reduce_stream_t stream);
 
