@@ -362,6 +362,10 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
     int m = 0;
     bool ovf = false;
     long long v = vfirst;
+    // batches past the two prefetched ones are loaded four at a time (chunks
+    // of very short segments need dozens: one round trip per four, not per one)
+    long long q0 = 0, q1 = 0, q2 = 0, q3 = 0;
+    int nq = 0;
 #pragma unroll 1
     for (long long base = s0;;) {
       const int loc = v < clo ? -1 : (v >= chi ? (int)B::C : (int)(v - clo));
@@ -375,7 +379,22 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
       m += cnt;
       if (stop) break;
       base += 32;
-      v = base == s0 + 32 ? vsecond : (base + lane <= nseg ? __ldg(p.offsets + base + lane) : LLONG_MAX);
+      if (base == s0 + 32) {
+        v = vsecond;
+      } else {
+        if (nq == 0) {
+          q0 = base + lane <= nseg ? __ldg(p.offsets + base + lane) : LLONG_MAX;
+          q1 = base + 32 + lane <= nseg ? __ldg(p.offsets + base + 32 + lane) : LLONG_MAX;
+          q2 = base + 64 + lane <= nseg ? __ldg(p.offsets + base + 64 + lane) : LLONG_MAX;
+          q3 = base + 96 + lane <= nseg ? __ldg(p.offsets + base + 96 + lane) : LLONG_MAX;
+          nq = 4;
+        }
+        v = q0;
+        q0 = q1;
+        q1 = q2;
+        q2 = q3;
+        --nq;
+      }
     }
     __syncwarp();
     BalChunk<T> k;
