@@ -248,12 +248,9 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
     const size_t smem16 = ((size_t)(p.nbins + 1) / 2 + 32) * sizeof(unsigned);
     if (smem16 <= (size_t)optin) {
-      e = cudaFuncSetAttribute(k_histogram16<DT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem16);
+      e = opt_in_smem((const void*)k_histogram16<DT>, (int)smem16);
       if (e != cudaSuccess) return e;
-      int per_sm = 0;
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_histogram16<DT>, 1024, smem16);
-      if (e != cudaSuccess) return e;
-      if (per_sm < 1) per_sm = 1;
+      const int per_sm = blocks_per_sm((const void*)k_histogram16<DT>, 1024, smem16);
       long long grid = (long long)sms * per_sm;
       const long long need = (long long)((p.body_vecs + 1023) / 1024);
       if (need < grid) grid = need < 1 ? 1 : need;
@@ -273,14 +270,11 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
   const size_t smem = shared ? ((size_t)per_block_bins * ((size_t)1 << rep_log2) + 32) * sizeof(unsigned) : 0;
   auto kernel = shared ? k_histogram<DT, true> : k_histogram<DT, false>;
   if (smem > 48 * 1024) {
-    e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = opt_in_smem((const void*)kernel, (int)smem);
     if (e != cudaSuccess) return e;
   }
   // one wave per part group: as many blocks as fit (the shared bins limit residency)
-  int per_sm = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, block, smem);
-  if (e != cudaSuccess) return e;
-  if (per_sm < 1) per_sm = 1;
+  const int per_sm = blocks_per_sm((const void*)kernel, block, smem);
   long long per_part = (long long)sms * per_sm / (shared ? parts : 1);
   const long long need = (long long)((p.body_vecs + block - 1) / block);
   if (need < per_part) per_part = need;

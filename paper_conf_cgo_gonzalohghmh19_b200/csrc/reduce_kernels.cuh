@@ -21,9 +21,10 @@
 //   * grid combine (S5) and finalise (S6): by desc.gc, see grid_combine().
 #pragma once
 #include <cooperative_groups.h>
+#include <map>
 #include <mutex>
+#include <tuple>
 #include <type_traits>
-#include <unordered_set>
 #include "reduce_device.cuh"
 #include "reduce_internal.h"
 
@@ -334,6 +335,46 @@ inline KParams make_params(const LaunchDesc& d) {
   return p;
 }
 
+// Function attributes belong to each device's instance of the module: opt a
+// kernel in to at least `smem_bytes` of dynamic shared memory (and, if asked,
+// to non-portable cluster sizes).  The attribute is a maximum, so it is only
+// ever raised: a later, smaller request must not undercut an earlier size.
+inline cudaError_t opt_in_smem(const void* kern, int smem_bytes, bool nonportable_cluster = false) {
+  static std::mutex mu;
+  static std::map<std::pair<int, const void*>, int> granted;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(mu);
+  const auto key = std::make_pair(dev, kern);
+  auto it = granted.find(key);
+  if (it != granted.end() && it->second >= smem_bytes) return cudaSuccess;
+  cudaError_t e = cudaSuccess;
+  if (nonportable_cluster) e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+  if (e == cudaSuccess) granted[key] = smem_bytes;
+  return e;
+}
+
+// Resident blocks per SM of (kernel, block size, dynamic shared memory) on the
+// current device (at least 1), computed once per (device, kernel, shape).
+inline int blocks_per_sm(const void* kern, int block, size_t smem) {
+  static std::mutex mu;
+  static std::map<std::tuple<int, const void*, int, size_t>, int> cache;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(mu);
+  const auto key = std::make_tuple(dev, kern, block, smem);
+  auto it = cache.find(key);
+  if (it != cache.end()) return it->second;
+  int nb = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, block, smem) != cudaSuccess || nb < 1) {
+    cudaGetLastError();
+    nb = 1;
+  }
+  cache[key] = nb;
+  return nb;
+}
+
 // Launch one k_reduce instantiation; GC_CLUSTER launches exactly one cluster
 // of d.grid CTAs (sizes above the portable 8 need the non-portable opt-in);
 // STAGE_SMEM needs block*U*32 bytes of dynamic shared memory (opt-in above 48 KB).
@@ -341,15 +382,8 @@ inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& 
   const size_t smem = d.stage == STAGE_SMEM ? (size_t)d.block * d.unroll * kVecBytes : 0;
   // any dynamic tile opts in (static scratch + a 32 KB tile can already pass the 48 KB default)
   if (smem > 0 || (d.gc == GC_CLUSTER && d.grid > 8)) {
-    static std::mutex mu;
-    static std::unordered_set<const void*> opted;
-    std::lock_guard<std::mutex> lk(mu);
-    if (!opted.count((const void*)kern)) {
-      cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-      if (e == cudaSuccess) e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmemTileBytes);
-      if (e != cudaSuccess) return e;
-      opted.insert((const void*)kern);
-    }
+    const cudaError_t e = opt_in_smem((const void*)kern, kMaxSmemTileBytes, true);
+    if (e != cudaSuccess) return e;
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(d.grid, 1, 1);

@@ -587,23 +587,16 @@ template <int DT, int OP>
 cudaError_t launch_segbal_op(const SegParams& p0, int sms, cudaStream_t s) {
   using B = Bal<Tr<DT, OP>>;
   constexpr size_t smem = (size_t)kBalWarps * B::kWarpSmem;
-  static int per_sm = 0;
-  if (per_sm == 0) {
-    cudaError_t e = cudaFuncSetAttribute(k_segbal<DT, OP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    int nb = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessorWithFlags(&nb, k_segbal<DT, OP>, kBalWarps * 32, smem, 0) !=
-            cudaSuccess || nb < 1)
-      nb = 1;
-    per_sm = nb;
-  }
+  cudaError_t e = opt_in_smem((const void*)k_segbal<DT, OP>, (int)smem);
+  if (e != cudaSuccess) return e;
+  const int per_sm = blocks_per_sm((const void*)k_segbal<DT, OP>, kBalWarps * 32, smem);
   SegParams p = p0;
   long long grid = (long long)sms * per_sm;  // one wave: every warp owns one contiguous chunk range
   if (grid * kBalWarps > (long long)kBalRanges) grid = kBalRanges / kBalWarps;
   p.b.nranges = grid * kBalWarps;
   long long sgrid = (p.nseg + 255) / 256;
   if (sgrid > (long long)sms * 8) sgrid = (long long)sms * 8;
-  cudaError_t e = bal_launch(k_segbal_scan<DT, OP>, sgrid, 256, 0, p, s);
+  e = bal_launch(k_segbal_scan<DT, OP>, sgrid, 256, 0, p, s);
   if (e != cudaSuccess) return e;
   e = bal_launch(k_segbal<DT, OP>, grid, kBalWarps * 32, smem, p, s);
   if (e != cudaSuccess) return e;

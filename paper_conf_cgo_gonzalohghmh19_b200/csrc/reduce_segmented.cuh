@@ -441,15 +441,6 @@ __global__ void __launch_bounds__(256) k_seg_finish(const SegParams p) {
   pdl_trigger();
 }
 
-// Resident blocks per SM of a kernel at a block size (persistent grids are one
-// full wave of them).
-template <class K>
-int seg_blocks_per_sm(K kernel, int block) {
-  int nb = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, block, 0) != cudaSuccess || nb < 1) nb = 1;
-  return nb;
-}
-
 template <class K>
 cudaError_t seg_launch(K kernel, long long grid, int block, const SegParams& p, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
@@ -466,12 +457,10 @@ cudaError_t seg_launch(K kernel, long long grid, int block, const SegParams& p, 
 
 template <int DT, int OP, int kGroup, bool kTail>
 cudaError_t launch_segmented_group(const SegParams& p, int block, int sms, cudaStream_t s) {
-  static int per_sm[17] = {0};  // resident blocks by block / 32 (cached)
-  const int key = block / 32;
-  if (per_sm[key] == 0) per_sm[key] = seg_blocks_per_sm(k_segmented<DT, OP, kGroup, kTail>, block);
+  const int per_sm = blocks_per_sm((const void*)k_segmented<DT, OP, kGroup, kTail>, block, 0);
   const long long per_block = kGroup > 0 ? block / kGroup : 1;
   long long grid = (p.nseg + per_block - 1) / per_block;
-  const long long cap = (long long)sms * per_sm[key];  // one full wave
+  const long long cap = (long long)sms * per_sm;  // one full wave
   if (grid > cap) grid = cap;
   if (grid < 1) grid = 1;
   return seg_launch(k_segmented<DT, OP, kGroup, kTail>, grid, block, p, s);
@@ -493,8 +482,7 @@ cudaError_t launch_segmented_op(const SegParams& p, int group, int block, cudaSt
   cudaError_t e = p.tail ? launch_segmented_groups<DT, OP, true>(p, group, block, sms, s)
                          : launch_segmented_groups<DT, OP, false>(p, group, block, sms, s);
   if (e != cudaSuccess || !p.use_q) return e;
-  static int chunk_per_sm = 0;
-  if (chunk_per_sm == 0) chunk_per_sm = seg_blocks_per_sm(k_seg_chunks<DT, OP>, 256);
+  const int chunk_per_sm = blocks_per_sm((const void*)k_seg_chunks<DT, OP>, 256, 0);
   e = seg_launch(k_seg_chunks<DT, OP>, (long long)sms * chunk_per_sm, 256, p, s);
   if (e != cudaSuccess) return e;
   return seg_launch(k_seg_finish<DT, OP>, sms, 256, p, s);
