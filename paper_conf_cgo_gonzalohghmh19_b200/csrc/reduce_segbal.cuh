@@ -11,7 +11,8 @@
 // partition is by data, as the paper's tiled distribution of a single array
 // (Fig. 1(b)), with segment boundaries carried inside it.
 //
-//   k_segbal_scan : one thread per segment: the identity for empty segments,
+//   k_segbal_scan : a one-wave grid striding over the segments: the identity
+//                   for empty segments,
 //                   a flag if the offsets are not monotone (then the chunk
 //                   kernel falls back to one warp per segment), and for every
 //                   chunk range the segment holding its first element.
@@ -61,13 +62,13 @@ constexpr int kBalWarps = 4;                    // warps per block of k_segbal
 // resident blocks asked of ptxas: 5 (96 registers, 20 warps per SM) for the
 // 4-byte plain ops; fp64 and accurate sums need more registers (4 blocks)
 constexpr int bal_min_blocks(int dt, int op) { return (dt != 2 && op != 3) ? RB_SEGBAL_MINB : 4; }
-constexpr int kBalVecsPerLane = RB_SEGBAL_VPL;  // 32-byte vectors per lane per chunk (256 contiguous bytes)
+constexpr int kBalVecsPerLane = RB_SEGBAL_VPL;  // 32-byte vectors per lane per chunk (128 contiguous bytes)
 
 template <class T>
 struct Bal {
   using Acc = typename T::Acc;
   static constexpr int s = sizeof(typename T::Elem);
-  static constexpr int EL = kBalVecsPerLane * T::VE;  // elements per lane (64 or 32)
+  static constexpr int EL = kBalVecsPerLane * T::VE;  // elements per lane (32 or 16)
   static constexpr long long C = 32LL * EL;           // elements per chunk (32 lanes x kBalVecsPerLane x 32 B = 4 KB)
   static constexpr int kList = (int)C + 64;           // offsets entries kept in shared memory
   static constexpr size_t kPieceBytes = (size_t)EL * 32 * sizeof(Acc);
@@ -89,7 +90,7 @@ __device__ __forceinline__ typename T::Elem elem_ident() {
   else return (typename T::Elem)T::ident();
 }
 
-// element e of a lane's 8 vectors (e is a constant after unrolling)
+// element e of a lane's vectors (e is a constant after unrolling)
 template <class T>
 __device__ __forceinline__ typename T::Elem bal_elem(const uint32_t (&r)[kBalVecsPerLane][8], int e) {
   using Elem = typename T::Elem;
