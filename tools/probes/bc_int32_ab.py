@@ -19,8 +19,8 @@ dev = torch.device("cuda", 0)
 stream = torch.cuda.Stream(dev)
 DTYPE = sys.argv[1] if len(sys.argv) > 1 else "int32"
 OPS = sys.argv[2].split(",") if len(sys.argv) > 2 else ["sum", "max"]
-DTC = {"int32": 0, "float32": 1}[DTYPE]
-pool = torch.empty((2 << 30) // 4, dtype=getattr(torch, DTYPE), device=dev)
+DTC = {"int32": 0, "float32": 1, "float64": 2}[DTYPE]
+pool = torch.empty((2 << 30) // (8 if DTYPE == "float64" else 4), dtype=getattr(torch, DTYPE), device=dev)
 if DTYPE == "int32":
     pool.random_(-1000, 1000)
 else:
@@ -29,7 +29,7 @@ rb.prepare(stream, pool.numel())
 out = torch.empty(4096, dtype=pool.dtype, device=dev)
 for op in OPS:
     for lb in range(12, 31, 2):
-        n = (1 << lb) // 4
+        n = (1 << lb) // (8 if DTYPE == "float64" else 4)
         R = max(20, min(100, (400 << 20) // (1 << lb))) if (1 << lb) >= (256 << 20) else max(5, min(100, (400 << 20) // (1 << lb)))
         warm, timed = disjoint_regions(pool, R, n)
         plan = rb.query_plan(DTYPE, op, n, in_ptr=pool.data_ptr())
@@ -40,7 +40,7 @@ for op in OPS:
             base = dict(block=plan["block"], unroll=plan["unroll"], grid_combine=plan["grid_combine"], grid=-1,
                         stage=plan["stage"])
         row = {"dtype": DTYPE, "op": op, "bytes": f"2^{lb}", "plan": base}
-        for bc, name in ((0, "Vs"), (1, "VA2+S"), (2, "VA1")):
+        for bc, name in ((0, "Vs"), (1, "VA2+S"), (2, "VA1"), (3, "V")):
             opts = rb.make_opts(mode="fast", block_combine=bc, **base)
             k = [0]
 
