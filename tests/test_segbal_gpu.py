@@ -217,6 +217,7 @@ def test_matches_group_kernels_exactly_for_ints():
 
 def _reduceat(x, offs, op):
     """numpy reference per segment (vectorised; empty segments -> identity)."""
+    x = x[: int(offs[-1])]  # reduceat's last segment runs to the end of its input
     lo = offs[:-1]
     empty = offs[1:] <= lo
     idx = np.minimum(lo, max(x.size - 1, 0))
@@ -264,3 +265,30 @@ def test_bench_workload_full_size(dtype):
             assert (err <= gate).all(), (np.nonzero(err > gate)[0][:5], err.max())
         else:
             assert (got.view(np.uint32) == want.astype(x.dtype).view(np.uint32)).all(), op
+
+
+def test_concurrent_streams_independent_workspaces():
+    """two streams run balanced segmented calls at the same time: each stream's
+    chunk arrays (and flags / tickets) are its own"""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    rng = np.random.Generator(np.random.PCG64(44))
+    cases = []
+    for k in range(2):
+        lens = np.minimum((rng.pareto(1.2, 30000) * 12.8).astype(np.int64) + 1, 300_000)
+        offs = _offsets(lens, start=k)
+        x = _data("int32", int(offs[-1]) + 1, 50 + k)
+        cases.append((x, offs, to_device(x, k), torch.from_numpy(offs).cuda()))
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    for s in streams:
+        rb.prepare(s, 1 << 20)
+    outs = [torch.empty(len(c[1]) - 1, dtype=torch.int32, device="cuda") for c in cases]
+    torch.cuda.synchronize()
+    for rep in range(5):
+        for (x, offs, xt, ot), s, o in zip(cases, streams, outs):
+            rb.reduce_segmented(xt, ot, "sum", out=o, stream=s)
+    torch.cuda.synchronize()
+    for (x, offs, xt, ot), o in zip(cases, outs):
+        want = _reduceat(x, offs, "sum")
+        want = ((want + 2 ** 31) % 2 ** 32 - 2 ** 31).astype(np.int32)
+        assert (o.cpu().numpy() == want).all()
