@@ -152,6 +152,32 @@ def gpu_identity(index: int):
         return {"error": repr(e)[:80]}
 
 
+def software_env(dev):
+    """GPU shape and software versions for the JSON line (metrics)."""
+    import torch
+    env = {}
+    try:
+        p = torch.cuda.get_device_properties(dev)
+        env.update(sm_count=p.multi_processor_count, l2_bytes=getattr(p, "L2_cache_size", None),
+                   hbm_bytes=p.total_memory, cc=f"{p.major}.{p.minor}")
+    except Exception as e:
+        env["device_error"] = repr(e)[:80]
+    env["torch"] = torch.__version__
+    env["cuda_runtime"] = torch.version.cuda
+    try:
+        env["nccl"] = ".".join(str(v) for v in torch.cuda.nccl.version())
+    except Exception:
+        pass
+    try:
+        import pynvml
+        pynvml.nvmlInit()
+        d = pynvml.nvmlSystemGetDriverVersion()
+        env["driver"] = d.decode() if isinstance(d, bytes) else d
+    except Exception:
+        pass
+    return env
+
+
 def host_info():
     model = ""
     try:
@@ -745,6 +771,7 @@ def main():
             "roofline": roofline, "e2e": e2e, "clocks": clocks.summary(),
             "gpu_launches": args.steps * launches_per_step,
             "gpu": gpu_identity(local),
+            "env": software_env(dev),
         }
         if decomposition is not None:
             line["sharded_decomposition"] = decomposition
