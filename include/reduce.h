@@ -163,6 +163,16 @@ typedef struct {
   long long chain;     /* longest fp addition chain L (error bound (L+1)u*sum|x|) */
 } reduce_plan_t;
 
+/* Stream ordering.  Kernels are launched with programmatic dependent launch:
+ * a reduction's first blocks may start while the previous kernel on the stream
+ * drains.  A reduce() / reduce_ex() whose input does not overlap the previous
+ * library call's output on the stream loads its first tile before its
+ * dependency resolves (it waits before touching anything else); this is safe
+ * for any producer that is not itself a programmatic-launch primary writing
+ * the input -- callers whose own kernels trigger early completion
+ * (griddepcontrol.launch_dependents) before writing a reduction's input set
+ * REDUCE_NO_EARLY=1 (REDUCE_NO_PDL=1 disables programmatic launch altogether). */
+
 /* Reduce in[0..n) with `op` into *out (device).  Uses the process-default mode. */
 int reduce(int dtype, int op, const void* in, size_t n, void* out, reduce_stream_t stream);
 

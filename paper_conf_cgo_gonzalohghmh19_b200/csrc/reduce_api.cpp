@@ -365,16 +365,39 @@ int get_seg_bal(cudaStream_t stream, char** out) {
   return REDUCE_OK;
 }
 
-int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream) {
+int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream, bool allow_early) {
   LaunchDesc& d = P->d;
   const int combo = combo_index(d.dtype, d.op);
   d.out = out;
   d.slots = ws->slots + combo * kSlotRegionBytes;
   d.ticket = (unsigned*)(ws->tickets + combo * (size_t)kSlotBytes);
   d.partials = ws->partials;
+  d.early = 0;
+  if (allow_early && early_enabled() && pdl_enabled() && P->n > 0) {
+    const uintptr_t lo = (uintptr_t)d.in, hi = lo + (uintptr_t)P->n * (uintptr_t)P->elem;
+    d.early = (hi <= ws->last_out_lo.load(std::memory_order_relaxed) ||
+               lo >= ws->last_out_hi.load(std::memory_order_relaxed)) ? 1 : 0;
+  }
   cudaError_t e = launch_reduce(d, stream);
+  if (allow_early) {  // this call wrote `out` only (one value of at most 16 bytes)
+    ws->last_out_lo.store((uintptr_t)out, std::memory_order_relaxed);
+    ws->last_out_hi.store((uintptr_t)out + 16, std::memory_order_relaxed);
+  } else {
+    ws->last_out_lo.store(0, std::memory_order_relaxed);
+    ws->last_out_hi.store(~(uintptr_t)0, std::memory_order_relaxed);
+  }
   if (e != cudaSuccess) return cuda_fail(e, "reduction kernel launch");
   return REDUCE_OK;
+}
+
+void note_unknown_output(cudaStream_t stream) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return;
+  std::lock_guard<std::mutex> lk(g_ws_mu);
+  auto it = g_ws.find(std::make_pair(dev, stream));
+  if (it == g_ws.end() || it->second == nullptr) return;
+  it->second->last_out_lo.store(0, std::memory_order_relaxed);
+  it->second->last_out_hi.store(~(uintptr_t)0, std::memory_order_relaxed);
 }
 
 static size_t partials_needed(const Plan& P) {
@@ -400,7 +423,7 @@ int reduce_ex(int dtype, int op, const void* in, size_t n, void* out, reduce_str
   Workspace* ws = nullptr;
   st = get_workspace((cudaStream_t)stream, partials_needed(P), &ws);
   if (st != REDUCE_OK) return st;
-  return launch_plan(&P, ws, out, (cudaStream_t)stream);
+  return launch_plan(&P, ws, out, (cudaStream_t)stream, /*allow_early=*/true);
 }
 
 static int segmented_common(int dtype, int op, const void* in, const int64_t* offsets, size_t seg_len,
@@ -412,6 +435,7 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   const int s = dtype == REDUCE_FLOAT64 ? 8 : 4;
   if (nseg == 0) return REDUCE_OK;
   if (out == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "out is NULL");
+  note_unknown_output((cudaStream_t)stream);  // its kernels write `out` and trigger dependents early
   if (((uintptr_t)out % (uintptr_t)s) != 0) return fail(REDUCE_ERR_INVALID_ARG, "out is not aligned to the element size");
   const bool uniform = offsets == nullptr;
   if (in == nullptr && (!uniform || seg_len > 0)) return fail(REDUCE_ERR_INVALID_ARG, "in is NULL");
@@ -546,6 +570,7 @@ int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, 
   }
   p.nbins = nbins;
   p.counts = counts;
+  note_unknown_output((cudaStream_t)stream);
   cudaError_t e = launch_histogram(dtype, p, 256, (cudaStream_t)stream);
   if (e != cudaSuccess) return cuda_fail(e, "histogram launch");
   return REDUCE_OK;

@@ -79,6 +79,8 @@ struct LaunchDesc {
   unsigned* ticket;              // this (dtype, op)'s ticket (GC_ATOMIC / GC_LAST_BLOCK)
   void* partials;                // Grid[grid] (GC_TWO_PASS / GC_LAST_BLOCK)
   TeamArgs team;                 // team.k > 0: exchange the raw result with the team first
+  int early;                     // 1: load the first tile before griddepcontrol.wait (the input is
+                                 //    not an output of the previous call on the stream)
 };
 
 // Long-segment queue of a segmented call (lives in the stream's workspace):
@@ -191,6 +193,9 @@ cudaError_t launch_init_workspace(void* slots_base, void* tickets_base, cudaStre
 // Programmatic dependent launch of the library's kernels (default on; the
 // environment variable REDUCE_NO_PDL=1 turns it off, for A/B measurements).
 bool pdl_enabled();
+// Loads of the input before the programmatic dependency resolves (default on;
+// REDUCE_NO_EARLY=1 turns it off, for A/B measurements).
+bool early_enabled();
 
 constexpr int kCombos = 12;  // 3 dtypes x 4 ops (sum, min, max, accurate sum)
 constexpr int combo_index(int dtype, int op) { return dtype * 4 + op; }

@@ -44,6 +44,7 @@ struct KParams {
   unsigned* ticket;
   void* partials;
   TeamArgs team;
+  int early;
 };
 
 // ---- one-shot cross-GPU combine through peer memory ------
@@ -220,6 +221,26 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
   // A team call whose members share this GPU never triggers: the next grid's
   // parked CTAs could fill the SMs a co-resident member needs to reach the
   // exchange this grid's last block is waiting in.
+  // Early loads (p.early, set by the host only when the input does not overlap
+  // the previous call's output on this stream): a block that is resident before
+  // the dependency resolves issues its first tile's loads first -- they fill the
+  // previous grid's drain -- and folds them after the wait (same order, same
+  // numerics).  The input is the only memory touched before the wait.
+  // (U <= 4 only: with 8 loads per thread the prefetched registers would be
+  // allocated beside the loop's -- 94 -> 120 registers, one block less per SM;
+  // the U = 8 kernels compile exactly as without early loads)
+  constexpr bool kEarly = STAGE == STAGE_REG && U <= 4;
+  uint32_t pre[kEarly ? U : 1][8];
+  bool have_pre = false;
+  if constexpr (kEarly) {
+    const long long tv = (long long)blockDim.x * U;
+    if (p.early && (long long)blockIdx.x < p.tiles && (unsigned long long)((blockIdx.x + 1) * tv) <= p.body_vecs) {
+      const char* ptr = p.body + ((unsigned long long)(blockIdx.x * tv) + threadIdx.x) * kVecBytes;
+#pragma unroll
+      for (int u = 0; u < U; ++u) ld_v8(ptr + (size_t)u * blockDim.x * kVecBytes, pre[u]);
+      have_pre = true;
+    }
+  }
   pdl_wait();
   const bool may_trigger = !p.team.shared_gpu;
   const bool early_trigger = may_trigger && gridDim.x > kPdlTriggerWindow && blockIdx.x + kPdlTriggerWindow >= gridDim.x;
@@ -231,12 +252,21 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
 
   const long long B = blockDim.x;
   const long long tile_vecs = B * U;
+  long long tile_first = blockIdx.x;
+  if constexpr (kEarly) {
+    if (have_pre) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, pre[u], u);
+      tile_first += gridDim.x;
+    }
+  }
+
   // no unrolling: an unrolled loop makes the compiler compute the trip count
   // with a 64-bit division (a CALL to the division routine) in every block's
   // prologue -- measurable latency at medium sizes, where the default grid
   // runs this loop exactly once
 #pragma unroll 1
-  for (long long tile = blockIdx.x; tile < p.tiles; tile += gridDim.x) {
+  for (long long tile = tile_first; tile < p.tiles; tile += gridDim.x) {
     const unsigned long long v0 = (unsigned long long)(tile * tile_vecs) + threadIdx.x;
     const char* ptr = p.body + v0 * kVecBytes;
     const bool full = (unsigned long long)((tile + 1) * tile_vecs) <= p.body_vecs;
@@ -330,6 +360,7 @@ inline KParams make_params(const LaunchDesc& d) {
   p.ticket = d.ticket;
   p.partials = d.partials;
   p.team = d.team;
+  p.early = d.early;
   // TWO_PASS: the exchange happens in the second kernel, not per block
   if (d.gc == GC_TWO_PASS) p.team.k = 0;
   return p;

@@ -1,6 +1,8 @@
 // reduce_runtime.h -- host runtime internals shared by reduce_api.cpp,
 // reduce_host.cpp and reduce_multi.cpp (not part of the ABI).
 #pragma once
+#include <atomic>
+#include <cstdint>
 #include <cstddef>
 #include <cstdint>
 #include <string>
@@ -23,6 +25,10 @@ struct Workspace {
   size_t partials_bytes = 0;
   char* segq = nullptr;        // long-segment queue of reduce_segmented / reduce_batched (kSegQBytes)
   char* segbal = nullptr;      // chunk arrays of the element-balanced reduce_segmented (kBalBytes)
+  // device bytes the last library call on this stream wrote for the caller
+  // ([0, max) = unknown): a reduce whose input does not overlap them may load
+  // its first tile before its programmatic dependency resolves
+  std::atomic<uintptr_t> last_out_lo{0}, last_out_hi{~(uintptr_t)0};
   // reduce_host staging (lazily created)
   char* staging = nullptr;     // 2 x staging_bytes
   size_t staging_bytes = 0;
@@ -58,8 +64,14 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
 // allocation would be needed during stream capture.
 int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** ws);
 
-// Fill the workspace pointers of plan->d and launch it.
-int launch_plan(Plan* plan, Workspace* ws, void* out, cudaStream_t stream);
+// Fill the workspace pointers of plan->d and launch it.  allow_early: a public
+// single-array call (reduce / reduce_ex), whose written bytes are exactly
+// `out`; other callers leave the stream's last output unknown.
+int launch_plan(Plan* plan, Workspace* ws, void* out, cudaStream_t stream, bool allow_early = false);
+
+// The stream's last output becomes unknown (entry points that launch other
+// kernels: segmented, histogram).  No-op if the stream has no workspace yet.
+void note_unknown_output(cudaStream_t stream);
 
 int num_sms();
 int default_mode();

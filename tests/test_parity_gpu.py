@@ -363,3 +363,33 @@ def test_reduce_host_chunks(dtype):
     for op in OPS:
         g = rb.reduce_host(x[:0], op)
         check(x[:0], op, np.array([g], NP[dtype]))
+
+
+def test_chained_calls_read_the_previous_output():
+    """Chains of calls on one stream where a call reads the previous call's
+    output (a reduce of the scalar just written; a reduce of a segmented
+    output), back to back with distinct values every iteration.  (The host
+    disables a kernel's early, pre-dependency loads when its input overlaps
+    the last output, or after entry points whose outputs it does not track.)"""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    s = torch.cuda.Stream()
+    rb.prepare(s, 1 << 20)
+    n = 1 << 16
+    xs = [torch.full((n,), float(k + 1), device="cuda") for k in range(64)]
+    buf = torch.full((4,), float("-inf"), device="cuda")
+    res = torch.empty(64, device="cuda")
+    seg_out = torch.empty(8, device="cuda")
+    res2 = torch.empty(64, device="cuda")
+    offs = torch.arange(0, n + 1, n // 8, dtype=torch.int64, device="cuda")
+    torch.cuda.synchronize()
+    with torch.cuda.stream(s):
+        for k in range(64):
+            rb.reduce(xs[k], "sum", out=buf[0:1], stream=s)          # buf[0] = (k+1) * n
+            rb.reduce(buf, "max", out=res[k:k + 1], stream=s)         # reads buf[0] just written
+            rb.reduce_segmented(xs[k], offs, "sum", out=seg_out, stream=s)
+            rb.reduce(seg_out, "sum", out=res2[k:k + 1], stream=s)    # reads the segmented output
+    torch.cuda.synchronize()
+    want = np.array([(k + 1) * n for k in range(64)], np.float32)
+    assert (res.cpu().numpy() == want).all(), res.cpu().numpy()[:8]
+    assert (res2.cpu().numpy() == want).all(), res2.cpu().numpy()[:8]
