@@ -1,5 +1,5 @@
 """The paper's variant study recast on B200: from the autotuner's measurements
-(profiles/tune/r01_tune_v5.json, graph-timed, cold inputs) print, per size,
+(profiles/tune/r01_tune_v7_early.json, graph-timed, cold inputs) print, per size,
 the best time of each block combine (the paper's cooperative codelets:
 Vs = shuffle/redux + shared partials, Listing 4; VA2+S = a shared atomic per
 warp, Fig. 3(b); VA1 = a shared atomic per thread, Fig. 3(a); V = shared tree,
@@ -19,9 +19,9 @@ GC = {0: "DIRECT", 1: "ATOMIC", 2: "TWO_PASS", 3: "LAST_BLOCK", 4: "CLUSTER"}
 
 
 def main():
-    d = json.load(open(os.path.join(ROOT, "profiles", "tune", "r01_tune_v5.json")))
+    d = json.load(open(os.path.join(ROOT, "profiles", "tune", "r01_tune_v7_early.json")))
     print("# The paper's reduction variants on B200 (graph-timed µs per call, cold input)\n")
-    print("Source: `profiles/tune/r01_tune_v5.json` (tools/tune.py), table by `tools/variant_table.py`.")
+    print("Source: `profiles/tune/r01_tune_v7_early.json` (tools/tune.py), table by `tools/variant_table.py`.")
     print("Block combines are compared at the launch shape the tuner measured them at "
           "(256 threads, 2 vectors per thread, the tuner's grid combine for that size); "
           "grid combines at their best launch shape.  Bold = fastest in the row.\n")
