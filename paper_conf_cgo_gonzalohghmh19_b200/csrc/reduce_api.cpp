@@ -493,7 +493,12 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
                                      row_bytes > (64u << 10));
   p.use_q = 0;
   p.q = SegQueue{nullptr, nullptr, nullptr, nullptr};
-  if (may_long) {
+  // uniform rows of whole 32-byte vectors on 32-byte boundaries, up to 256
+  // bytes, one thread per row: every load of a row in flight at once
+  if (uniform && lanes == 1 && in != nullptr && ((uintptr_t)in % 32u) == 0 && row_bytes > 0 &&
+      row_bytes % 32u == 0 && row_bytes <= 256 && !(op == REDUCE_SUM_ACCURATE && row_bytes == 32))
+    p.rows_nv = (int)(row_bytes / 32u);
+  if (may_long && p.rows_nv == 0) {
     char* q = nullptr;
     if (get_seg_queue((cudaStream_t)stream, &q) == REDUCE_OK) {  // else (capture without prepare): no queue
       p.use_q = 1;

@@ -147,6 +147,8 @@ struct SegParams {
   int use_q;                 // 1: offload long segments to q (2 more launches)
   int tail;                  // 1: fold a segment's last vectors in one predicated round
   SegQueue q;
+  int rows_nv;               // > 0: uniform 32-byte-aligned rows of rows_nv (<= 8) vectors, one
+                             //      thread per row with all its loads in flight (k_rows_aligned)
   int balanced;              // 1: element-balanced chunks (offsets arrays, reduce_segbal.cuh)
   SegBal b;
 };

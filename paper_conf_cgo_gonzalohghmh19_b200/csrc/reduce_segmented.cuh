@@ -441,6 +441,58 @@ __global__ void __launch_bounds__(256) k_seg_finish(const SegParams p) {
   pdl_trigger();
 }
 
+// Uniform rows of nv 32-byte vectors that all start on 32-byte boundaries
+// (row bytes a multiple of 32, aligned input) and are at most 256 bytes: one
+// thread per row issues every load of its row at once (the group kernels'
+// first round plus a dependent second round cost a load latency per row),
+// folds them with the vector tree and writes out[row].  Rows of NV = 1, 2 or 4
+// vectors take R = 8 / NV rows per thread per step (rows r, r + stride, ...),
+// so eight 32-byte loads are in flight per thread whatever the row length.
+// One-wave grid striding over the rows.  NV = 0: the row length is a runtime
+// value (<= 8 vectors), one row per step.
+template <int DT, int OP, int NV>
+__global__ void __launch_bounds__(256) k_rows_aligned(const SegParams p) {
+  using T = Tr<DT, OP>;
+  constexpr int R = NV > 0 ? 8 / NV : 1;
+  pdl_wait();
+  const int nv = NV > 0 ? NV : p.rows_nv;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  const long long row_bytes = (long long)nv * kVecBytes;
+#pragma unroll 1
+  for (long long row0 = (long long)blockIdx.x * blockDim.x + threadIdx.x; row0 < p.nseg; row0 += stride * R) {
+    uint32_t r[8][8];
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      const long long row = row0 + j * stride;
+      const char* rp = p.in + row * row_bytes;
+#pragma unroll
+      for (int v = 0; v < (NV > 0 ? NV : 8); ++v)
+        if (row < p.nseg && v < nv) ld_v8(rp + v * kVecBytes, r[j * (NV > 0 ? NV : 0) + v]);
+    }
+#pragma unroll
+    for (int j = 0; j < R; ++j) {
+      const long long row = row0 + j * stride;
+      if (row >= p.nseg) break;
+      Part<T> a[T::NA];
+      init_parts<T>(a);
+      uint32_t aux = 0;
+#pragma unroll
+      for (int v = 0; v < (NV > 0 ? NV : 8); ++v)
+        if (v < nv) fold_vec<T>(a, aux, r[j * (NV > 0 ? NV : 0) + v], v);
+      seg_store<T>(p, row, T::to_grid(thread_result<T>(a, aux)));
+    }
+  }
+  pdl_trigger();
+}
+
+template <int DT, int OP, int NV>
+cudaError_t launch_rows_aligned(const SegParams& p, int sms, cudaStream_t s) {
+  const int per_sm = blocks_per_sm((const void*)k_rows_aligned<DT, OP, NV>, 256, 0);
+  long long grid = (p.nseg + 255) / 256;
+  if (grid > (long long)sms * per_sm) grid = (long long)sms * per_sm;
+  return seg_launch(k_rows_aligned<DT, OP, NV>, grid < 1 ? 1 : grid, 256, p, s);
+}
+
 template <class K>
 cudaError_t seg_launch(K kernel, long long grid, int block, const SegParams& p, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
@@ -479,6 +531,14 @@ cudaError_t launch_segmented_op(const SegParams& p, int group, int block, cudaSt
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (p.rows_nv > 0) {
+    if constexpr (OP != OP_SUMACC) {  // several rows per thread: the accurate pairs would not fit
+      if (p.rows_nv == 1) return launch_rows_aligned<DT, OP, 1>(p, sms, s);
+      if (p.rows_nv == 2) return launch_rows_aligned<DT, OP, 2>(p, sms, s);
+      if (p.rows_nv == 4) return launch_rows_aligned<DT, OP, 4>(p, sms, s);
+    }
+    return launch_rows_aligned<DT, OP, 0>(p, sms, s);
+  }
   cudaError_t e = p.tail ? launch_segmented_groups<DT, OP, true>(p, group, block, sms, s)
                          : launch_segmented_groups<DT, OP, false>(p, group, block, sms, s);
   if (e != cudaSuccess || !p.use_q) return e;

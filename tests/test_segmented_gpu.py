@@ -74,7 +74,7 @@ def test_segmented_matches_oracle_per_segment(dtype, group, skew):
 
 @pytest.mark.parametrize("dtype", DTYPES)
 @pytest.mark.parametrize("rows,cols", [(1, 1), (7, 33), (1000, 1024), (64, 100003), (4096, 17), (100003, 64),
-                                       (3000, 129)])
+                                       (3000, 129), (50001, 8), (30001, 32), (1001, 56), (2, 64)])
 def test_batched_rows(dtype, rows, cols):
     import torch
     import paper_conf_cgo_gonzalohghmh19_b200 as rb
@@ -221,3 +221,21 @@ def test_segmented_decreasing_pairs_are_empty(group):
             lo, hi = int(offs[i]), int(offs[i + 1])
             want = oracle.reduce(x[lo:hi], op).value if hi > lo else ident[op]
             assert int(got[i]) == int(want), (op, i, lo, hi, got[i], want)
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+def test_batched_aligned_short_rows_vs_misaligned(dtype):
+    """rows of whole 32-byte vectors on 32-byte boundaries (<= 256 B) take the
+    one-thread-per-row kernel with all loads in flight; the same rows starting
+    one element off 32-byte alignment take the group kernel -- both exact"""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    ve = 4 if dtype == "float64" else 8
+    for nv in (1, 3, 8):
+        cols, rows = nv * ve, 20011
+        x = synth.make(dtype, rows * cols + 1, "int_full" if dtype == "int32" else "intvalued", nv)
+        for off in (0, 1):
+            xt = to_device(x[off:off + rows * cols], off).view(rows, cols)
+            for op in OPS:
+                got = rb.reduce_batched(xt, op).cpu().numpy()
+                _check_segments(x[off:off + rows * cols], [(r * cols, (r + 1) * cols) for r in range(rows)], op, got, 1)
