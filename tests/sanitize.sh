@@ -38,6 +38,14 @@ for dt in (torch.int32, torch.float32, torch.float64):
     mbase = torch.arange(int(moffs[-1]) + 16, device="cuda").to(dt)[1:]
     for op in ("sum", "min", "max") + (("sum_accurate",) if dt != torch.int32 else ()):
         rb.reduce_segmented(mbase, moffs, op, seg_group=5)
+    # aligned short uniform rows (k_rows_aligned: 1, 2, 4 vectors per row and a runtime count)
+    abase = torch.arange(8 * 4099, device="cuda").to(dt)
+    ve = 4 if dt == torch.float64 else 8
+    for nvv in (1, 2, 3, 4, 8):
+        rows = abase.numel() // (nvv * ve)
+        rb.reduce_batched(abase[: rows * nvv * ve].view(rows, nvv * ve), "max")
+        if dt != torch.int32:
+            rb.reduce_batched(abase[: rows * nvv * ve].view(rows, nvv * ve), "sum_accurate")
     for g in (0, 1, 2, 3, 4):
         rb.reduce_segmented(base, offs, "sum", seg_group=g)
         rb.reduce_batched(base[:4096].view(64, 64), "max", seg_group=g)
