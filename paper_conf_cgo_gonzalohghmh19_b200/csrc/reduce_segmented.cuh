@@ -450,8 +450,11 @@ __global__ void __launch_bounds__(256) k_seg_finish(const SegParams p) {
 // so eight 32-byte loads are in flight per thread whatever the row length.
 // One-wave grid striding over the rows.  NV = 0: the row length is a runtime
 // value (<= 8 vectors), one row per step.
+#ifndef RB_ROWS_BLOCK
+#define RB_ROWS_BLOCK 128
+#endif
 template <int DT, int OP, int NV>
-__global__ void __launch_bounds__(256) k_rows_aligned(const SegParams p) {
+__global__ void __launch_bounds__(RB_ROWS_BLOCK) k_rows_aligned(const SegParams p) {
   using T = Tr<DT, OP>;
   constexpr int R = NV > 0 ? 8 / NV : 1;
   pdl_wait();
@@ -487,10 +490,10 @@ __global__ void __launch_bounds__(256) k_rows_aligned(const SegParams p) {
 
 template <int DT, int OP, int NV>
 cudaError_t launch_rows_aligned(const SegParams& p, int sms, cudaStream_t s) {
-  const int per_sm = blocks_per_sm((const void*)k_rows_aligned<DT, OP, NV>, 256, 0);
-  long long grid = (p.nseg + 255) / 256;
+  const int per_sm = blocks_per_sm((const void*)k_rows_aligned<DT, OP, NV>, RB_ROWS_BLOCK, 0);
+  long long grid = (p.nseg + RB_ROWS_BLOCK - 1) / RB_ROWS_BLOCK;
   if (grid > (long long)sms * per_sm) grid = (long long)sms * per_sm;
-  return seg_launch(k_rows_aligned<DT, OP, NV>, grid < 1 ? 1 : grid, 256, p, s);
+  return seg_launch(k_rows_aligned<DT, OP, NV>, grid < 1 ? 1 : grid, RB_ROWS_BLOCK, p, s);
 }
 
 template <class K>
