@@ -29,8 +29,23 @@ constexpr int kVecBytes = 32;    // one 256-bit load per thread per vector
 // Streaming 32-byte read-only load; never allocates in L1 (each byte is read
 // once).  Not `volatile`: the compiler may hoist/batch these (they read memory
 // no thread writes during the kernel).
+// RB_LD_HINT (A/B experiment hook: REDUCE_B200_NVCC_FLAGS=-DRB_LD_HINT=k builds,
+// tools/probes/lib_ab.sh + sweep_ab.py): 1 adds the 256-byte L2 prefetch-size
+// hint (SASS LTC256B), 2 the L2 evict_first priority (EFL2).  Neither moves any
+// size 16 KB-1 GiB by more than run-to-run noise (profiles/r01_ld_hint_ab.jsonl):
+// each warp's 256-bit load already covers 1 KB of whole 256-byte sectors.
+#ifndef RB_LD_HINT
+#define RB_LD_HINT 0
+#endif
+#if RB_LD_HINT == 1
+#define RB_LD_V8 "ld.global.nc.L1::no_allocate.L2::256B.v8.u32"
+#elif RB_LD_HINT == 2
+#define RB_LD_V8 "ld.global.nc.L1::no_allocate.L2::evict_first.v8.u32"
+#else
+#define RB_LD_V8 "ld.global.nc.L1::no_allocate.v8.u32"
+#endif
 __device__ __forceinline__ void ld_v8(const void* p, uint32_t (&r)[8]) {
-  asm("ld.global.nc.L1::no_allocate.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+  asm(RB_LD_V8 " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
       : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7])
       : "l"(p));
 }
