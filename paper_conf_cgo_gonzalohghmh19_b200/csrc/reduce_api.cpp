@@ -444,8 +444,9 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   if (opts) {
     if (opts->block != 0 && (opts->block < 32 || opts->block > 512 || opts->block % 32 != 0))
       return fail(REDUCE_ERR_INVALID_ARG, "segmented block must be 0 or a multiple of 32 in [32, 512]");
-    if (opts->seg_group < 0 || opts->seg_group > 5) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0..5");
+    if (opts->seg_group < 0 || opts->seg_group > 6) return fail(REDUCE_ERR_INVALID_ARG, "seg_group must be 0..6");
     if (opts->seg_group == 5 && uniform) return fail(REDUCE_ERR_INVALID_ARG, "seg_group 5 (balanced) needs an offsets array");
+    if (opts->seg_group == 6 && !uniform) return fail(REDUCE_ERR_INVALID_ARG, "seg_group 6 (tiled rows) is for reduce_batched");
     if (opts->block) block = opts->block;
     group = opts->seg_group;
   }
@@ -470,6 +471,26 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   }
   if (group == 5) group = 3;
   const unsigned long long row_bytes = (unsigned long long)seg_len * (unsigned long long)s;
+  // uniform rows of 1, 2, 4, 8, 16 or 32 KB on 32-byte boundaries: the flat
+  // kernel's 32 KB tile walk (k_rows_tiled); seg_group 6 asks for it, auto takes
+  // it unless REDUCE_NO_ROWS_TILED=1
+  int tiled_lv = -1;
+  if (uniform && in != nullptr && ((uintptr_t)in % 32u) == 0)
+    for (int lv = 0; lv <= 5; ++lv)
+      if (row_bytes == (1024ull << lv)) tiled_lv = lv;
+  if (group == 6 && tiled_lv < 0)
+    return fail(REDUCE_ERR_INVALID_ARG, "seg_group 6 needs 32-byte-aligned rows of 1, 2, 4, 8, 16 or 32 KB");
+  if (tiled_lv >= 0 && (group == 6 || (group == 0 && rows_tiled_enabled()))) {
+    SegParams p{};
+    p.in = (const char*)in;
+    p.seg_len = (long long)seg_len;
+    p.nseg = (long long)nseg;
+    p.out = out;
+    p.rows_tiled = 1 + tiled_lv;
+    cudaError_t e = launch_segmented(dtype, op, p, 0, 0, (cudaStream_t)stream);
+    if (e != cudaSuccess) return cuda_fail(e, "segmented reduction launch");
+    return REDUCE_OK;
+  }
   if (group == 0)
     group = !uniform ? 3 : (row_bytes <= 512 ? 4 : (row_bytes <= 4096 ? 3 : (row_bytes <= 16384 ? 1 : 2)));
   const int lanes = group == 1 ? 32 : (group == 3 ? 8 : (group == 4 ? 1 : 0));

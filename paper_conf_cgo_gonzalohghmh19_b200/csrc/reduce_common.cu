@@ -51,6 +51,14 @@ bool early_enabled() {
   return on;
 }
 
+bool rows_tiled_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("REDUCE_NO_ROWS_TILED");
+    return !(e && e[0] == '1');
+  }();
+  return on;
+}
+
 int grid_value_bytes(int dtype, int op) {
   if (dtype == 0) return 4;                                // int32: uint32 / int32
   if (dtype == 1) return (op == 0 || op == 3) ? 8 : 4;     // fp32: double sums / uint32 key

@@ -149,6 +149,8 @@ struct SegParams {
   SegQueue q;
   int rows_nv;               // > 0: uniform 32-byte-aligned rows of rows_nv (<= 8) vectors, one
                              //      thread per row with all its loads in flight (k_rows_aligned)
+  int rows_tiled;            // 1 + LV > 0: uniform 32-byte-aligned rows of 32 << LV vectors
+                             //      (1-32 KB), the flat tile walk (k_rows_tiled)
   int balanced;              // 1: element-balanced chunks (offsets arrays, reduce_segbal.cuh)
   SegBal b;
 };
@@ -198,6 +200,8 @@ bool pdl_enabled();
 // Loads of the input before the programmatic dependency resolves (default on;
 // REDUCE_NO_EARLY=1 turns it off, for A/B measurements).
 bool early_enabled();
+// REDUCE_NO_ROWS_TILED=1: reduce_batched's auto choice skips k_rows_tiled
+bool rows_tiled_enabled();
 
 constexpr int kCombos = 12;  // 3 dtypes x 4 ops (sum, min, max, accurate sum)
 constexpr int combo_index(int dtype, int op) { return dtype * 4 + op; }

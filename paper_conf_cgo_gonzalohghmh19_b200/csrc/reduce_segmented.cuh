@@ -496,6 +496,74 @@ cudaError_t launch_rows_aligned(const SegParams& p, int sms, cudaStream_t s) {
   return seg_launch(k_rows_aligned<DT, OP, NV>, grid < 1 ? 1 : grid, RB_ROWS_BLOCK, p, s);
 }
 
+// Uniform rows of 1, 2, 4, 8, 16 or 32 KB (L = 32 << LV vectors) on 32-byte
+// boundaries: the flat kernel's tile walk over the batch.  Block b reads the
+// contiguous 32 KB tile b exactly as k_reduce does (256 threads x 4 loads of
+// 256 bits, all in flight); each warp-load of 32 vectors lies inside one row,
+// so every (load, warp) pair is warp-reduced on its own, the tile's 32
+// warp-vector partials meet in shared memory, and warp 0 combines each row's
+// WPR = L / 32 consecutive partials with a butterfly of width WPR (fixed tree,
+// deterministic, no atomics).  The tile holds 32 / WPR whole rows.
+template <int DT, int OP, int LV>
+__global__ void __launch_bounds__(256) k_rows_tiled(const SegParams p) {
+  using T = Tr<DT, OP>;
+  using Acc = typename T::Acc;
+  constexpr int U = 4, B = 256, WPR = 1 << LV;
+  constexpr long long kTile = (long long)U * B;  // vectors
+  __shared__ Acc part[U * (B / 32)];
+  pdl_wait();
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const long long total = p.nseg << (5 + LV);  // vectors in the batch
+#pragma unroll 1
+  for (long long tile = blockIdx.x; tile * kTile < total; tile += gridDim.x) {
+    const long long left = total - tile * kTile;  // a multiple of 32: whole warp-loads only
+    const char* base = p.in + (tile * kTile + threadIdx.x) * kVecBytes;
+    uint32_t r[U][8];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if ((long long)(u * B + threadIdx.x) < left) ld_v8(base + (size_t)u * B * kVecBytes, r[u]);
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      Part<T> a[T::NA];
+      init_parts<T>(a);
+      uint32_t aux = 0;
+      if ((long long)(u * B + threadIdx.x) < left) fold_vec<T>(a, aux, r[u], 0);
+      const Acc w = T::warp(thread_result<T>(a, aux));
+      if (lane == 0) part[u * (B / 32) + wid] = w;
+    }
+    __syncthreads();
+    if (wid == 0) {
+      Acc x = part[lane];
+#pragma unroll
+      for (int o = WPR / 2; o > 0; o >>= 1) x = T::comb(x, shfl_xor(x, o));
+      const long long row = (tile << (5 - LV)) + (lane >> LV);
+      if ((lane & (WPR - 1)) == 0 && row < p.nseg) seg_store<T>(p, row, T::to_grid(x));
+    }
+    __syncthreads();  // part[] is reused by the next tile
+  }
+  pdl_trigger();
+}
+
+template <int DT, int OP, int LV>
+cudaError_t launch_rows_tiled_lv(const SegParams& p, cudaStream_t s) {
+  const long long tiles = (p.nseg + (32 >> LV) - 1) >> (5 - LV);  // one block per 32 KB tile
+  const long long grid = tiles < (1ll << 30) ? tiles : (1ll << 30);
+  return seg_launch(k_rows_tiled<DT, OP, LV>, grid < 1 ? 1 : grid, 256, p, s);
+}
+
+template <int DT, int OP>
+cudaError_t launch_rows_tiled(const SegParams& p, cudaStream_t s) {
+  switch (p.rows_tiled - 1) {
+    case 0: return launch_rows_tiled_lv<DT, OP, 0>(p, s);
+    case 1: return launch_rows_tiled_lv<DT, OP, 1>(p, s);
+    case 2: return launch_rows_tiled_lv<DT, OP, 2>(p, s);
+    case 3: return launch_rows_tiled_lv<DT, OP, 3>(p, s);
+    case 4: return launch_rows_tiled_lv<DT, OP, 4>(p, s);
+    case 5: return launch_rows_tiled_lv<DT, OP, 5>(p, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
 template <class K>
 cudaError_t seg_launch(K kernel, long long grid, int block, const SegParams& p, cudaStream_t s) {
   cudaLaunchConfig_t cfg = {};
@@ -534,6 +602,7 @@ cudaError_t launch_segmented_op(const SegParams& p, int group, int block, cudaSt
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (p.rows_tiled > 0) return launch_rows_tiled<DT, OP>(p, s);
   if (p.rows_nv > 0) {
     if constexpr (OP != OP_SUMACC) {  // several rows per thread: the accurate pairs would not fit
       if (p.rows_nv == 1) return launch_rows_aligned<DT, OP, 1>(p, sms, s);

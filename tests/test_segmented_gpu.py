@@ -239,3 +239,55 @@ def test_batched_aligned_short_rows_vs_misaligned(dtype):
             for op in OPS:
                 got = rb.reduce_batched(xt, op).cpu().numpy()
                 _check_segments(x[off:off + rows * cols], [(r * cols, (r + 1) * cols) for r in range(rows)], op, got, 1)
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("row_kb,rows", [(1, 1), (1, 33), (2, 4099), (4, 17), (4, 1000), (8, 9), (16, 5), (32, 3),
+                                         (32, 40)])
+def test_batched_tiled_rows(dtype, row_kb, rows):
+    """seg_group 6 (k_rows_tiled): 32 KB tiles of whole 1-32 KB rows, including
+    a partial last tile; bit-exact (int32, min/max) or G1 + G2 (fp sums) per row,
+    the auto choice identical, the fixed tree reproducible, special values."""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    s = np.dtype(NP[dtype]).itemsize
+    cols = row_kb * 1024 // s
+    x = synth.make(dtype, rows * cols, "int_full" if dtype == "int32" else "uniform_pm1", 31 * row_kb + rows)
+    if dtype != "int32" and rows > 3:
+        x[cols + 5] = np.nan          # row 1: NaN
+        x[2 * cols + 7] = -np.inf     # row 2: -inf
+        x[3 * cols:4 * cols] = 0.0
+        x[3 * cols + 2] = -0.0        # row 3: all zeros with one -0.0
+    xt = torch.from_numpy(x).cuda().view(rows, cols)
+    bounds = [(r * cols, (r + 1) * cols) for r in range(rows)]
+    ops = OPS + (["sum_accurate"] if dtype != "int32" else [])
+    for op in ops:
+        got = rb.reduce_batched(xt, op, seg_group=6).cpu().numpy()
+        if op == "sum_accurate":  # the exact sum and test_accurate_gpu's gate (chain <= 64)
+            from oracle import ref as exact
+            from tests.test_accurate_gpu import _gate
+            for i, (lo, hi) in enumerate(bounds):
+                S = exact.sum_fp(x[lo:hi])
+                r = float(got[i])
+                if not math.isfinite(S):
+                    assert (math.isnan(S) and math.isnan(r)) or r == S, (i, r, S)
+                else:
+                    assert abs(r - S) <= _gate(dtype, S, exact.abs_sum(x[lo:hi]), 64), (op, i, r, S)
+        else:
+            _check_segments(x, bounds, op, got, 32)
+        again = rb.reduce_batched(xt, op, seg_group=6).cpu().numpy()
+        auto = rb.reduce_batched(xt, op).cpu().numpy()
+        assert got.tobytes() == again.tobytes() == auto.tobytes(), op
+
+
+def test_batched_tiled_rows_rejects_ineligible():
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    x = torch.zeros(64 * 1024 + 8, dtype=torch.float32, device="cuda")
+    with pytest.raises(rb.ReduceError):  # 3 KB rows
+        rb.reduce_batched(x[:48 * 768].view(48, 768), "sum", seg_group=6)
+    with pytest.raises(rb.ReduceError):  # misaligned start
+        rb.reduce_batched(x[1:1 + 64 * 256].view(64, 256), "sum", seg_group=6)
+    # ineligible rows under auto still take the group kernels
+    got = rb.reduce_batched(x[1:1 + 64 * 256].view(64, 256), "sum").cpu().numpy()
+    assert (got == 0).all()
