@@ -478,15 +478,25 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   if (uniform && in != nullptr && ((uintptr_t)in % 32u) == 0)
     for (int lv = 0; lv <= 5; ++lv)
       if (row_bytes == (1024ull << lv)) tiled_lv = lv;
-  if (group == 6 && tiled_lv < 0)
-    return fail(REDUCE_ERR_INVALID_ARG, "seg_group 6 needs 32-byte-aligned rows of 1, 2, 4, 8, 16 or 32 KB");
-  if (tiled_lv >= 0 && (group == 6 || (group == 0 && rows_tiled_enabled()))) {
+  // longer rows of whole 32 KB tiles, when there are enough of them to fill the
+  // GPU with one block per row (B200 A/B, profiles/r01_rows_big_ab.jsonl: 0-19 %
+  // faster from 2048 rows, up to 7 % slower at 1024 rows of 256 KB, where the
+  // group kernels and the chunk queue keep their place)
+  long long tiled_big = 0;
+  if (uniform && in != nullptr && ((uintptr_t)in % 32u) == 0 && row_bytes >= (64u << 10) &&
+      row_bytes % (32u << 10) == 0 && nseg >= 2048)
+    tiled_big = (long long)(row_bytes / 32u);
+  if (group == 6 && tiled_lv < 0 && tiled_big == 0)
+    return fail(REDUCE_ERR_INVALID_ARG, "seg_group 6 needs 32-byte-aligned rows of 1, 2, 4, 8, 16 or 32 KB, "
+                                        "or >= 2048 rows of a multiple of 32 KB");
+  if ((tiled_lv >= 0 || tiled_big > 0) && (group == 6 || (group == 0 && rows_tiled_enabled()))) {
     SegParams p{};
     p.in = (const char*)in;
     p.seg_len = (long long)seg_len;
     p.nseg = (long long)nseg;
     p.out = out;
-    p.rows_tiled = 1 + tiled_lv;
+    p.rows_tiled = tiled_lv >= 0 ? 1 + tiled_lv : 7;
+    p.rows_tiled_vecs = tiled_lv >= 0 ? 0 : tiled_big;
     cudaError_t e = launch_segmented(dtype, op, p, 0, 0, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "segmented reduction launch");
     return REDUCE_OK;

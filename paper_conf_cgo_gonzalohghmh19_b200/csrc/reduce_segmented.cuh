@@ -544,6 +544,38 @@ __global__ void __launch_bounds__(256) k_rows_tiled(const SegParams p) {
   pdl_trigger();
 }
 
+// Uniform rows of a whole number (>= 2) of 32 KB tiles, 32-byte aligned, and
+// enough rows to fill the GPU (host side): one block per row walks the row's
+// tiles with k_reduce's access pattern (4 loads of 256 bits per thread in
+// flight), then the "Vs" block combine.  Rows beyond the grid are strided.
+template <int DT, int OP>
+__global__ void __launch_bounds__(256) k_rows_tiled_big(const SegParams p) {
+  using T = Tr<DT, OP>;
+  constexpr int U = 4, B = 256;
+  constexpr long long kTile = (long long)U * B;  // vectors
+  pdl_wait();
+  const long long row_vecs = (long long)p.rows_tiled_vecs;
+#pragma unroll 1
+  for (long long row = blockIdx.x; row < p.nseg; row += gridDim.x) {
+    Part<T> a[T::NA];
+    init_parts<T>(a);
+    uint32_t aux = 0;
+    const char* base = p.in + (row * row_vecs + threadIdx.x) * kVecBytes;
+#pragma unroll 1
+    for (long long v = 0; v < row_vecs; v += kTile) {
+      uint32_t r[U][8];
+#pragma unroll
+      for (int u = 0; u < U; ++u) ld_v8(base + (v + (long long)u * B) * kVecBytes, r[u]);
+#pragma unroll
+      for (int u = 0; u < U; ++u) fold_vec<T>(a, aux, r[u], u);
+    }
+    const typename T::Grid g = block_combine<T, BC_SHFL>(thread_result<T>(a, aux));
+    if (threadIdx.x == 0) seg_store<T>(p, row, g);
+    __syncthreads();  // block_combine's shared scratch is reused by the next row
+  }
+  pdl_trigger();
+}
+
 template <int DT, int OP, int LV>
 cudaError_t launch_rows_tiled_lv(const SegParams& p, cudaStream_t s) {
   const long long tiles = (p.nseg + (32 >> LV) - 1) >> (5 - LV);  // one block per 32 KB tile
@@ -553,6 +585,10 @@ cudaError_t launch_rows_tiled_lv(const SegParams& p, cudaStream_t s) {
 
 template <int DT, int OP>
 cudaError_t launch_rows_tiled(const SegParams& p, cudaStream_t s) {
+  if (p.rows_tiled_vecs > 0) {
+    const long long grid = p.nseg < (1ll << 30) ? p.nseg : (1ll << 30);
+    return seg_launch(k_rows_tiled_big<DT, OP>, grid, 256, p, s);
+  }
   switch (p.rows_tiled - 1) {
     case 0: return launch_rows_tiled_lv<DT, OP, 0>(p, s);
     case 1: return launch_rows_tiled_lv<DT, OP, 1>(p, s);

@@ -243,7 +243,7 @@ def test_batched_aligned_short_rows_vs_misaligned(dtype):
 
 @pytest.mark.parametrize("dtype", DTYPES)
 @pytest.mark.parametrize("row_kb,rows", [(1, 1), (1, 33), (2, 4099), (4, 17), (4, 1000), (8, 9), (16, 5), (32, 3),
-                                         (32, 40)])
+                                         (32, 40), (64, 2048), (96, 2051)])
 def test_batched_tiled_rows(dtype, row_kb, rows):
     """seg_group 6 (k_rows_tiled): 32 KB tiles of whole 1-32 KB rows, including
     a partial last tile; bit-exact (int32, min/max) or G1 + G2 (fp sums) per row,
@@ -286,6 +286,8 @@ def test_batched_tiled_rows_rejects_ineligible():
     x = torch.zeros(64 * 1024 + 8, dtype=torch.float32, device="cuda")
     with pytest.raises(rb.ReduceError):  # 3 KB rows
         rb.reduce_batched(x[:48 * 768].view(48, 768), "sum", seg_group=6)
+    with pytest.raises(rb.ReduceError):  # rows of whole 32 KB tiles, but too few of them
+        rb.reduce_batched(x[:4 * 16384].view(4, 16384), "sum", seg_group=6)
     with pytest.raises(rb.ReduceError):  # misaligned start
         rb.reduce_batched(x[1:1 + 64 * 256].view(64, 256), "sum", seg_group=6)
     # ineligible rows under auto still take the group kernels
