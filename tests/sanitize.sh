@@ -46,6 +46,16 @@ for dt in (torch.int32, torch.float32, torch.float64):
         rb.reduce_batched(abase[: rows * nvv * ve].view(rows, nvv * ve), "max")
         if dt != torch.int32:
             rb.reduce_batched(abase[: rows * nvv * ve].view(rows, nvv * ve), "sum_accurate")
+    # tiled rows (k_rows_tiled: 1 KB and 32 KB rows, partial last tile;
+    # k_rows_tiled_big: 2048 rows of 64 KB)
+    tbase = torch.arange(2048 * 64 * 1024 // 4 + 64, device="cuda").to(dt)[:2048 * 64 * 1024 // dt.itemsize]
+    for kb, rows in ((1, 33), (32, 3)):
+        cols = kb * 1024 // dt.itemsize
+        for op in ("sum", "max") + (("sum_accurate",) if dt != torch.int32 else ()):
+            rb.reduce_batched(tbase[:rows * cols].view(rows, cols), op, seg_group=6)
+    rb.reduce_batched(tbase.view(2048, -1), "min", seg_group=6)
+    if dt != torch.int32:
+        rb.reduce_batched(tbase.view(2048, -1), "sum_accurate", seg_group=6)
     for g in (0, 1, 2, 3, 4):
         rb.reduce_segmented(base, offs, "sum", seg_group=g)
         rb.reduce_batched(base[:4096].view(64, 64), "max", seg_group=g)
