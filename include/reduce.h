@@ -145,12 +145,13 @@ typedef struct {
                          fewer than 4096 uniform rows of > 64 KB) are cut into chunks
                          of >= 16 KB that warps reduce (two more launches);
                          6 = tiled rows (reduce_batched only; 32-byte-aligned input,
-                         rows of exactly 1, 2, 4, 8, 16 or 32 KB, or >= 2048 rows of
+                         rows of 32 B times a power of two up to 32 KB, or >= 2048 rows of
                          a multiple of 32 KB, else REDUCE_ERR_INVALID_ARG): each block
                          reads one contiguous 32 KB tile of whole rows, warp-loads are
                          reduced per row and combined in a fixed tree (longer rows: one
                          block per row walking its tiles) -- auto picks it for such
-                         rows unless REDUCE_NO_ROWS_TILED=1 */
+                         rows (except accurate fp32 sums of 128-512 B rows) unless
+                         REDUCE_NO_ROWS_TILED=1 */
   int stage;          /* 0 = auto; REDUCE_STAGE_REG: 256-bit loads straight into
                          registers; REDUCE_STAGE_SMEM: cp.async 16-byte copies into a
                          shared-memory tile (block*unroll*32 <= 128 KiB), then shared

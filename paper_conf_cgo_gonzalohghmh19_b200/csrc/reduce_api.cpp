@@ -426,6 +426,11 @@ int reduce_ex(int dtype, int op, const void* in, size_t n, void* out, reduce_str
   return launch_plan(&P, ws, out, (cudaStream_t)stream, /*allow_early=*/true);
 }
 
+#ifndef RB_TILED_AUTO_MIN_LV
+#define RB_TILED_AUTO_MIN_LV (-5)
+#endif
+static constexpr int kTiledAutoMinLv = RB_TILED_AUTO_MIN_LV;
+
 static int segmented_common(int dtype, int op, const void* in, const int64_t* offsets, size_t seg_len,
                             size_t nseg, void* out, reduce_stream_t stream, const reduce_opts_t* opts) {
   if (dtype < 0 || dtype > 2) return fail(REDUCE_ERR_INVALID_ARG, "dtype must be REDUCE_INT32/FLOAT32/FLOAT64");
@@ -471,13 +476,13 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   }
   if (group == 5) group = 3;
   const unsigned long long row_bytes = (unsigned long long)seg_len * (unsigned long long)s;
-  // uniform rows of 1, 2, 4, 8, 16 or 32 KB on 32-byte boundaries: the flat
+  // uniform rows of 32 B x 2^k (up to 32 KB) on 32-byte boundaries: the flat
   // kernel's 32 KB tile walk (k_rows_tiled); seg_group 6 asks for it, auto takes
   // it unless REDUCE_NO_ROWS_TILED=1
-  int tiled_lv = -1;
+  int tiled_lv = -6;  // log2(row vectors) - 5 of an eligible row, -6: none
   if (uniform && in != nullptr && ((uintptr_t)in % 32u) == 0)
-    for (int lv = 0; lv <= 5; ++lv)
-      if (row_bytes == (1024ull << lv)) tiled_lv = lv;
+    for (int lv = -5; lv <= 5; ++lv)
+      if (row_bytes == (32ull << (lv + 5))) tiled_lv = lv;
   // longer rows of whole 32 KB tiles, when there are enough of them to fill the
   // GPU with one block per row (B200 A/B, profiles/r01_rows_big_ab.jsonl: 0-19 %
   // faster from 2048 rows, up to 7 % slower at 1024 rows of 256 KB, where the
@@ -486,17 +491,23 @@ static int segmented_common(int dtype, int op, const void* in, const int64_t* of
   if (uniform && in != nullptr && ((uintptr_t)in % 32u) == 0 && row_bytes >= (64u << 10) &&
       row_bytes % (32u << 10) == 0 && nseg >= 2048)
     tiled_big = (long long)(row_bytes / 32u);
-  if (group == 6 && tiled_lv < 0 && tiled_big == 0)
-    return fail(REDUCE_ERR_INVALID_ARG, "seg_group 6 needs 32-byte-aligned rows of 1, 2, 4, 8, 16 or 32 KB, "
+  if (group == 6 && tiled_lv < -5 && tiled_big == 0)
+    return fail(REDUCE_ERR_INVALID_ARG, "seg_group 6 needs 32-byte-aligned rows of 32 B x 2^k up to 32 KB, "
                                         "or >= 2048 rows of a multiple of 32 KB");
-  if ((tiled_lv >= 0 || tiled_big > 0) && (group == 6 || (group == 0 && rows_tiled_enabled()))) {
+  // auto: rows of >= 2^(kTiledAutoMinLv + 5) vectors (measured: profiles/r01_rows_tiled_ab.jsonl,
+  // profiles/r01_rows_small_ab.jsonl)
+  // (every row size wins 1.05-1.75x, except accurate fp32 sums of 128-512 B rows:
+  // 0.94-0.96x, those keep the one-thread-per-row kernel)
+  const bool acc_f32_mid = op == REDUCE_SUM_ACCURATE && dtype == REDUCE_FLOAT32 && tiled_lv >= -3 && tiled_lv <= -1;
+  const bool auto_tiled = ((tiled_lv >= kTiledAutoMinLv && !acc_f32_mid) || tiled_big > 0) && rows_tiled_enabled();
+  if ((tiled_lv >= -5 || tiled_big > 0) && (group == 6 || (group == 0 && auto_tiled))) {
     SegParams p{};
     p.in = (const char*)in;
     p.seg_len = (long long)seg_len;
     p.nseg = (long long)nseg;
     p.out = out;
-    p.rows_tiled = tiled_lv >= 0 ? 1 + tiled_lv : 7;
-    p.rows_tiled_vecs = tiled_lv >= 0 ? 0 : tiled_big;
+    p.rows_tiled = tiled_lv >= -5 ? 6 + tiled_lv : 12;
+    p.rows_tiled_vecs = tiled_lv >= -5 ? 0 : tiled_big;
     cudaError_t e = launch_segmented(dtype, op, p, 0, 0, (cudaStream_t)stream);
     if (e != cudaSuccess) return cuda_fail(e, "segmented reduction launch");
     return REDUCE_OK;

@@ -149,8 +149,8 @@ struct SegParams {
   SegQueue q;
   int rows_nv;               // > 0: uniform 32-byte-aligned rows of rows_nv (<= 8) vectors, one
                              //      thread per row with all its loads in flight (k_rows_aligned)
-  int rows_tiled;            // 1 + LV > 0: uniform 32-byte-aligned rows of 32 << LV vectors
-                             //      (1-32 KB), the flat tile walk (k_rows_tiled)
+  int rows_tiled;            // 6 + LV > 0: uniform 32-byte-aligned rows of 32 << LV vectors
+                             //      (LV = -5..5: 32 B-32 KB), the flat tile walk (k_rows_tiled)
   long long rows_tiled_vecs; // > 0 (with rows_tiled > 0): rows of this many vectors, a multiple
                              //      of 1024 (32 KB tiles), one block per row (k_rows_tiled_big)
   int balanced;              // 1: element-balanced chunks (offsets arrays, reduce_segbal.cuh)

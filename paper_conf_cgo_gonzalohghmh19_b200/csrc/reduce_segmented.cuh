@@ -503,12 +503,14 @@ cudaError_t launch_rows_aligned(const SegParams& p, int sms, cudaStream_t s) {
 // so every (load, warp) pair is warp-reduced on its own, the tile's 32
 // warp-vector partials meet in shared memory, and warp 0 combines each row's
 // WPR = L / 32 consecutive partials with a butterfly of width WPR (fixed tree,
-// deterministic, no atomics).  The tile holds 32 / WPR whole rows.
+// deterministic, no atomics).  The tile holds 32 / WPR whole rows.  LV < 0:
+// rows of 1-16 vectors (32-512 bytes), 32 / L rows per warp-load, each reduced
+// by a butterfly of width L and stored by its first lane (no shared memory).
 template <int DT, int OP, int LV>
 __global__ void __launch_bounds__(256) k_rows_tiled(const SegParams p) {
   using T = Tr<DT, OP>;
   using Acc = typename T::Acc;
-  constexpr int U = 4, B = 256, WPR = 1 << LV;
+  constexpr int U = 4, B = 256, WPR = LV >= 0 ? 1 << LV : 1;
   constexpr long long kTile = (long long)U * B;  // vectors
   __shared__ Acc part[U * (B / 32)];
   pdl_wait();
@@ -516,7 +518,7 @@ __global__ void __launch_bounds__(256) k_rows_tiled(const SegParams p) {
   const long long total = p.nseg << (5 + LV);  // vectors in the batch
 #pragma unroll 1
   for (long long tile = blockIdx.x; tile * kTile < total; tile += gridDim.x) {
-    const long long left = total - tile * kTile;  // a multiple of 32: whole warp-loads only
+    const long long left = total - tile * kTile;  // a multiple of the row length
     const char* base = p.in + (tile * kTile + threadIdx.x) * kVecBytes;
     uint32_t r[U][8];
 #pragma unroll
@@ -527,19 +529,31 @@ __global__ void __launch_bounds__(256) k_rows_tiled(const SegParams p) {
       Part<T> a[T::NA];
       init_parts<T>(a);
       uint32_t aux = 0;
-      if ((long long)(u * B + threadIdx.x) < left) fold_vec<T>(a, aux, r[u], 0);
-      const Acc w = T::warp(thread_result<T>(a, aux));
-      if (lane == 0) part[u * (B / 32) + wid] = w;
-    }
-    __syncthreads();
-    if (wid == 0) {
-      Acc x = part[lane];
+      const bool valid = (long long)(u * B + threadIdx.x) < left;
+      if (valid) fold_vec<T>(a, aux, r[u], 0);
+      if constexpr (LV < 0) {
+        // rows of 1-16 vectors: 32 / L rows per warp-load, a butterfly of width L
+        Acc w = thread_result<T>(a, aux);
 #pragma unroll
-      for (int o = WPR / 2; o > 0; o >>= 1) x = T::comb(x, shfl_xor(x, o));
-      const long long row = (tile << (5 - LV)) + (lane >> LV);
-      if ((lane & (WPR - 1)) == 0 && row < p.nseg) seg_store<T>(p, row, T::to_grid(x));
+        for (int o = (1 << (LV + 5)) / 2; o > 0; o >>= 1) w = T::comb(w, shfl_xor(w, o));
+        if (valid && (lane & ((1 << (LV + 5)) - 1)) == 0)
+          seg_store<T>(p, (tile * kTile + u * B + threadIdx.x) >> (LV + 5), T::to_grid(w));
+      } else {
+        const Acc w = T::warp(thread_result<T>(a, aux));
+        if (lane == 0) part[u * (B / 32) + wid] = w;
+      }
     }
-    __syncthreads();  // part[] is reused by the next tile
+    if constexpr (LV >= 0) {
+      __syncthreads();
+      if (wid == 0) {
+        Acc x = part[lane];
+#pragma unroll
+        for (int o = WPR / 2; o > 0; o >>= 1) x = T::comb(x, shfl_xor(x, o));
+        const long long row = (tile << (5 - LV)) + (lane >> LV);
+        if ((lane & (WPR - 1)) == 0 && row < p.nseg) seg_store<T>(p, row, T::to_grid(x));
+      }
+      __syncthreads();  // part[] is reused by the next tile
+    }
   }
   pdl_trigger();
 }
@@ -578,7 +592,7 @@ __global__ void __launch_bounds__(256) k_rows_tiled_big(const SegParams p) {
 
 template <int DT, int OP, int LV>
 cudaError_t launch_rows_tiled_lv(const SegParams& p, cudaStream_t s) {
-  const long long tiles = (p.nseg + (32 >> LV) - 1) >> (5 - LV);  // one block per 32 KB tile
+  const long long tiles = ((p.nseg << (5 + LV)) + 1023) >> 10;  // one block per 32 KB tile
   const long long grid = tiles < (1ll << 30) ? tiles : (1ll << 30);
   return seg_launch(k_rows_tiled<DT, OP, LV>, grid < 1 ? 1 : grid, 256, p, s);
 }
@@ -589,7 +603,12 @@ cudaError_t launch_rows_tiled(const SegParams& p, cudaStream_t s) {
     const long long grid = p.nseg < (1ll << 30) ? p.nseg : (1ll << 30);
     return seg_launch(k_rows_tiled_big<DT, OP>, grid, 256, p, s);
   }
-  switch (p.rows_tiled - 1) {
+  switch (p.rows_tiled - 6) {  // LV = log2(row vectors) - 5
+    case -5: return launch_rows_tiled_lv<DT, OP, -5>(p, s);
+    case -4: return launch_rows_tiled_lv<DT, OP, -4>(p, s);
+    case -3: return launch_rows_tiled_lv<DT, OP, -3>(p, s);
+    case -2: return launch_rows_tiled_lv<DT, OP, -2>(p, s);
+    case -1: return launch_rows_tiled_lv<DT, OP, -1>(p, s);
     case 0: return launch_rows_tiled_lv<DT, OP, 0>(p, s);
     case 1: return launch_rows_tiled_lv<DT, OP, 1>(p, s);
     case 2: return launch_rows_tiled_lv<DT, OP, 2>(p, s);

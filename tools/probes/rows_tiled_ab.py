@@ -1,8 +1,8 @@
 """A/B: reduce_batched on 256 MB of uniform rows of 1-32 KB -- the tiled-rows
 kernel (seg_group 6) against the group kernel the auto choice used before it
-(8 lanes <= 4 KB, one warp <= 16 KB, one block above; rows of >= 64 KB:
+(one thread <= 512 B, 8 lanes <= 4 KB, one warp <= 16 KB, one block above; rows of >= 64 KB:
 one block per row, k_rows_tiled_big, needs >= 1024 rows).  Graph of R calls over
-disjoint cold regions (tools/cudatiming.py).  Usage: python tools/probes/rows_tiled_ab.py [kb,kb,...]"""
+disjoint cold regions (tools/cudatiming.py).  Usage: python tools/probes/rows_tiled_ab.py [row_bytes,row_bytes,...]"""
 import json
 import os
 import sys
@@ -17,17 +17,18 @@ from cudatiming import time_calls, disjoint_regions  # noqa: E402
 dev = torch.device("cuda", 0)
 stream = torch.cuda.Stream(dev)
 TOTAL = 256 << 20
-KBS = [int(k) for k in sys.argv[1].split(',')] if len(sys.argv) > 1 else [1, 2, 4, 8, 16, 32, 64, 128, 256]
+SIZES = [int(k) for k in sys.argv[1].split(',')] if len(sys.argv) > 1 else [1 << k for k in range(5, 19)]  # row bytes
 for dtype, ops in (("float32", ("sum", "max", "sum_accurate")), ("int32", ("sum",)), ("float64", ("sum", "min"))):
     es = 8 if dtype == "float64" else 4
     pool = torch.empty((2 << 30) // es, dtype=getattr(torch, dtype), device=dev)
     pool.random_(-1000, 1000) if dtype == "int32" else pool.uniform_(-1, 1)
     rb.prepare(stream, pool.numel())
     for op in ops:
-        for kb in KBS:
-            cols = kb * 1024 // es
-            rows = TOTAL // (kb * 1024)
-            old = 3 if kb <= 4 else (1 if kb <= 16 else 2)
+        for nbytes in SIZES:
+            kb = nbytes / 1024
+            cols = nbytes // es
+            rows = TOTAL // nbytes
+            old = 4 if nbytes <= 512 else (3 if nbytes <= 4096 else (1 if nbytes <= 16384 else 2))
             warm, timed = disjoint_regions(pool, 6, rows * cols, align_elems=256)
             outs = torch.empty(rows, dtype=pool.dtype, device=dev)
             row = {"dtype": dtype, "op": op, "row_kb": kb, "rows": rows}
