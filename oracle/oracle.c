@@ -149,7 +149,11 @@ uint64_t oracle_max_f64_bits(const double* x, size_t n) {
  *          (the quotient in double, then rounded to float); x counted iff
  *          lo_f <= x < hi_f and 0 <= b < nbins with
  *          b = floor(fl32(fl32(x - lo_f) * scale))   (two fp32 RN operations).
- * NaN is never counted.  counts is overwritten. */
+ * NaN is never counted.  counts is overwritten.
+ * The fp32 rule is a definition chosen for the kernel (the paper defines no
+ * bin rule); tests/test_oracle.py pins it element by element against the
+ * exact-rational bins of oracle/ref.py: they differ only within the rule's
+ * rounding reach of a bin edge. */
 void oracle_histogram_i32(const int32_t* x, size_t n, double lo, double hi, int nbins, uint32_t* counts) {
   for (int b = 0; b < nbins; ++b) counts[b] = 0u;
   const long long l = (long long)lo, h = (long long)hi;

@@ -6,6 +6,7 @@ from __future__ import annotations
 import numpy as np
 
 import oracle
+from tests._chain import checked_chain
 
 NP = {"int32": np.int32, "float32": np.float32, "float64": np.float64}
 BITS = {"int32": np.uint32, "float32": np.uint32, "float64": np.uint64}
@@ -46,6 +47,8 @@ def check(x: np.ndarray, op: str, got: np.ndarray, plan: dict | None = None, gat
         gb = int(got.view(BITS[dt])[0])
         assert gb == ref.bits, f"{dt} {op} n={x.size}: got bits {gb:#x} want {ref.bits:#x} ({got[0]!r} vs {ref.value!r})"
         return
-    chain = plan["chain"] if (plan is not None and "g2" in gates) else None
+    # G2's L comes from the test-side formula over the plan's launch shape
+    # (tests/_chain.py), never from the library's own plan["chain"]
+    chain = checked_chain(dt, op, plan) if (plan is not None and "g2" in gates) else None
     ok, msg = oracle.check_sum(float(got[0]), ref, x.dtype, x.size, chain=chain)
     assert ok, f"{dt} sum n={x.size}: {msg} plan={plan}"

@@ -4,7 +4,7 @@ checked against the EXACT sum (math.fsum via oracle/ref.py):
 |r - S| <= u|S| + E*sum|x| with u the output unit roundoff and E the
 accumulation error: (L+1)^2 * 2^-48 for fp32 (compensated fp32 chains of
 length <= L, then fp64), (L+1) * 2^-100 for double-double; L is the variant's
-chain length.  Plus cancellation pins a plain
+chain length (tests/_chain.py, computed from the launch shape).  Plus cancellation pins a plain
 sum fails, special values, every grid combine, segmented and host entry."""
 import math
 
@@ -15,6 +15,7 @@ from oracle import ref
 import oracle
 import synth
 from tests._util import to_device
+from tests._chain import checked_chain
 
 pytestmark = pytest.mark.gpu
 
@@ -37,7 +38,8 @@ def _check(x, r, plan):
         return
     A = ref.abs_sum(x)
     err = abs(float(r) - S)
-    assert err <= _gate(x.dtype.name, S, A, plan["chain"]), (x.dtype.name, x.size, r, S, err, plan)
+    L = checked_chain(x.dtype.name, "sum_accurate", plan)  # test-side chain, not the library's
+    assert err <= _gate(x.dtype.name, S, A, L), (x.dtype.name, x.size, r, S, err, L, plan)
 
 
 VARIANTS = [dict(), dict(mode="deterministic"), dict(grid_combine=0, block=256), dict(grid_combine=2),

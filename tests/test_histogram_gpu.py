@@ -1,6 +1,9 @@
 """Histogram on the GPU against oracle.histogram, bit-exact:
-both sides decide each bin in fp64 with the same three correctly rounded
-operations (R13).  Shared-memory and global-memory bin paths, ragged
+int32 bins are exact integer arithmetic on both sides; fp32 bins are decided
+in fp32 on both sides by the rule DESIGN.md R13 defines,
+floor(fl32(fl32(x - lo_f) * scale)) -- a definition chosen for the kernel (the
+paper only motivates histograms), itself pinned against the
+exact-rational bins on non-power-of-two grids by tests/test_oracle.py.  Shared-memory and global-memory bin paths, ragged
 head/tail, out-of-range values, NaN/inf, large inputs."""
 import numpy as np
 import pytest

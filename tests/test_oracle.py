@@ -273,3 +273,79 @@ def test_histogram_vs_exact_rational(dtype, nbins):
         assert c.tolist() == want
     assert int(c.sum()) == sum(want) == int(((x >= lo) & (x < hi)).sum())
     assert np.abs(c.astype(np.int64) - np.array(want)).sum() <= 2 * max(1, nbins // 100) + 2
+
+
+def _edge_distance_bound(p, lo, hi, nbins):
+    """Largest shift, in bin units, that the fp32 rule's roundings can give the
+    position p = (x - lo) * nbins / (hi - lo): lo_f = fl32(lo) moves the origin
+    by <= u|lo|, scale = fl32(nbins / (hi - lo)) is off by <= u * scale, and
+    fl32(x - lo_f), fl32(d * scale) each add <= u of their result (u = 2^-24);
+    doubled for slack in the products."""
+    u = 2.0 ** -24
+    scale = nbins / (hi - lo)
+    return 2 * (3 * u * (abs(p) + 1) + u * abs(lo) * scale) + 2.0 ** -40
+
+
+@pytest.mark.parametrize("lo,hi,nbins", [(0.0, 1.0, 7), (0.0, 1.0, 1000), (-3.7, 11.3, 257),
+                                         (0.1, 0.7, 100), (-1.0, 1.0, 65535), (1000.0, 1000.5, 3),
+                                         (-2.0 ** 20, 3.0, 12345)])
+def test_histogram_f32_rule_vs_exact_rational_per_element(lo, hi, nbins):
+    """oracle_histogram_f32 off power-of-two grids: its bin
+    rule floor(fl32(fl32(x - lo_f) * scale)) is a definition chosen for the
+    kernel (DESIGN R13), so it is pinned here against the exact-rational
+    definition floor((x - lo) * nbins / (hi - lo)) of oracle/ref.py element by
+    element: every element where the two disagree must sit within the fp32
+    rule's rounding reach of an integer bin edge (0, ..., nbins), and nowhere
+    else.  Inputs mix uniform values with values planted on both sides of
+    every kind of edge (the first few, some interior ones, lo and hi), so the
+    disagreements actually occur."""
+    from fractions import Fraction
+    rng = np.random.Generator(np.random.PCG64(nbins))
+    width = hi - lo
+    xs = list((lo - 0.05 * width + rng.random(1500) * 1.1 * width).astype(np.float32))
+    edges = list(range(0, min(nbins, 40) + 1)) + list(rng.integers(0, nbins + 1, 40)) + [nbins]
+    for k in edges:
+        e = np.float32(lo + width * int(k) / nbins)
+        for step in range(-3, 4):
+            v = e
+            for _ in range(abs(step)):
+                v = np.nextafter(v, np.float32(np.inf if step > 0 else -np.inf), dtype=np.float32)
+            xs.append(np.float32(v))
+    x = np.array(xs, np.float32)
+    flo, fw = Fraction(lo), Fraction(hi) - Fraction(lo)
+    disagree = 0
+    for v in x:
+        c = oracle.histogram(np.array([v], np.float32), lo, hi, nbins)
+        got = int(np.flatnonzero(c)[0]) if c.any() else None
+        p = (Fraction(float(v)) - flo) * nbins / fw
+        want = int(p // 1) if 0 <= p < nbins else None
+        if got == want:
+            continue
+        disagree += 1
+        dist = abs(float(p - round(p)))
+        assert dist <= _edge_distance_bound(float(p), lo, hi, nbins), (float(v), got, want, float(p), dist)
+        # a rounding moves x by at most one bin, never further
+        assert got is None or want is None or abs(got - want) == 1, (float(v), got, want)
+    assert disagree <= len(x) // 4
+    # the whole-array counts: the same totals up to the edge elements
+    c = oracle.histogram(x, lo, hi, nbins)
+    want = ref.histogram(x, lo, hi, nbins)
+    assert np.abs(c.astype(np.int64) - np.array(want)).sum() <= 2 * disagree
+
+
+def test_histogram_f32_rule_disagreements_exist():
+    """The per-element pin above is not vacuous: on a non-power-of-two grid
+    with points planted at the edges, the fp32 rule and the exact-rational rule
+    do disagree somewhere (else the pin would pass a kernel that used either)."""
+    from fractions import Fraction
+    lo, hi, nbins = 0.1, 0.7, 100
+    n_dis = 0
+    for k in range(nbins + 1):
+        e = np.float32(lo + (hi - lo) * k / nbins)
+        for v in (np.nextafter(e, np.float32(-1), dtype=np.float32), e, np.nextafter(e, np.float32(2), dtype=np.float32)):
+            c = oracle.histogram(np.array([v], np.float32), lo, hi, nbins)
+            got = int(np.flatnonzero(c)[0]) if c.any() else None
+            p = (Fraction(float(v)) - Fraction(lo)) * nbins / (Fraction(hi) - Fraction(lo))
+            want = int(p // 1) if 0 <= p < nbins else None
+            n_dis += got != want
+    assert n_dis > 0
