@@ -156,9 +156,19 @@ typedef struct {
                          registers; REDUCE_STAGE_SMEM: cp.async 16-byte copies into a
                          shared-memory tile (block*unroll*32 <= 128 KiB), then shared
                          loads -- more bytes in flight per SM.  Same numerics. */
+  int flags;          /* REDUCE_FLAG_* bits, 0 = none (reduce / reduce_ex only) */
 } reduce_opts_t;
 
 typedef enum { REDUCE_STAGE_AUTO = 0, REDUCE_STAGE_REG = 1, REDUCE_STAGE_SMEM = 2 } reduce_stage_t;
+
+/* reduce_opts_t.flags:
+ *   REDUCE_FLAG_INPUT_READY : the caller guarantees that no kernel that may
+ *     still be running when this call is launched on `stream` writes `in`
+ *     (e.g. the input was written before the previous kernel on the stream
+ *     was launched, or was produced by another stream synchronised earlier).
+ *     The reduction may then load its first tile before its programmatic
+ *     dependency resolves ("early loads", see Stream ordering below). */
+typedef enum { REDUCE_FLAG_INPUT_READY = 1 } reduce_flag_t;
 
 /* What a call will launch (filled by reduce_query_plan). */
 typedef struct {
@@ -173,13 +183,17 @@ typedef struct {
 
 /* Stream ordering.  Kernels are launched with programmatic dependent launch:
  * a reduction's first blocks may start while the previous kernel on the stream
- * drains.  A reduce() / reduce_ex() whose input does not overlap the previous
- * library call's output on the stream loads its first tile before its
- * dependency resolves (it waits before touching anything else); this is safe
- * for any producer that is not itself a programmatic-launch primary writing
- * the input -- callers whose own kernels trigger early completion
- * (griddepcontrol.launch_dependents) before writing a reduction's input set
- * REDUCE_NO_EARLY=1 (REDUCE_NO_PDL=1 disables programmatic launch altogether). */
+ * drains, but by default they execute griddepcontrol.wait before touching any
+ * memory, so the previous kernel's writes -- whoever launched it, and even if
+ * it triggered its dependents early (griddepcontrol.launch_dependents, as
+ * cuBLAS / CUTLASS kernels do) -- are complete and visible first.
+ * Early loads are opt-in: with REDUCE_FLAG_INPUT_READY in reduce_opts_t.flags
+ * (and an input that does not overlap the previous library call's output on
+ * the stream) each block that is resident before the dependency resolves
+ * loads its first tile of `in` before waiting.  That is only correct when the
+ * caller's guarantee above holds; a producer kernel still writing `in` would
+ * be read stale.  REDUCE_NO_EARLY=1 ignores the flag; REDUCE_NO_PDL=1 disables
+ * programmatic launch altogether. */
 
 /* Reduce in[0..n) with `op` into *out (device).  Uses the process-default mode. */
 int reduce(int dtype, int op, const void* in, size_t n, void* out, reduce_stream_t stream);
@@ -279,6 +293,7 @@ int reduce_comm_unique_id_bytes(void);           /* 128 (sizeof ncclUniqueId) */
 int reduce_comm_get_unique_id(void* id_out);     /* rank 0; broadcast the bytes */
 int reduce_comm_init(void** comm_out, const void* id, int nranks, int rank); /* after cudaSetDevice */
 int reduce_comm_destroy(void* comm);
+int reduce_comm_count(void* comm, int* nranks);   /* ncclCommCount: ranks in the communicator */
 
 /* ---- sharded mode with the cross-GPU combine fused into the kernel --------
  * (the one-shot combine "fused as the epilogue of the last

@@ -22,6 +22,7 @@ MODE_FAST, MODE_DETERMINISTIC = 0, 1
 BC_SHFL, BC_SMEM_ATOMIC_WARP, BC_SMEM_ATOMIC_ALL, BC_SMEM_TREE = 0, 1, 2, 3
 GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER = 0, 1, 2, 3, 4
 STAGE_REG, STAGE_SMEM = 1, 2
+FLAG_INPUT_READY = 1
 OK = 0
 
 OPS = {"sum": SUM, "min": MIN, "max": MAX, "sum_accurate": SUM_ACCURATE}
@@ -33,7 +34,7 @@ ABI_SYMBOLS = (
     "reduce", "reduce_ex", "reduce_query_plan", "reduce_prepare", "reduce_set_mode",
     "reduce_get_mode", "reduce_host", "reduce_multi", "reduce_multi_ex",
     "reduce_comm_unique_id_bytes", "reduce_comm_get_unique_id", "reduce_comm_init",
-    "reduce_comm_destroy", "reduce_status_string", "reduce_last_error", "reduce_version",
+    "reduce_comm_destroy", "reduce_comm_count", "reduce_status_string", "reduce_last_error", "reduce_version",
     "reduce_shutdown", "reduce_segmented", "reduce_batched", "reduce_histogram",
     "reduce_team_create", "reduce_team_ipc_handle_bytes", "reduce_team_buffer", "reduce_team_connect",
     "reduce_team_connect_local", "reduce_team_destroy", "reduce_multi_team",
@@ -50,7 +51,7 @@ class ReduceError(RuntimeError):
 class reduce_opts_t(ctypes.Structure):
     _fields_ = [("mode", ctypes.c_int), ("grid_combine", ctypes.c_int), ("block_combine", ctypes.c_int),
                 ("block", ctypes.c_int), ("unroll", ctypes.c_int), ("grid", ctypes.c_int),
-                ("seg_group", ctypes.c_int), ("stage", ctypes.c_int)]
+                ("seg_group", ctypes.c_int), ("stage", ctypes.c_int), ("flags", ctypes.c_int)]
 
 
 class reduce_plan_t(ctypes.Structure):
@@ -86,6 +87,7 @@ def _load() -> ctypes.CDLL:
         "reduce_comm_get_unique_id": (i, [vp]),
         "reduce_comm_init": (i, [ctypes.POINTER(vp), vp, i, i]),
         "reduce_comm_destroy": (i, [vp]),
+        "reduce_comm_count": (i, [vp, ctypes.POINTER(i)]),
         "reduce_status_string": (ctypes.c_char_p, [i]),
         "reduce_last_error": (ctypes.c_char_p, []),
         "reduce_version": (i, []),
@@ -124,7 +126,11 @@ def _check(status: int, where: str) -> None:
         raise ReduceError(status, where)
 
 
-def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=0, grid=0, stage=0, seg_group=0):
+def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=0, grid=0, stage=0, seg_group=0,
+              input_ready=False, flags=0):
+    """reduce_opts_t from keywords.  input_ready=True sets REDUCE_FLAG_INPUT_READY
+    (the caller guarantees no kernel still running writes the input: early loads
+    allowed, include/reduce.h "Stream ordering")."""
     if isinstance(mode, str):
         mode = {"fast": MODE_FAST, "deterministic": MODE_DETERMINISTIC}[mode]
     if isinstance(stage, str):
@@ -132,7 +138,8 @@ def make_opts(mode=None, grid_combine=None, block_combine=None, block=0, unroll=
     return reduce_opts_t(-1 if mode is None else int(mode),
                          -1 if grid_combine is None else int(grid_combine),
                          -1 if block_combine is None else int(block_combine),
-                         int(block), int(unroll), int(grid), int(seg_group), int(stage))
+                         int(block), int(unroll), int(grid), int(seg_group), int(stage),
+                         int(flags) | (FLAG_INPUT_READY if input_ready else 0))
 
 
 def _op(op) -> int:
@@ -311,6 +318,12 @@ class Comm:
                "reduce_comm_init")
         self.handle = handle.value
         self.rank, self.world = rank, world
+
+    def nranks(self) -> int:
+        """ncclCommCount of the communicator (ranks NCCL itself sees)."""
+        k = ctypes.c_int(0)
+        _check(lib.reduce_comm_count(ctypes.c_void_p(self.handle), ctypes.byref(k)), "reduce_comm_count")
+        return k.value
 
     def destroy(self) -> None:
         if self.handle:

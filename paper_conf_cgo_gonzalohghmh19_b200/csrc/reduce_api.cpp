@@ -63,8 +63,9 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
 
   reduce_opts_t o;
   o.mode = -1; o.grid_combine = -1; o.block_combine = -1; o.block = 0; o.unroll = 0; o.grid = 0; o.seg_group = 0;
-  o.stage = 0;
+  o.stage = 0; o.flags = 0;
   if (opts) o = *opts;
+  if (o.flags & ~REDUCE_FLAG_INPUT_READY) return fail(REDUCE_ERR_INVALID_ARG, "unknown bits in flags");
   int mode = o.mode < 0 ? g_mode.load() : o.mode;
   if (mode != REDUCE_MODE_FAST && mode != REDUCE_MODE_DETERMINISTIC)
     return fail(REDUCE_ERR_INVALID_ARG, "mode must be -1, REDUCE_MODE_FAST or REDUCE_MODE_DETERMINISTIC");
@@ -217,6 +218,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   }
 
   P->dtype = dtype; P->op = op; P->mode = mode; P->n = n; P->elem = s;
+  P->input_ready = (o.flags & REDUCE_FLAG_INPUT_READY) != 0;
   LaunchDesc& d = P->d;
   std::memset(&d, 0, sizeof(d));
   d.dtype = dtype; d.op = op; d.in = in;
@@ -373,10 +375,20 @@ int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream, bool all
   d.ticket = (unsigned*)(ws->tickets + combo * (size_t)kSlotBytes);
   d.partials = ws->partials;
   d.early = 0;
-  if (allow_early && early_enabled() && pdl_enabled() && P->n > 0) {
-    const uintptr_t lo = (uintptr_t)d.in, hi = lo + (uintptr_t)P->n * (uintptr_t)P->elem;
-    d.early = (hi <= ws->last_out_lo.load(std::memory_order_relaxed) ||
-               lo >= ws->last_out_hi.load(std::memory_order_relaxed)) ? 1 : 0;
+  // Before the programmatic dependency resolves a kernel may touch its input:
+  //  1 = register loads of the first tile, only on the caller's explicit
+  //      guarantee (REDUCE_FLAG_INPUT_READY) and when the input is not the
+  //      previous library output -- a producer the library cannot see (a
+  //      foreign kernel that triggered its dependents early) could still be
+  //      writing it otherwise;
+  //  2 = a bulk L2 prefetch of the first tile (always correct: a hint)
+  if (early_enabled() && pdl_enabled() && P->n > 0) {
+    d.early = prefetch_enabled() ? 2 : 0;
+    if (allow_early && P->input_ready) {
+      const uintptr_t lo = (uintptr_t)d.in, hi = lo + (uintptr_t)P->n * (uintptr_t)P->elem;
+      if (hi <= ws->last_out_lo.load(std::memory_order_relaxed) || lo >= ws->last_out_hi.load(std::memory_order_relaxed))
+        d.early = 1;
+    }
   }
   cudaError_t e = launch_reduce(d, stream);
   if (allow_early) {  // this call wrote `out` only (one value of at most 16 bytes)

@@ -51,6 +51,23 @@ bool early_enabled() {
   return on;
 }
 
+bool prefetch_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("REDUCE_NO_PREFETCH");
+    return !(e && e[0] == '1');
+  }();
+  return on;
+}
+
+long long prefetch_budget_bytes() {
+  static const long long b = [] {
+    const char* e = std::getenv("REDUCE_PREFETCH_MB");
+    long long mb = e ? std::atoll(e) : 32;
+    return (mb < 0 ? 0 : mb) << 20;
+  }();
+  return b;
+}
+
 bool rows_tiled_enabled() {
   static const bool on = [] {
     const char* e = std::getenv("REDUCE_NO_ROWS_TILED");

@@ -55,6 +55,15 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
   const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(s), "l"(gmem) : "memory");
 }
+// Bulk L2 prefetch (sm_90+, UBLKPF): a hint that moves `bytes` (multiple of
+// 16, 16-byte-aligned source) from HBM into L2 without touching registers or
+// shared memory.  A prefetch has no effect on memory consistency, so it may be
+// issued before griddepcontrol.wait: a store of the previous kernel reaching
+// L2 afterwards updates the prefetched line, and the loads after the wait read
+// the current data from L2.
+__device__ __forceinline__ void prefetch_l2_bulk(const void* gmem, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(gmem), "r"(bytes) : "memory");
+}
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 // one 32-byte vector from shared memory as 8 words
 __device__ __forceinline__ void lds_v8(const void* smem, uint32_t (&r)[8]) {
@@ -171,6 +180,9 @@ template <int OP> struct TrI32 {
   using Grid = Acc;
   static constexpr int VE = 8, NA = 2, kLaneWords = 1;
   static constexpr bool kVecTree = true;
+  // The ATOMIC grid combine of int32 sums carries value and ticket in ONE
+  // 64-bit atomic add (grid_combine): no fence, no second round trip.
+  static constexpr bool kPackedTicket = OP == OP_SUM;
   __device__ static Acc lift(uint32_t w) { return Acc(w); }
   __device__ static Acc ident() {
     return OP == OP_SUM ? Acc(0) : (OP == OP_MIN ? Acc(0x7FFFFFFF) : Acc(0x80000000));
@@ -438,6 +450,9 @@ template <class T> using Part = typename PartOf<T>::type;
 //     which keeps the small-unroll kernels at 32 registers (full occupancy).
 //   fp64 min/max: the same tree of selects, NaN in the sticky flag.
 //   otherwise (accurate sums): lane k folds into accumulator k.
+template <class T, class = void> struct HasPackedTicket : std::false_type {};
+template <class T> struct HasPackedTicket<T, std::enable_if_t<T::kPackedTicket>> : std::true_type {};
+
 template <class T, class = void> struct HasSelNaN : std::false_type {};
 template <class T> struct HasSelNaN<T, std::enable_if_t<T::kSelNaN>> : std::true_type {};
 

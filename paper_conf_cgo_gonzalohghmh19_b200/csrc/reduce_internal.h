@@ -79,8 +79,9 @@ struct LaunchDesc {
   unsigned* ticket;              // this (dtype, op)'s ticket (GC_ATOMIC / GC_LAST_BLOCK)
   void* partials;                // Grid[grid] (GC_TWO_PASS / GC_LAST_BLOCK)
   TeamArgs team;                 // team.k > 0: exchange the raw result with the team first
-  int early;                     // 1: load the first tile before griddepcontrol.wait (the input is
-                                 //    not an output of the previous call on the stream)
+  int early;                     // before griddepcontrol.wait: 1 = load the first tile into registers
+                                 // (REDUCE_FLAG_INPUT_READY, input not the previous library output),
+                                 // 2 = bulk L2 prefetch of the first tile (a hint, always correct)
 };
 
 // Long-segment queue of a segmented call (lives in the stream's workspace):
@@ -199,9 +200,15 @@ cudaError_t launch_init_workspace(void* slots_base, void* tickets_base, cudaStre
 // Programmatic dependent launch of the library's kernels (default on; the
 // environment variable REDUCE_NO_PDL=1 turns it off, for A/B measurements).
 bool pdl_enabled();
-// Loads of the input before the programmatic dependency resolves (default on;
-// REDUCE_NO_EARLY=1 turns it off, for A/B measurements).
+// Touching the input before the programmatic dependency resolves at all
+// (default on; REDUCE_NO_EARLY=1 turns both forms off, for A/B measurements).
 bool early_enabled();
+// The bulk L2 prefetch of a block's first tile before the wait (default on;
+// REDUCE_NO_PREFETCH=1 turns it off).
+bool prefetch_enabled();
+// Bytes a grid prefetches into L2 before its dependency resolves (at least
+// every early-resident block's first tile); REDUCE_PREFETCH_MB, default 32.
+long long prefetch_budget_bytes();
 // REDUCE_NO_ROWS_TILED=1: reduce_batched's auto choice skips k_rows_tiled
 bool rows_tiled_enabled();
 

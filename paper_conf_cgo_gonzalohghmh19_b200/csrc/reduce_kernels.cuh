@@ -45,6 +45,8 @@ struct KParams {
   void* partials;
   TeamArgs team;
   int early;
+  int pf_stride;   // early != 0: blocks below pf_stride prefetch tiles blockIdx + k*pf_stride,
+  int pf_tiles;    //   k < pf_tiles, into L2 before the wait (set by launch_kernel)
 };
 
 // ---- one-shot cross-GPU combine through peer memory ------
@@ -164,6 +166,27 @@ __device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& 
     if (threadIdx.x == 0) ((Grid*)p.partials)[blockIdx.x] = g;
     return;
   }
+  if constexpr (HasPackedTicket<T>::value) {
+    // int32 sums: Listing 2's `atomicAdd(Return, ...)` and the ticket
+    // in one 64-bit atomic add on slot 0: bits 48-63 count the blocks, bits
+    // 0-31 hold the sum mod 2^32 and bits 32-47 absorb its carries (at most one
+    // per block, so < 2^16 for grids below 2^16).  The block that sees count
+    // G-1 owns the complete sum in old + add -- no release fence before a
+    // separate ticket, no second round trip to collect slots (B200 probe,
+    // tools/probes/probe_mid.cu: -0.9 to -1.5 us per call at 1-64 MB).  It
+    // resets the word for the next call.
+    if (p.gc == GC_ATOMIC && gridDim.x < 65536u) {
+      if (threadIdx.x == 0) {
+        const unsigned long long add = (1ull << 48) | (unsigned long long)(uint32_t)g;
+        const unsigned long long old = atomicAdd((unsigned long long*)p.slots, add);
+        if ((unsigned)(old >> 48) == gridDim.x - 1) {
+          atomicExch((unsigned long long*)p.slots, 0ull);
+          store_out<T>((Grid)(uint32_t)(old + add), p);
+        }
+      }
+      return;
+    }
+  }
   if (p.gc == GC_ATOMIC) {
     // Listing 2's `atomicAdd(Return, ...)` per block, spread over
     // nslots accumulators on separate L2 lines; the ticket's last holder
@@ -221,24 +244,41 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
   // A team call whose members share this GPU never triggers: the next grid's
   // parked CTAs could fill the SMs a co-resident member needs to reach the
   // exchange this grid's last block is waiting in.
-  // Early loads (p.early, set by the host only when the input does not overlap
-  // the previous call's output on this stream): a block that is resident before
-  // the dependency resolves issues its first tile's loads first -- they fill the
-  // previous grid's drain -- and folds them after the wait (same order, same
-  // numerics).  The input is the only memory touched before the wait.
-  // (U <= 4 only: with 8 loads per thread the prefetched registers would be
-  // allocated beside the loop's -- 94 -> 120 registers, one block less per SM;
-  // the U = 8 kernels compile exactly as without early loads)
+  // Before the dependency resolves only the input is touched, in one of two ways:
+  //  * p.early == 2 (default): thread 0 issues one bulk L2 prefetch of the
+  //    block's first tile -- a hint with no effect on memory consistency, so it
+  //    is correct whoever writes the input and whenever; the bytes stream into
+  //    L2 during the previous grid's drain and the loads after the wait hit L2.
+  //  * p.early == 1 (REDUCE_FLAG_INPUT_READY, the caller guarantees no running
+  //    kernel writes the input, and it is not the previous library output): a
+  //    block that is resident before the dependency resolves loads its first
+  //    tile into registers, and folds it after the wait (same order, same
+  //    numerics).  (U <= 4 only: with 8 loads per thread the prefetched
+  //    registers would be allocated beside the loop's -- 94 -> 120 registers,
+  //    one block less per SM; the U = 8 kernels prefetch into L2 instead.)
   constexpr bool kEarly = STAGE == STAGE_REG && U <= 4;
   uint32_t pre[kEarly ? U : 1][8];
   bool have_pre = false;
   if constexpr (kEarly) {
     const long long tv = (long long)blockDim.x * U;
-    if (p.early && (long long)blockIdx.x < p.tiles && (unsigned long long)((blockIdx.x + 1) * tv) <= p.body_vecs) {
+    if (p.early == 1 && (long long)blockIdx.x < p.tiles && (unsigned long long)((blockIdx.x + 1) * tv) <= p.body_vecs) {
       const char* ptr = p.body + ((unsigned long long)(blockIdx.x * tv) + threadIdx.x) * kVecBytes;
 #pragma unroll
       for (int u = 0; u < U; ++u) ld_v8(ptr + (size_t)u * blockDim.x * kVecBytes, pre[u]);
       have_pre = true;
+    }
+  }
+  if (p.early != 0 && threadIdx.x == 0 && (int)blockIdx.x < p.pf_stride) {
+    // bulk L2 prefetches of the tiles this block (and, when the grid has more
+    // blocks than fit at once, the blocks of later waves) will read: the HBM
+    // reads run while the previous grid drains; the loads after the wait hit L2
+    const unsigned long long tv = (unsigned long long)blockDim.x * U;
+    long long t = blockIdx.x + (have_pre ? p.pf_stride : 0);
+#pragma unroll 1
+    for (int k = have_pre ? 1 : 0; k < p.pf_tiles && t < p.tiles; ++k, t += p.pf_stride) {
+      const unsigned long long v0 = (unsigned long long)t * tv;
+      const unsigned long long nv = v0 + tv <= p.body_vecs ? tv : p.body_vecs - v0;
+      prefetch_l2_bulk(p.body + v0 * kVecBytes, (uint32_t)(nv * kVecBytes));
     }
   }
   pdl_wait();
@@ -340,7 +380,12 @@ __global__ void __launch_bounds__(1024) k_combine(const void* vals, long long co
 template <int DT, int OP>
 __global__ void k_init_slots(void* slots, unsigned* ticket) {
   using T = Tr<DT, OP>;
-  if (threadIdx.x < kMaxSlots) *(typename T::Grid*)((char*)slots + threadIdx.x * kSlotBytes) = T::gident();
+  if (threadIdx.x < kMaxSlots) {
+    unsigned long long* w = (unsigned long long*)((char*)slots + threadIdx.x * kSlotBytes);
+    w[0] = 0ull;  // the packed int32-sum word is 8 bytes wide; Grid values are <= 16
+    w[1] = 0ull;
+    *(typename T::Grid*)w = T::gident();
+  }
   if (threadIdx.x == 0) *ticket = 0u;
 }
 
@@ -361,6 +406,7 @@ inline KParams make_params(const LaunchDesc& d) {
   p.partials = d.partials;
   p.team = d.team;
   p.early = d.early;
+  p.pf_stride = p.pf_tiles = 0;
   // TWO_PASS: the exchange happens in the second kernel, not per block
   if (d.gc == GC_TWO_PASS) p.team.k = 0;
   return p;
@@ -406,6 +452,24 @@ inline int blocks_per_sm(const void* kern, int block, size_t smem) {
   return nb;
 }
 
+// SM count of the current device, cached per device.
+inline int num_sms_cached() {
+  static std::mutex mu;
+  static std::map<int, int> cache;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = cache.find(dev);
+  if (it != cache.end()) return it->second;
+  int sms = 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms < 1) {
+    cudaGetLastError();
+    sms = 148;
+  }
+  cache[dev] = sms;
+  return sms;
+}
+
 // Launch one k_reduce instantiation; GC_CLUSTER launches exactly one cluster
 // of d.grid CTAs (sizes above the portable 8 need the non-portable opt-in);
 // STAGE_SMEM needs block*U*32 bytes of dynamic shared memory (opt-in above 48 KB).
@@ -415,6 +479,22 @@ inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& 
   if (smem > 0 || (d.gc == GC_CLUSTER && d.grid > 8)) {
     const cudaError_t e = opt_in_smem((const void*)kern, kMaxSmemTileBytes, true);
     if (e != cudaSuccess) return e;
+  }
+  KParams q = p;
+  q.pf_stride = 0;
+  q.pf_tiles = 0;
+  if (p.early != 0 && d.tiles > 0) {
+    // blocks resident at once (one wave): they issue the prefetches, striding
+    // over the tiles, up to prefetch_budget_bytes() (L2 is 126 MB; the previous
+    // grid's and this grid's streams share it)
+    const long long wave = (long long)blocks_per_sm((const void*)kern, d.block, smem) * num_sms_cached();
+    const long long stride = d.grid < wave ? d.grid : wave;
+    const long long tile_bytes = (long long)d.block * d.unroll * kVecBytes;
+    long long cap = prefetch_budget_bytes() / tile_bytes;
+    if (cap < stride) cap = stride;  // at least every early block's first tile
+    const long long want = d.tiles < cap ? d.tiles : cap;
+    q.pf_stride = (int)stride;
+    q.pf_tiles = (int)((want + stride - 1) / stride);
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(d.grid, 1, 1);
@@ -437,7 +517,7 @@ inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& 
   }
   cfg.attrs = attr;
   cfg.numAttrs = na;
-  return cudaLaunchKernelEx(&cfg, kern, p);
+  return cudaLaunchKernelEx(&cfg, kern, q);
 }
 
 // k_combine with the same programmatic-dependent-launch attribute.

@@ -119,6 +119,14 @@ int reduce_comm_destroy(void* comm) {
   return REDUCE_OK;
 }
 
+int reduce_comm_count(void* comm, int* nranks) {
+  if (!comm || !nranks) return fail(REDUCE_ERR_INVALID_ARG, "comm / nranks is NULL");
+  if (!load_nccl()) return REDUCE_ERR_UNSUPPORTED;
+  ncclResult_t r = g_nccl.CommCount((ncclComm_t)comm, nranks);
+  if (r != ncclSuccess) return nccl_fail(r, "ncclCommCount");
+  return REDUCE_OK;
+}
+
 int reduce_multi_ex(int dtype, int op, const void* in_local, size_t n_local, void* out, reduce_stream_t stream,
                     void* comm, const reduce_opts_t* opts) {
   if (out == nullptr) return fail(REDUCE_ERR_INVALID_ARG, "out is NULL");

@@ -46,6 +46,7 @@ struct Plan {
   int dtype, op, mode;
   size_t n;
   int elem;  // bytes per element
+  bool input_ready;  // REDUCE_FLAG_INPUT_READY: early loads allowed (reduce / reduce_ex)
   LaunchDesc d;
   reduce_plan_t pub;
 };

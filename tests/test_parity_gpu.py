@@ -393,3 +393,25 @@ def test_chained_calls_read_the_previous_output():
     want = np.array([(k + 1) * n for k in range(64)], np.float32)
     assert (res.cpu().numpy() == want).all(), res.cpu().numpy()[:8]
     assert (res2.cpu().numpy() == want).all(), res2.cpu().numpy()[:8]
+
+
+@pytest.mark.parametrize("tiles", [1, 2, 65534, 65535, 65536, 65537])
+def test_int32_sum_packed_atomic_around_its_grid_limit(tiles):
+    """int32 sums under the ATOMIC combine carry value and block count in one
+    64-bit atomic word (count in bits 48-63, so grids below 2^16); 65536 blocks
+    and up take the slots + ticket path.  Full-range values make every block
+    carry into bits 32-47.  Back-to-back calls check the word is reset."""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    n = tiles * 256 - 3  # 32 threads x 1 vector of 8 int32 per tile; a ragged tail
+    x = synth.make("int32", n, "int_full", 77 + tiles)
+    t = to_device(x)
+    opts = dict(grid_combine=1, block=32, unroll=1, grid=-1)
+    p = rb.query_plan("int32", "sum", n, in_ptr=t.data_ptr(), **opts)
+    assert p["grid"] == tiles and p["grid_combine"] == 1
+    outs = torch.empty(3, dtype=torch.int32, device="cuda")
+    for i in range(3):
+        rb.reduce(t, "sum", out=outs[i:i + 1], **opts)
+    got = outs.cpu().numpy()
+    want = oracle.reduce(x, "sum").bits
+    assert all(int(g.view(np.uint32)) == want for g in got), (got, want)

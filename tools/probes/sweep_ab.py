@@ -1,7 +1,9 @@
 """Per-call device time of the auto-dispatched reduce over a size sweep (graph
 of R calls over disjoint cold regions, tools/tune.py's harness): for A/B of
 library builds swapped in by tools/probes/lib_ab.sh.
-Usage: python tools/probes/sweep_ab.py TAG"""
+Usage: python tools/probes/sweep_ab.py TAG [--input-ready]
+(--input-ready: every call passes REDUCE_FLAG_INPUT_READY -- the inputs are
+written once, long before -- so early register loads are allowed)"""
 import json
 import os
 import sys
@@ -14,6 +16,7 @@ import paper_conf_cgo_gonzalohghmh19_b200 as rb  # noqa: E402
 from cudatiming import time_calls, disjoint_regions  # noqa: E402
 
 tag = sys.argv[1] if len(sys.argv) > 1 else ""
+kw = dict(input_ready=True) if "--input-ready" in sys.argv else {}
 dev = torch.device("cuda", 0)
 stream = torch.cuda.Stream(dev)
 for dtype, ops in (("float32", ("sum",)), ("int32", ("sum", "max")), ("float64", ("max",))):
@@ -32,7 +35,7 @@ for dtype, ops in (("float32", ("sum",)), ("int32", ("sum", "max")), ("float64",
 
             def launch(t):
                 i = k[0] = (k[0] + 1) % 4096
-                rb.reduce(t, op, out=out[i:i + 1], stream=stream)
+                rb.reduce(t, op, out=out[i:i + 1], stream=stream, **kw)
             row[f"2^{lb}"] = round(time_calls(launch, warm, timed, stream, repeats=3) * 1e6, 3)
         print(json.dumps(row), flush=True)
     del pool
