@@ -9,10 +9,17 @@ one batch of synthetic input already resident in HBM:
   N > 1 : reduce_multi_team(fp32, sum): every rank reduces its own 2^28-element
           shard and the per-rank scalars meet in the kernel's epilogue over
           peer memory (--collective nccl: one NCCL all-reduce instead; the
-          team path falls back to it if the peer mapping cannot be made)
-          (configs[4]: at N = 8 this is the 8 GiB array).  Weak scaling.
+          team path falls back to it if the peer mapping cannot be made).
+          `value` is weak scaling (2^28 per GPU; at N = 8 this is the 8 GiB
+          array of configs[4]); the same line carries `strong_scaling`: the
+          fixed 2^31-element (8 GiB) array of configs[4], n_local = 2^31 / N
+          per rank (`--scaling strong` makes it the `value`).
           The sharded result is checked against the sum of the per-rank local
-          results once after warm-up (`cross_rank_check`).
+          results once after warm-up, for every combine available
+          (`cross_rank_check`).
+`python bench.py --gpus N` without a torchrun environment re-executes itself
+under torch.distributed.run with N ranks (one per GPU); under torchrun,
+WORLD_SIZE must equal --gpus.
 The 1 GiB per-GPU input is larger than the 126 MB L2, so consecutive steps
 read from HBM without an explicit flush.
 
@@ -61,6 +68,11 @@ def parse():
     ap.add_argument("--collective", default="team", choices=["team", "nccl"],
                     help="cross-GPU combine: 'team' = fused into the reduction kernel over peer memory "
                          "(reduce_multi_team), 'nccl' = one ncclAllReduce of the per-rank scalar")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="which series is the line's `value`: weak = --elements per GPU, strong = "
+                         "--strong-total elements split over the N GPUs (both are always reported)")
+    ap.add_argument("--strong-total", type=int, default=1 << 31,
+                    help="total elements of the strong-scaling array (default 2^31 = 8 GiB fp32, configs[4])")
     ap.add_argument("--share-gpu", action="store_true",
                     help="TEST MODE: every rank on cuda:0, gloo control plane, team combine over CUDA IPC "
                          "(validates the multi-rank path on a one-GPU box; timings are not scaling numbers)")
@@ -206,6 +218,56 @@ def host_times(xh):
     return outs
 
 
+# The paper's own numbers (speedup ratios only -- it reports no absolute
+# throughput), quoted with their hardware: context, never a B200 target.
+PAPER_CONTEXT = {
+    "source": "Garcia De Gonzalo et al., CGO 2019 (PAPER.md); fp32, 64..2^28 elements, host<->device copies untimed "
+              "(P:L463-L469, P:L641); baselines CUB 1.8.0 on the same GPU, OpenMP 4.0 on 2x8-core POWER8+",
+    "hardware": {"Kepler": "K40c, nvcc 8.0.44", "Maxwell": "GTX980, nvcc 9.1.85", "Pascal": "P100, nvcc 9.2.88"},
+    "claims": [
+        {"where": "P:L601", "gpus": "K40c / GTX980 / P100", "sizes": "< 1M elements",
+         "tangram_vs_cub": "2x-6x faster on average"},
+        {"where": "P:L601", "gpus": "K40c / GTX980 / P100", "sizes": "> 1M elements",
+         "tangram_vs_cub": "17%-38% slower (CUB's vector loads)"},
+        {"where": "P:L685", "gpus": "Kepler K40c", "sizes": "1K-4M", "version": "(m)",
+         "tangram_vs_cub": "4.6x", "tangram_vs_openmp": "3.6x"},
+        {"where": "P:L687", "gpus": "Kepler K40c", "sizes": "> 4M", "tangram_vs_cub": "~38% slower"},
+        {"where": "P:L733", "gpus": "Maxwell GTX980", "sizes": "65K-4M", "version": "(p)",
+         "tangram_vs_cub": "4.6x", "tangram_vs_openmp": "3.4x"},
+        {"where": "P:L735", "gpus": "Maxwell GTX980", "sizes": "> 4M", "tangram_vs_cub": "~7% slower"},
+        {"where": "P:L777", "gpus": "Pascal P100", "sizes": "<= 1K", "tangram_vs_openmp": "on par"},
+        {"where": "P:L777", "gpus": "Pascal P100", "sizes": "4K-65K", "tangram_vs_cub": "~8.5x",
+         "tangram_vs_openmp": "~4.8x"},
+        {"where": "P:L779", "gpus": "Pascal P100", "sizes": "65K-4M", "tangram_vs_cub": "4x"},
+        {"where": "P:L781", "gpus": "Pascal P100", "sizes": "> 4M", "tangram_vs_cub": "27% slower"},
+    ],
+}
+
+
+def paper_context(sweep):
+    """PAPER_CONTEXT plus this run's like-for-like ratios on the B200: the
+    library vs CUB 12.9's DeviceReduce on the same device, per size class of
+    the paper (geometric mean over the fp32 U[0,1) sweep points in the class)."""
+    ctx = dict(PAPER_CONTEXT)
+    if not sweep:
+        return ctx
+    classes = (("< 1M elements", 0, 1 << 20), ("1K-4M", 1 << 10, 1 << 22), ("65K-4M", 1 << 16, 1 << 22),
+               ("4K-65K", 1 << 12, 1 << 16), ("> 1M elements", (1 << 20) + 1, 1 << 40), ("> 4M", (1 << 22) + 1, 1 << 40))
+    b200 = {}
+    for name, lo, hi in classes:
+        r = [e["speedup_vs_cub"] for e in sweep if e.get("dist") == "U[0,1)" and lo <= e["n"] <= hi
+             and e.get("speedup_vs_cub")]
+        if r:
+            g = 1.0
+            for v in r:
+                g *= v
+            b200[name] = {"ours_vs_cub_geomean": round(g ** (1 / len(r)), 3), "points": len(r)}
+    ctx["b200_this_run"] = b200
+    ctx["note"] = ("the paper's gains over CUB 1.8 came from CUB's small-array overheads on Kepler-Pascal; "
+                   "CUB in CUDA 12.9 on B200 has none of them, so like-for-like ratios here are smaller")
+    return ctx
+
+
 # --------------------------------------------------------------- reference arm
 def run_reference(args, rank, world):
     """This tier's reference arm: the CPU oracle, as it stands, on the host cores."""
@@ -260,14 +322,39 @@ def workload_config(args, world, plan, sharded=False):
     return cfg
 
 
+def spawn_or_check_world(args):
+    """One process per GPU.  `--gpus N` (N > 1) outside torchrun re-executes this
+    script under torch.distributed.run with N ranks and exits with its status;
+    under torchrun, WORLD_SIZE must equal --gpus (else exit 2: a bench line
+    must never claim N GPUs while timing a different number of ranks)."""
+    ws = os.environ.get("WORLD_SIZE")
+    if ws is None:
+        if args.gpus > 1 and args.impl == "ours":
+            import socket
+            import subprocess
+            with socket.socket() as sk:
+                sk.bind(("127.0.0.1", 0))
+                port = sk.getsockname()[1]
+            cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+                   "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+            print(f"bench: spawning {args.gpus} ranks: {' '.join(cmd)}", file=sys.stderr, flush=True)
+            sys.exit(subprocess.run(cmd).returncode)
+        return
+    if int(ws) != args.gpus:
+        print(f"bench: WORLD_SIZE={ws} but --gpus {args.gpus}: refusing to time a different rank count",
+              file=sys.stderr, flush=True)
+        sys.exit(2)
+
+
 # --------------------------------------------------------------- our arm
 def main():
     args = parse()
+    spawn_or_check_world(args)
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
-        return run_reference(args, rank, world)
+        return run_reference(args, rank, world if "WORLD_SIZE" in os.environ else args.gpus)
 
     import numpy as np
     import torch
@@ -305,28 +392,48 @@ def main():
     stream = torch.cuda.Stream(dev)
     comm = None
     collective_note = None
+    combines = {}  # name -> Team / Comm of every cross-GPU combine this run could build
+    comm_info = None
     if sharded:
-        if args.collective == "team":
-            try:
-                comm = rb.Team()
-            except rb.ReduceError as e:  # e.g. no peer mapping between the GPUs: use the NCCL combine
-                if args.share_gpu:
-                    raise
-                collective_note = f"team combine unavailable ({e}); fell back to the NCCL all-reduce"
+        try:
+            combines["team"] = rb.Team()
+        except rb.ReduceError as e:  # e.g. no peer mapping between the GPUs
+            if args.share_gpu:
+                raise
+            combines["team"] = None
+            collective_note = f"team combine unavailable ({e})"
+        if args.share_gpu:
+            combines["nccl"] = None  # NCCL refuses two ranks on one GPU
+        else:
+            combines["nccl"] = rb.Comm()
+        if combines.get(args.collective) is None:
+            if args.collective == "team" and combines.get("nccl") is not None:
+                collective_note = (collective_note or "team combine unavailable") + "; fell back to the NCCL all-reduce"
                 print(f"bench: {collective_note}", file=sys.stderr)
                 args.collective = "nccl"
-        if comm is None:
-            comm = rb.Comm()
+            else:
+                raise SystemExit(f"bench: the {args.collective} combine is unavailable")
+        comm = combines[args.collective]
+        comm_info = {"world_size": world,
+                     "team_members": None if combines.get("team") is None else combines["team"].world,
+                     "nccl_comm_nranks": None if combines.get("nccl") is None else combines["nccl"].nranks(),
+                     "process_group_backend": dist.get_backend()}
+        if comm_info["nccl_comm_nranks"] not in (None, world) or comm_info["team_members"] not in (None, world):
+            raise SystemExit(f"bench: communicator size disagrees with WORLD_SIZE: {comm_info}")
     plan = rb.query_plan("float32", "sum", n, in_ptr=x.data_ptr(), mode=args.mode)
     rb.prepare(stream, n)
+
+    def sharded_call(name, xt, o):
+        if name == "team":
+            rb.reduce_multi_team(xt, "sum", combines["team"], out=o, stream=stream, mode=args.mode)
+        else:
+            rb.reduce_multi(xt, "sum", combines["nccl"], out=o, stream=stream, mode=args.mode)
 
     def step():
         if comm is None:
             rb.reduce(x, "sum", out=out, stream=stream, mode=args.mode)
-        elif args.collective == "team":
-            rb.reduce_multi_team(x, "sum", comm, out=out, stream=stream, mode=args.mode)
         else:
-            rb.reduce_multi(x, "sum", comm, out=out, stream=stream, mode=args.mode)
+            sharded_call(args.collective, x, out)
 
     def sync_all():
         torch.cuda.synchronize(dev)
@@ -334,26 +441,42 @@ def main():
             dist.barrier()
         torch.cuda.synchronize(dev)
 
+    def cross_rank_check(name, xt):
+        """The sharded result of combine `name` against the per-rank local
+        results summed over the torch process group (an independent path): the
+        relative gap must be at the fp32 rounding level of the final conversions."""
+        o = torch.empty(1, dtype=torch.float32, device=dev)
+        loc = torch.empty(1, dtype=torch.float32, device=dev)
+        with torch.cuda.stream(stream):
+            sharded_call(name, xt, o)
+            rb.reduce(xt, "sum", out=loc, stream=stream, mode=args.mode)
+        torch.cuda.synchronize(dev)
+        got = float(o.item())
+        t = torch.tensor([float(loc.item())], dtype=torch.float64, device="cpu" if args.share_gpu else dev)
+        dist.all_reduce(t)
+        want = float(t.item())
+        rel = abs(got - want) / max(abs(want), 1e-30)
+        # every rank must agree on the bits as well (the combine is one value for all)
+        g = torch.tensor([got], dtype=torch.float64, device="cpu" if args.share_gpu else dev)
+        gmax, gmin = g.clone(), g.clone()
+        dist.all_reduce(gmax, op=dist.ReduceOp.MAX)
+        dist.all_reduce(gmin, op=dist.ReduceOp.MIN)
+        res = {"sharded": got, "sum_of_local": want, "rel_gap": rel, "ranks_agree": float(gmax) == float(gmin),
+               "ok": rel <= 4 * world * 2.0 ** -24 and float(gmax) == float(gmin)}
+        if not res["ok"]:
+            print(f"bench: {name} sharded result check failed: {res}", file=sys.stderr)
+        return res
+
     with torch.cuda.stream(stream):
         for _ in range(max(3, args.warmup)):
             step()
     sync_all()
     cross_check = None
     if comm is not None:
-        # the sharded result against the per-rank local results summed over the
-        # torch process group (an independent path): relative gap must be at
-        # the fp32 rounding level of one final conversion
-        got = float(out.item())
-        loc = torch.empty(1, dtype=torch.float32, device=dev)
-        rb.reduce(x, "sum", out=loc, stream=stream, mode=args.mode)
-        torch.cuda.synchronize(dev)
-        t = torch.tensor([float(loc.item())], dtype=torch.float64, device="cpu" if args.share_gpu else dev)
-        dist.all_reduce(t)
-        want = float(t.item())
-        rel = abs(got - want) / max(abs(want), 1e-30)
-        cross_check = {"sharded": got, "sum_of_local": want, "rel_gap": rel, "ok": rel <= 4 * world * 2.0 ** -24}
-        if not cross_check["ok"]:
-            print(f"bench: sharded result disagrees with the sum of local results: {cross_check}", file=sys.stderr)
+        cross_check = {}
+        for name in ("team", "nccl"):
+            cross_check[name] = (cross_rank_check(name, x) if combines.get(name) is not None
+                                 else "unavailable" + (" (ranks share one GPU)" if args.share_gpu and name == "nccl" else ""))
         sync_all()
     # Single GPU: the K steps are captured once into a CUDA graph and replayed
     # (no host launch gaps between steps; the same kernels on the same
@@ -385,6 +508,65 @@ def main():
     if world > 1:
         ms = allmax(ms)
     value = world * n * 4 / (ms * 1e-3) / 1e9
+
+    # ---- strong scaling: the fixed --strong-total array
+    # (2^31 fp32 = 8 GiB, configs[4]) split into contiguous shards, rank r owns
+    # [floor(r T / N), floor((r+1) T / N)) drawn on its own GPU; K steps of the
+    # same path (graph-replayed at N = 1, stream-launched sharded calls at N > 1).
+    strong = None
+    strong_clocks = None
+    if args.strong_total > 0:
+        lo_s, hi_s = rb.shard_range(args.strong_total, world, rank)
+        n_s = hi_s - lo_s
+        gen = torch.Generator(device=dev).manual_seed(2019 + 1000 * 4 + 31 + rank)
+        xs = torch.rand(n_s, dtype=torch.float32, device=dev, generator=gen)
+        os_ = torch.empty(1, dtype=torch.float32, device=dev)
+        rb.prepare(stream, n_s)
+
+        def sstep():
+            if comm is None:
+                rb.reduce(xs, "sum", out=os_, stream=stream, mode=args.mode)
+            else:
+                sharded_call(args.collective, xs, os_)
+        with torch.cuda.stream(stream):
+            for _ in range(max(3, args.warmup)):
+                sstep()
+        sync_all()
+        s_check = cross_rank_check(args.collective, xs) if comm is not None else None
+        sync_all()
+        sgraph = None
+        if comm is None:
+            sgraph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(sgraph, stream=stream):
+                for _ in range(args.steps):
+                    sstep()
+            with torch.cuda.stream(stream):
+                sgraph.replay()
+            sync_all()
+        strong_clocks = ClockSampler(local)
+        with strong_clocks:
+            with torch.cuda.stream(stream):
+                e0.record(stream)
+                if sgraph is not None:
+                    sgraph.replay()
+                else:
+                    for _ in range(args.steps):
+                        sstep()
+                e1.record(stream)
+            e1.synchronize()
+        sync_all()
+        s_ms = allmax(e0.elapsed_time(e1) / args.steps) if world > 1 else e0.elapsed_time(e1) / args.steps
+        strong = {"total_elements": args.strong_total, "total_bytes": args.strong_total * 4,
+                  "n_local_rank0": rb.shard_range(args.strong_total, world, 0)[1], "ms_per_step": round(s_ms, 5),
+                  "value": round(args.strong_total * 4 / (s_ms * 1e-3) / 1e9, 2), "unit": "GB/s",
+                  "elements_per_s": round(args.strong_total / (s_ms * 1e-3), 1),
+                  "launch": "cuda-graph replay" if sgraph is not None else f"stream (sharded, {args.collective})",
+                  "data": "torch.rand U[0,1) fp32 on each rank's own GPU, seed 2019+4031+rank",
+                  "clocks": strong_clocks.summary()}
+        if s_check is not None:
+            strong["cross_rank_check"] = s_check
+        del sgraph, xs
+        torch.cuda.empty_cache()
     # sharded: the same K steps without the cross-rank combine (local reduce
     # only), so the combine's cost per step is visible
     decomposition = None
@@ -524,36 +706,55 @@ def main():
         except Exception:
             cubref = None
         outs = torch.empty(4096, dtype=torch.float32, device=dev)
+        # C2: every power of two 2^10..2^28 elements, U[0,1) and
+        # U[-1,1).  Columns: cold (each call of the graph reads a region nobody
+        # touched recently: HBM) with the default stream ordering; cold with
+        # REDUCE_FLAG_INPUT_READY (inputs written long before: early register
+        # loads allowed); L2-warm (the same region every call; above the 126 MB
+        # L2 it is HBM again); CUB's DeviceReduce on the cold regions.
+        x_pm1 = (x * 2 - 1).contiguous()
         sweep = []
-        for k in range(6, 29, 2):
-            m = 1 << k
-            R = max(3, min(100, (256 << 20) // (4 * m))) if 4 * m < (256 << 20) else 20
-            warm, timed = disjoint_regions(x, R, m)
-            p = rb.query_plan("float32", "sum", m, in_ptr=timed[0].data_ptr(), mode=args.mode)
-            ctr = [0]
+        for dist_name, pool in (("U[0,1)", x), ("U[-1,1)", x_pm1)):
+            for k in range(10, 29):
+                m = 1 << k
+                R = max(3, min(100, (256 << 20) // (4 * m))) if 4 * m < (256 << 20) else 20
+                warm, timed = disjoint_regions(pool, R, m)
+                p = rb.query_plan("float32", "sum", m, in_ptr=timed[0].data_ptr(), mode=args.mode)
+                ctr = [0]
 
-            def launch(t):
-                ctr[0] = (ctr[0] + 1) % 4096
-                rb.reduce(t, "sum", out=outs[ctr[0]:ctr[0] + 1], stream=stream, mode=args.mode)
-            sec = time_calls(launch, warm, timed, stream, repeats=3)
-            gbs = m * 4 / sec / 1e9
-            cub_sec = None
-            if cubref is not None:  # the paper's comparison system, on the same device (context)
-                def launch_cub(t):
+                def launch(t, **kw):
                     ctr[0] = (ctr[0] + 1) % 4096
-                    cubref.reduce(1, 0, t.data_ptr(), t.numel(), outs[ctr[0]:ctr[0] + 1].data_ptr(), stream.cuda_stream)
-                cubref.reduce(1, 0, timed[0].data_ptr(), m, outs.data_ptr(), stream.cuda_stream)  # size temp storage
-                torch.cuda.synchronize(dev)
-                cub_sec = time_calls(launch_cub, warm, timed, stream, repeats=3)
-            # the CPU beside it at the same n (the paper's CPU
-            # crossover): the oracle (1 thread) and the OpenMP pragma loop
-            cpu_o, cpu_p = host_times(x_host[:m])
-            sweep.append({"n": m, "us": round(sec * 1e6, 3), "GBps": round(gbs, 1),
-                          "cpu_oracle_us": cpu_o, "cpu_omp_us": cpu_p,
-                          "cub_us": None if cub_sec is None else round(cub_sec * 1e6, 3),
-                          "speedup_vs_cub": None if cub_sec is None else round(cub_sec / sec, 3),
-                          "elements_per_s": round(m / sec, 1), "frac_of_peak": round(gbs / peak, 4),
-                          "variant": f"gc{p['grid_combine']} g{p['grid']}x{p['block']} u{p['unroll']}"})
+                    rb.reduce(t, "sum", out=outs[ctr[0]:ctr[0] + 1], stream=stream, mode=args.mode, **kw)
+                sec = time_calls(launch, warm, timed, stream, repeats=3)
+                sec_ready = time_calls(lambda t: launch(t, input_ready=True), warm, timed, stream, repeats=3)
+                sec_warm = time_calls(launch, [timed[0]] * R, [timed[0]] * R, stream, repeats=3)
+                gbs = m * 4 / sec / 1e9
+                cub_sec = None
+                if cubref is not None:  # the paper's comparison system, on the same device (context)
+                    def launch_cub(t):
+                        ctr[0] = (ctr[0] + 1) % 4096
+                        cubref.reduce(1, 0, t.data_ptr(), t.numel(), outs[ctr[0]:ctr[0] + 1].data_ptr(),
+                                      stream.cuda_stream)
+                    cubref.reduce(1, 0, timed[0].data_ptr(), m, outs.data_ptr(), stream.cuda_stream)  # temp storage
+                    torch.cuda.synchronize(dev)
+                    cub_sec = time_calls(launch_cub, warm, timed, stream, repeats=3)
+                row = {"dist": dist_name, "n": m, "log2_n": k, "paper_size_point": k % 2 == 0,
+                       "us": round(sec * 1e6, 3), "GBps": round(gbs, 1),
+                       "elements_per_s": round(m / sec, 1), "frac_of_peak": round(gbs / peak, 4),
+                       "frac_of_nominal_8TBps": round(gbs / 8000.0, 4),
+                       "input_ready_us": round(sec_ready * 1e6, 3),
+                       "input_ready_GBps": round(m * 4 / sec_ready / 1e9, 1),
+                       "l2_warm_us": round(sec_warm * 1e6, 3),
+                       "l2_warm_GBps": round(m * 4 / sec_warm / 1e9, 1),
+                       "cub_us": None if cub_sec is None else round(cub_sec * 1e6, 3),
+                       "speedup_vs_cub": None if cub_sec is None else round(cub_sec / sec, 3),
+                       "variant": f"gc{p['grid_combine']} g{p['grid']}x{p['block']} u{p['unroll']}"}
+                if dist_name == "U[0,1)":
+                    # the CPU beside it at the same n (the paper's CPU
+                    # crossover): the oracle (1 thread) and the OpenMP pragma loop
+                    row["cpu_oracle_us"], row["cpu_omp_us"] = host_times(x_host[:m])
+                sweep.append(row)
+        del x_pm1
         latency = []
         for dt in ("int32", "float32"):
             tdt = getattr(torch, dt)
@@ -607,22 +808,34 @@ def main():
     if not args.no_sweep and world == 1:
         import oracle
         m = 1 << 20
-        xi_h = synth.make("int32", m, "int_full", synth.seed_for(0, m))
-        xi = torch.from_numpy(xi_h).to(dev)
         oi = torch.empty(4096, dtype=torch.int32, device=dev)
-        warm_i, timed_i = disjoint_regions(x.view(torch.int32), 50, m)
-        ctr = [0]
+        cfg1 = []
+        # C1: full-range values (every block's sum wraps) and the
+        # small range randint(-1000, 1001), each in both modes; device time per
+        # call from a graph over cold regions holding that very distribution,
+        # the bit-exact check of one call on the seeded array, and the oracle.
+        for dist_i in ("int_full", "int_small"):
+            xi_h = synth.make("int32", m, dist_i, synth.seed_for(0, m))
+            xi = torch.from_numpy(xi_h).to(dev)
+            pool_i = xi.repeat(64)  # 64 cold-able copies (256 MB > L2)
+            warm_i, timed_i = disjoint_regions(pool_i, 32, m)
+            t0 = time.perf_counter()
+            want = int(oracle.reduce(xi_h, "sum").value)
+            cpu_us = (time.perf_counter() - t0) * 1e6
+            for mode_i in ("fast", "deterministic"):
+                ctr = [0]
 
-        def launch_i(t):
-            ctr[0] = (ctr[0] + 1) % 4096
-            rb.reduce(t, "sum", out=oi[ctr[0]:ctr[0] + 1], stream=stream)
-        gpu_us = time_calls(launch_i, warm_i, timed_i, stream, repeats=3) * 1e6
-        got = int(rb.reduce(xi, "sum", stream=stream).cpu().item())
-        t0 = time.perf_counter()
-        want = int(oracle.reduce(xi_h, "sum").value)
-        cpu_us = (time.perf_counter() - t0) * 1e6
-        cfg1 = {"n": m, "gpu_us": round(gpu_us, 3), "GBps": round(m * 4 / gpu_us / 1e3, 1), "cpu_oracle_us": round(cpu_us, 1),
-                "bit_exact": got == want}
+                def launch_i(t, mode_i=mode_i):
+                    ctr[0] = (ctr[0] + 1) % 4096
+                    rb.reduce(t, "sum", out=oi[ctr[0]:ctr[0] + 1], stream=stream, mode=mode_i)
+                gpu_us = time_calls(launch_i, warm_i, timed_i, stream, repeats=3) * 1e6
+                got = int(rb.reduce(xi, "sum", stream=stream, mode=mode_i).cpu().item())
+                pp = rb.query_plan("int32", "sum", m, in_ptr=xi.data_ptr(), mode=mode_i)
+                cfg1.append({"n": m, "dist": dist_i, "mode": mode_i, "gpu_us": round(gpu_us, 3),
+                             "GBps": round(m * 4 / gpu_us / 1e3, 1), "cpu_oracle_us": round(cpu_us, 1),
+                             "bit_exact": got == want,
+                             "variant": f"gc{pp['grid_combine']} g{pp['grid']}x{pp['block']} u{pp['unroll']}"})
+            del pool_i
         # ---- BASELINE configs[2]: int32 / fp64 sum, min, max at 64 M elements,
         # atomic (fast) vs deterministic-tree grid combine
         cfg3 = []
@@ -657,22 +870,9 @@ def main():
                 cfg3.append(row)
 
     # ---- BASELINE configs[4] at k = 1: one 8 GiB (2^31 fp32) array on one GPU
-    # (64-bit indexing); timing only (its parity is tests/test_parity_gpu.py's
-    # full-size test), so the array is drawn on the device.
-    big = None
-    if not args.no_sweep and world == 1:
-        xb = torch.rand(1 << 31, dtype=torch.float32, device=dev, generator=torch.Generator(dev).manual_seed(2019))
-        ob = torch.empty(1, dtype=torch.float32, device=dev)
-
-        def launch_big(t):
-            rb.reduce(t, "sum", out=ob, stream=stream, mode=args.mode)
-        sec = time_calls(launch_big, [xb] * 2, [xb] * 10, stream, repeats=2)
-        pb = rb.query_plan("float32", "sum", xb.numel(), in_ptr=xb.data_ptr(), mode=args.mode)
-        big = {"n": 1 << 31, "bytes": (1 << 31) * 4, "us": round(sec * 1e6, 1),
-               "GBps": round((1 << 31) * 4 / sec / 1e9, 1), "frac_of_peak": round((1 << 31) * 4 / sec / 1e9 / peak, 4),
-               "variant": f"gc{pb['grid_combine']} g{pb['grid']}x{pb['block']} u{pb['unroll']} st{pb['stage']}"}
-        del xb
-        torch.cuda.empty_cache()
+    # (64-bit indexing) is the strong-scaling series' N = 1 point (above); its
+    # parity is tests/test_parity_gpu.py's full-size test.
+    big = strong if world == 1 else None
 
     # ---- histogram of the resident 1 GiB, 256 and 65536 bins
     hist = None
@@ -693,7 +893,7 @@ def main():
     batched = None
     if not args.no_sweep and world == 1:
         batched = []
-        per_call = {e["n"]: e["us"] for e in sweep}
+        per_call = {e["n"]: e["us"] for e in sweep if e["dist"] == "U[0,1)"}
         for cols in (64, 1024, 16384):
             rows = (256 << 20) // (4 * cols)
             xv = x[: rows * cols].view(rows, cols)
@@ -757,22 +957,35 @@ def main():
 
     if rank == 0:
         launches_per_step = plan["launches"] + (1 if (comm is not None and args.collective == "nccl") else 0)
+        weak = {"n_per_gpu": n, "total_bytes": world * n * 4, "ms_per_step": round(ms, 5), "value": round(value, 2),
+                "unit": "GB/s", "elements_per_s": round(world * n / (ms * 1e-3), 1)}
+        use_strong = args.scaling == "strong" and strong is not None
+        v_ms = strong["ms_per_step"] if use_strong else ms
+        v_val = strong["value"] if use_strong else value
         line = {
-            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
-            "data": "synthetic", "config": workload_config(args, world, plan, comm is not None),
-            "elements_per_s": round(world * n / (ms * 1e-3), 1),
+            "metric": METRIC, "value": round(v_val, 2), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(v_ms, 5),
+            "higher_is_better": True, "scaling": "strong" if use_strong else "weak", "vs_baseline": None,
+            "dtype": "f32", "data": "synthetic", "config": workload_config(args, world, plan, comm is not None),
+            "elements_per_s": strong["elements_per_s"] if use_strong else round(world * n / (ms * 1e-3), 1),
             "launch": "cuda-graph replay of the K steps" if comm is None else
                       f"stream (K sharded calls; cross-GPU combine: {args.collective})",
             "stream_launched": None if stream_ms is None else {
                 "ms_per_step": round(stream_ms, 5), "value": round(world * n * 4 / (stream_ms * 1e-3) / 1e9, 2)},
-            "frac_of_hbm_peak": round(value / world / peak, 4),
-            "roofline": roofline, "e2e": e2e, "clocks": clocks.summary(),
+            "frac_of_hbm_peak": round(v_val / world / peak, 4),
+            "weak_scaling": weak, "strong_scaling": strong,
+            "roofline": roofline, "e2e": e2e,
+            "clocks": (strong_clocks if use_strong else clocks).summary(),
             "gpu_launches": args.steps * launches_per_step,
             "gpu": gpu_identity(local),
             "env": software_env(dev),
         }
+        if use_strong:
+            line["config"]["workload"] = (f"fp32 sum of one {args.strong_total}-element array split over {world} GPU(s) "
+                                          f"-- BASELINE configs[4] strong scaling")
+            line["config"]["total_bytes"] = args.strong_total * 4
+        if comm_info is not None:
+            line["comm"] = comm_info
         if decomposition is not None:
             line["sharded_decomposition"] = decomposition
         if cross_check is not None:
@@ -784,6 +997,7 @@ def main():
         if cpu is not None:
             line["cpu_baseline"] = cpu
             line["cpu_openmp"] = cpu_omp
+        line["paper_context"] = paper_context(sweep)
         if sweep is not None:
             line["sweep"] = sweep
             line["small_array_latency"] = latency
@@ -801,7 +1015,9 @@ def main():
         torch.cuda.synchronize(dev)
         if world > 1:
             dist.barrier()  # no member may unmap its team buffer while others still use it
-        comm.destroy()
+        for c in combines.values():
+            if c is not None:
+                c.destroy()
         dist.destroy_process_group()
 
 

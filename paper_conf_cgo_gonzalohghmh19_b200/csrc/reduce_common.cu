@@ -62,7 +62,7 @@ bool prefetch_enabled() {
 long long prefetch_budget_bytes() {
   static const long long b = [] {
     const char* e = std::getenv("REDUCE_PREFETCH_MB");
-    long long mb = e ? std::atoll(e) : 32;
+    long long mb = e ? std::atoll(e) : 0;  // B200 A/B: deeper prefetch gains nothing (profiles/r02_prefetch_depth_ab.jsonl)
     return (mb < 0 ? 0 : mb) << 20;
   }();
   return b;

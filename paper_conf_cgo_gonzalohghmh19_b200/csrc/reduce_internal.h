@@ -207,7 +207,7 @@ bool early_enabled();
 // REDUCE_NO_PREFETCH=1 turns it off).
 bool prefetch_enabled();
 // Bytes a grid prefetches into L2 before its dependency resolves (at least
-// every early-resident block's first tile); REDUCE_PREFETCH_MB, default 32.
+// every early-resident block's first tile); REDUCE_PREFETCH_MB, default 0 (first tiles only).
 long long prefetch_budget_bytes();
 // REDUCE_NO_ROWS_TILED=1: reduce_batched's auto choice skips k_rows_tiled
 bool rows_tiled_enabled();
