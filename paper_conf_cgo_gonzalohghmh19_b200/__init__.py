@@ -168,6 +168,47 @@ def _stream_handle(stream, device=None) -> int:
     return stream.cuda_stream
 
 
+def _check_cuda_in(x, what: str = "input") -> None:
+    if not x.is_cuda:
+        raise ValueError(f"{what} must be a CUDA tensor")
+    if not x.is_contiguous():
+        raise ValueError(f"{what} must be contiguous")
+
+
+def _check_out(out, x, count: int, dtype=None) -> None:
+    """A caller-supplied output must hold `count` elements of the result dtype,
+    contiguous, on x's device (the C side writes count * sizeof(T) bytes)."""
+    want = x.dtype if dtype is None else dtype
+    if out.dtype != want:
+        raise ValueError(f"out has dtype {out.dtype}, expected {want}")
+    if not out.is_cuda or out.device != x.device:
+        raise ValueError(f"out must be a CUDA tensor on {x.device}, got {out.device}")
+    if not out.is_contiguous():
+        raise ValueError("out must be contiguous")
+    if out.numel() < count:
+        raise ValueError(f"out holds {out.numel()} elements, needs {count}")
+
+
+class _on_device:
+    """Make x's device current for the C call (the library resolves its
+    workspace and launches on the current device; the stream comes from x)."""
+
+    def __init__(self, dev):
+        self.dev = dev
+
+    def __enter__(self):
+        import torch
+        self.prev = torch.cuda.current_device()
+        if self.dev.index is not None and self.dev.index != self.prev:
+            torch.cuda.set_device(self.dev)
+        return self
+
+    def __exit__(self, *a):
+        import torch
+        if torch.cuda.current_device() != self.prev:
+            torch.cuda.set_device(self.prev)
+
+
 def reduce_ptr(dtype: int, op, in_ptr: int, n: int, out_ptr: int, stream: int = 0, opts=None) -> None:
     """Raw-pointer form of reduce_ex (device pointers, stream handle)."""
     st = lib.reduce_ex(dtype, OPS[op] if op.__class__ is str else op, in_ptr or None, n, out_ptr or None,
@@ -186,9 +227,12 @@ def reduce(x, op="sum", out=None, stream=None, **opt_kw):
     if out is None:
         import torch
         out = torch.empty(1, dtype=x.dtype, device=x.device)
+    else:
+        _check_out(out, x, 1)
     opts = make_opts(**opt_kw) if opt_kw else None
     s = stream.cuda_stream if stream is not None and not isinstance(stream, int) else _stream_handle(stream, x.device)
-    reduce_ptr(dt, op, x.data_ptr(), x.numel(), out.data_ptr(), s, opts)
+    with _on_device(x.device):
+        reduce_ptr(dt, op, x.data_ptr(), x.numel(), out.data_ptr(), s, opts)
     return out
 
 
@@ -197,15 +241,21 @@ def reduce_segmented(x, offsets, op="sum", out=None, stream=None, **opt_kw):
     int64 tensor offsets of num_segments + 1 entries (one launch, deterministic)."""
     import torch
     dt = _torch_dtype_code(x)
+    _check_cuda_in(x)
     nseg = offsets.numel() - 1
     if offsets.dtype != torch.int64 or not offsets.is_cuda or not offsets.is_contiguous():
         raise ValueError("offsets must be a contiguous CUDA int64 tensor")
+    if offsets.device != x.device:
+        raise ValueError("offsets must be on the input's device")
     if out is None:
         out = torch.empty(max(nseg, 0), dtype=x.dtype, device=x.device)
+    else:
+        _check_out(out, x, max(nseg, 0))
     opts = make_opts(**opt_kw) if opt_kw else None
-    st = lib.reduce_segmented(dt, _op(op), x.data_ptr() or None, offsets.data_ptr() or None, max(nseg, 0),
-                              out.data_ptr() or None, _stream_handle(stream, x.device),
-                              ctypes.byref(opts) if opts is not None else None)
+    with _on_device(x.device):
+        st = lib.reduce_segmented(dt, _op(op), x.data_ptr() or None, offsets.data_ptr() or None, max(nseg, 0),
+                                  out.data_ptr() or None, _stream_handle(stream, x.device),
+                                  ctypes.byref(opts) if opts is not None else None)
     _check(st, "reduce_segmented")
     return out
 
@@ -216,12 +266,16 @@ def reduce_batched(x, op="sum", out=None, stream=None, **opt_kw):
     dt = _torch_dtype_code(x)
     if x.dim() != 2 or not x.is_contiguous():
         raise ValueError("reduce_batched takes a contiguous 2-D tensor")
+    _check_cuda_in(x)
     rows, cols = x.shape
     if out is None:
         out = torch.empty(rows, dtype=x.dtype, device=x.device)
+    else:
+        _check_out(out, x, rows)
     opts = make_opts(**opt_kw) if opt_kw else None
-    st = lib.reduce_batched(dt, _op(op), x.data_ptr() or None, cols, rows, out.data_ptr() or None,
-                            _stream_handle(stream, x.device), ctypes.byref(opts) if opts is not None else None)
+    with _on_device(x.device):
+        st = lib.reduce_batched(dt, _op(op), x.data_ptr() or None, cols, rows, out.data_ptr() or None,
+                                _stream_handle(stream, x.device), ctypes.byref(opts) if opts is not None else None)
     _check(st, "reduce_batched")
     return out
 
@@ -230,10 +284,14 @@ def histogram(x, lo: float, hi: float, nbins: int, counts=None, stream=None):
     """counts[b] = #{lo <= x < hi, b = floor((x - lo) * nbins / (hi - lo))} (CUDA int32/fp32 tensor)."""
     import torch
     dt = _torch_dtype_code(x)
+    _check_cuda_in(x)
     if counts is None:
         counts = torch.empty(nbins, dtype=torch.int32, device=x.device)  # bit pattern of uint32 counts
-    st = lib.reduce_histogram(dt, x.data_ptr() or None, x.numel(), float(lo), float(hi), int(nbins),
-                              counts.data_ptr(), _stream_handle(stream, x.device))
+    else:
+        _check_out(counts, x, int(nbins), dtype=torch.int32)
+    with _on_device(x.device):
+        st = lib.reduce_histogram(dt, x.data_ptr() or None, x.numel(), float(lo), float(hi), int(nbins),
+                                  counts.data_ptr(), _stream_handle(stream, x.device))
     _check(st, "reduce_histogram")
     return counts
 
@@ -335,8 +393,11 @@ def reduce_multi(x, op, comm: Comm, out=None, stream=None, **opt_kw):
     """Every rank passes its local CUDA shard; every rank gets the global result."""
     import torch
     dt = _torch_dtype_code(x)
+    _check_cuda_in(x)
     if out is None:
         out = torch.empty(1, dtype=x.dtype, device=x.device)
+    else:
+        _check_out(out, x, 1)
     opts = make_opts(**opt_kw) if opt_kw else None
     st = lib.reduce_multi_ex(dt, _op(op), ctypes.c_void_p(x.data_ptr() or None), x.numel(),
                              ctypes.c_void_p(out.data_ptr()), ctypes.c_void_p(_stream_handle(stream, x.device)),
@@ -403,8 +464,11 @@ def reduce_multi_team(x, op, team: Team, out=None, stream=None, **opt_kw):
     """Every team member passes its local CUDA shard; every member gets the global result."""
     import torch
     dt = _torch_dtype_code(x)
+    _check_cuda_in(x)
     if out is None:
         out = torch.empty(1, dtype=x.dtype, device=x.device)
+    else:
+        _check_out(out, x, 1)
     opts = make_opts(**opt_kw) if opt_kw else None
     st = lib.reduce_multi_team(dt, _op(op), x.data_ptr() or None, x.numel(), out.data_ptr(),
                                _stream_handle(stream, x.device), team.handle,

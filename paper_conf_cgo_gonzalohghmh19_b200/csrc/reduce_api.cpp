@@ -23,7 +23,47 @@ struct DispatchEntry {
 static thread_local std::string g_err;
 static std::atomic<int> g_mode{REDUCE_MODE_FAST};
 static std::mutex g_ws_mu;
-static std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
+// Workspaces are keyed by (device, CUDA stream id): cudaStreamPerThread has the
+// same handle value in every host thread but names a different stream in each,
+// and a destroyed stream's handle value may be reused by a new stream -- the
+// id (cudaStreamGetId) is unique for both.
+static std::map<std::pair<int, unsigned long long>, Workspace*> g_ws;
+
+// cudaStreamGetId is not usable while the stream is being captured (it fails
+// and would invalidate the capture), so the id seen by the last non-capturing
+// call on a handle is cached: per host thread for the special handles (legacy
+// default, per-thread default), process-wide for created streams.
+static std::mutex g_sid_mu;
+static std::map<cudaStream_t, unsigned long long> g_sid;
+static thread_local std::map<cudaStream_t, unsigned long long> t_sid;
+
+static unsigned long long stream_id(cudaStream_t s) {
+  const bool special = (uintptr_t)s <= 2u;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  const bool capturing = cudaStreamIsCapturing(s, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone;
+  if (!capturing) {
+    unsigned long long id = 0;
+    if (cudaStreamGetId(s, &id) == cudaSuccess) {
+      if (special) {
+        t_sid[s] = id;
+      } else {
+        std::lock_guard<std::mutex> lk(g_sid_mu);
+        g_sid[s] = id;
+      }
+      return id;
+    }
+    cudaGetLastError();
+  }
+  if (special) {
+    auto it = t_sid.find(s);
+    if (it != t_sid.end()) return it->second;
+  } else {
+    std::lock_guard<std::mutex> lk(g_sid_mu);
+    auto it = g_sid.find(s);
+    if (it != g_sid.end()) return it->second;
+  }
+  return (unsigned long long)(uintptr_t)s | (1ull << 63);  // never seen outside a capture: no workspace yet
+}
 
 void set_error(const std::string& msg) { g_err = msg; }
 int fail(int status, const std::string& msg) {
@@ -259,14 +299,15 @@ int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+  const auto key = std::make_pair(dev, stream_id(stream));
   std::lock_guard<std::mutex> lk(g_ws_mu);
-  Workspace*& w = g_ws[std::make_pair(dev, stream)];
+  Workspace*& w = g_ws[key];
   const bool need_base = (w == nullptr);
   const bool need_partials = (w == nullptr || w->partials_bytes < partials_bytes);
   if (need_base || need_partials) {
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     if (cudaStreamIsCapturing(stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
-      if (need_base) g_ws.erase(std::make_pair(dev, stream));
+      if (need_base) g_ws.erase(key);
       return fail(REDUCE_ERR_NOT_PREPARED, "workspace missing or too small during stream capture: call reduce_prepare first");
     }
   }
@@ -278,7 +319,7 @@ int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
     e = cudaMalloc(&nw->base, base_bytes);
     if (e != cudaSuccess) {
       delete nw;
-      g_ws.erase(std::make_pair(dev, stream));
+      g_ws.erase(key);
       cudaGetLastError();
       return fail(REDUCE_ERR_NO_MEMORY, "cudaMalloc(workspace) failed");
     }
@@ -289,7 +330,7 @@ int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
     if (e != cudaSuccess) {
       cudaFree(nw->base);
       delete nw;
-      g_ws.erase(std::make_pair(dev, stream));
+      g_ws.erase(key);
       return cuda_fail(e, "workspace init kernel");
     }
     w = nw;
@@ -405,8 +446,9 @@ int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream, bool all
 void note_unknown_output(cudaStream_t stream) {
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) return;
+  const auto key = std::make_pair(dev, stream_id(stream));
   std::lock_guard<std::mutex> lk(g_ws_mu);
-  auto it = g_ws.find(std::make_pair(dev, stream));
+  auto it = g_ws.find(key);
   if (it == g_ws.end() || it->second == nullptr) return;
   it->second->last_out_lo.store(0, std::memory_order_relaxed);
   it->second->last_out_hi.store(~(uintptr_t)0, std::memory_order_relaxed);
@@ -651,12 +693,16 @@ int reduce_query_plan(int dtype, int op, const void* in, size_t n, const reduce_
 }
 
 int reduce_prepare(reduce_stream_t stream, size_t max_n) {
-  // partials for the largest possible partials-based grid at max_n
-  const unsigned long long tiles_min_tile = (max_n + 255) / 256;  // smallest tile is 32 threads x 1 vector
+  // partials for the largest partials-based grid any call of up to max_n
+  // elements can plan: the smallest tile is 32 threads x 1 vector = 128
+  // elements (fp64; 256 for 4-byte types), the widest cross-block value is 16
+  // bytes (fp64 accurate sums: double-double), the grid is capped at
+  // kMaxPartialBlocks
+  const unsigned long long tiles_min_tile = (max_n + 127) / 128;
   long long g = (long long)(tiles_min_tile < (unsigned long long)kMaxPartialBlocks ? tiles_min_tile : kMaxPartialBlocks);
   if (g < 1024) g = 1024;
   Workspace* ws = nullptr;
-  int st = get_workspace((cudaStream_t)stream, (size_t)g * 8, &ws);
+  int st = get_workspace((cudaStream_t)stream, (size_t)g * 16, &ws);
   if (st != REDUCE_OK) return st;
   char* q = nullptr;
   st = get_seg_queue((cudaStream_t)stream, &q);  // so segmented calls can be captured too
@@ -697,12 +743,19 @@ int reduce_version(void) { return 10000 * 0 + 100 * 1 + 0; }
 
 void reduce_shutdown(void) {
   std::lock_guard<std::mutex> lk(g_ws_mu);
+  // the stream a workspace was made for may be gone (or be another thread's
+  // per-thread stream): wait for each device instead
   for (auto& kv : g_ws) {
     if (kv.second) {
-      cudaStreamSynchronize(kv.second->stream);
+      int prev = 0;
+      cudaGetDevice(&prev);
+      cudaSetDevice(kv.second->device);
+      cudaDeviceSynchronize();
+      cudaSetDevice(prev);
       free_workspace(kv.second);
     }
   }
+  cudaGetLastError();
   g_ws.clear();
 }
 

@@ -75,7 +75,9 @@ __device__ __forceinline__ void lds_v8(const void* smem, uint32_t (&r)[8]) {
 // Programmatic dependent launch (sm_90+): wait for the preceding grid of the
 // stream (a no-op when it was not launched programmatically), and let the next
 // programmatic grid be scheduled.
-constexpr unsigned kPdlTriggerWindow = 148u * 8u;  // ~ one full wave of resident blocks
+// The trigger window (blocks of the last ~full wave) is 8 blocks per SM of the
+// device the kernel runs on; the host passes it in the kernel parameters.
+constexpr unsigned kPdlBlocksPerSm = 8u;
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 

@@ -47,6 +47,7 @@ struct KParams {
   int early;
   int pf_stride;   // early != 0: blocks below pf_stride prefetch tiles blockIdx + k*pf_stride,
   int pf_tiles;    //   k < pf_tiles, into L2 before the wait (set by launch_kernel)
+  unsigned trig_window;  // blocks of the last ~wave (kPdlBlocksPerSm x SMs), set by launch_kernel
 };
 
 // ---- one-shot cross-GPU combine through peer memory ------
@@ -283,7 +284,8 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
   }
   pdl_wait();
   const bool may_trigger = !p.team.shared_gpu;
-  const bool early_trigger = may_trigger && gridDim.x > kPdlTriggerWindow && blockIdx.x + kPdlTriggerWindow >= gridDim.x;
+  const unsigned win = p.trig_window;
+  const bool early_trigger = may_trigger && gridDim.x > win && blockIdx.x + win >= gridDim.x;
   if (early_trigger) pdl_trigger();
   if (p.gc == GC_CLUSTER) cluster_arrive_relaxed();  // phase 1: "this CTA has started"
   Part<T> a[T::NA];
@@ -350,7 +352,7 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
       }
     }
   }
-  if (may_trigger && !early_trigger && gridDim.x <= kPdlTriggerWindow) pdl_trigger();
+  if (may_trigger && !early_trigger && gridDim.x <= win) pdl_trigger();
   if (blockIdx.x == gridDim.x - 1) {
     using Elem = typename T::Elem;
     const int t = threadIdx.x;
@@ -407,6 +409,7 @@ inline KParams make_params(const LaunchDesc& d) {
   p.team = d.team;
   p.early = d.early;
   p.pf_stride = p.pf_tiles = 0;
+  p.trig_window = 0;
   // TWO_PASS: the exchange happens in the second kernel, not per block
   if (d.gc == GC_TWO_PASS) p.team.k = 0;
   return p;
@@ -483,6 +486,7 @@ inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& 
   KParams q = p;
   q.pf_stride = 0;
   q.pf_tiles = 0;
+  q.trig_window = kPdlBlocksPerSm * (unsigned)num_sms_cached();
   if (p.early != 0 && d.tiles > 0) {
     // blocks resident at once (one wave): they issue the prefetches, striding
     // over the tiles, up to prefetch_budget_bytes() (L2 is 126 MB; the previous

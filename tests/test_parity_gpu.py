@@ -415,3 +415,36 @@ def test_int32_sum_packed_atomic_around_its_grid_limit(tiles):
     got = outs.cpu().numpy()
     want = oracle.reduce(x, "sum").bits
     assert all(int(g.view(np.uint32)) == want for g in got), (got, want)
+
+
+def test_per_thread_default_streams_get_their_own_workspace():
+    """cudaStreamPerThread has one handle value (0x2) in every host thread but
+    names a different stream in each: concurrent ATOMIC calls from two threads
+    must not share a workspace (tickets / accumulators), so the library keys
+    workspaces by the CUDA stream id."""
+    import threading
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    n = 1 << 20
+    xs = [torch.full((n,), k + 1, dtype=torch.int32, device="cuda") for k in range(2)]
+    outs = [torch.empty(400, dtype=torch.int32, device="cuda") for _ in range(2)]
+    torch.cuda.synchronize()
+    opts = rb.make_opts(grid_combine=1, block=256, unroll=1)
+    errors = []
+
+    def work(k):
+        try:
+            torch.cuda.set_device(0)
+            for i in range(400):
+                rb.reduce_ptr(rb.INT32, "sum", xs[k].data_ptr(), n, outs[k][i:i + 1].data_ptr(), 2, opts)
+        except Exception as e:  # pragma: no cover
+            errors.append(e)
+    ts = [threading.Thread(target=work, args=(k,)) for k in range(2)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    torch.cuda.synchronize()
+    assert not errors, errors
+    for k in range(2):
+        assert (outs[k].cpu().numpy() == (k + 1) * n).all(), k

@@ -258,10 +258,11 @@ def test_batched_tiled_rows(dtype, row_kb, rows):
     cols = int(row_kb * 1024) // s
     x = synth.make(dtype, rows * cols, "int_full" if dtype == "int32" else "uniform_pm1", int(31 * row_kb) + rows)
     if dtype != "int32" and rows > 3:
-        x[cols + 5] = np.nan          # row 1: NaN
-        x[2 * cols + 7] = -np.inf     # row 2: -inf
+        # indexed per row (rows may be as short as 4 elements: fp64 32 B rows)
+        x[cols + min(5, cols - 1)] = np.nan          # row 1: NaN
+        x[2 * cols + min(7, cols - 1)] = -np.inf     # row 2: -inf
         x[3 * cols:4 * cols] = 0.0
-        x[3 * cols + 2] = -0.0        # row 3: all zeros with one -0.0
+        x[3 * cols + min(2, cols - 1)] = -0.0        # row 3: all zeros with one -0.0
     xt = torch.from_numpy(x).cuda().view(rows, cols)
     bounds = [(r * cols, (r + 1) * cols) for r in range(rows)]
     ops = OPS + (["sum_accurate"] if dtype != "int32" else [])
