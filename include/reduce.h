@@ -324,6 +324,42 @@ int reduce_team_destroy(void* team);
 int reduce_multi_team(int dtype, int op, const void* in_local, size_t n_local, void* out, reduce_stream_t stream,
                       void* team, const reduce_opts_t* opts);
 
+/* ---- sharded mode with an NVLink SHARP (NVLS) combine -----------------------
+ * (SURVEY 8(f) N2 as named there: NCCL symmetric memory + multimem).
+ *   reduce_nvls_create(&v, comm, mode): a COLLECTIVE over the NCCL
+ *     communicator `comm` (every rank calls it, after cudaSetDevice): each
+ *     rank ncclMemAlloc's a 2 MB buffer and registers it as a symmetric window
+ *     (ncclCommWindowRegister, NCCL_WIN_COLL_SYMMETRIC); ncclDevCommCreate with
+ *     lsaMultimem binds the windows to an NVLS multicast object.  mode 1: the
+ *     per-rank values are reduced IN THE NVSWITCH by one multimem.ld_reduce
+ *     after a barrier of one multimem.red per rank; mode 2: each rank puts its
+ *     value with the call's epoch into every rank's window with one multicast
+ *     store (multimem.st) and combines the k values locally in rank order
+ *     (deterministic).  Returns REDUCE_ERR_UNSUPPORTED -- with nothing left
+ *     allocated -- when the ranks do not share one NVLink domain with
+ *     multicast (a single GPU, no NVSwitch, NCCL without NVLS / symmetric
+ *     memory); `comm` stays usable for reduce_multi.  Every rank must get the
+ *     same status (the calls inside are collectives).
+ *   reduce_multi_nvls: as reduce_multi / reduce_multi_team (every rank calls
+ *     it with its own shard, in the same order; every rank's *out gets the
+ *     global result), the exchange fused into the kernel that completes the
+ *     rank's local reduction -- no NCCL launch per call, graph-capturable (the
+ *     call counters live in device memory).  REDUCE_MODE_DETERMINISTIC uses
+ *     mode 2's rank-order combine whatever `mode` was.
+ *   reduce_nvls_destroy: after every rank's last call completed (collective:
+ *     window deregistration). */
+int reduce_nvls_create(void** nvls_out, void* comm, int mode);
+/* A one-member multicast team on the current GPU, built with the CUDA driver's
+ * multicast API instead of NCCL (no second GPU needed): the same kernels and
+ * protocol at k = 1 -- multimem.st / multimem.red / multimem.ld_reduce through
+ * a real multicast object -- for tests and diagnostics.  Use it with
+ * reduce_multi_nvls; REDUCE_ERR_UNSUPPORTED where the device has no
+ * multicast. */
+int reduce_nvls_create_local(void** nvls_out, int mode);
+int reduce_nvls_destroy(void* nvls);
+int reduce_multi_nvls(int dtype, int op, const void* in_local, size_t n_local, void* out, reduce_stream_t stream,
+                      void* nvls, const reduce_opts_t* opts);
+
 /* ---- diagnostics ---------------------------------------------------------- */
 const char* reduce_status_string(int status);
 const char* reduce_last_error(void);   /* thread-local detail of the last failure */

@@ -38,6 +38,7 @@ ABI_SYMBOLS = (
     "reduce_shutdown", "reduce_segmented", "reduce_batched", "reduce_histogram",
     "reduce_team_create", "reduce_team_ipc_handle_bytes", "reduce_team_buffer", "reduce_team_connect",
     "reduce_team_connect_local", "reduce_team_destroy", "reduce_multi_team",
+    "reduce_nvls_create", "reduce_nvls_create_local", "reduce_nvls_destroy", "reduce_multi_nvls",
 )
 
 
@@ -102,6 +103,10 @@ def _load() -> ctypes.CDLL:
         "reduce_team_connect_local": (i, [vp, ctypes.POINTER(vp)]),
         "reduce_team_destroy": (i, [vp]),
         "reduce_multi_team": (i, [i, i, vp, sz, vp, vp, vp, opts_p]),
+        "reduce_nvls_create": (i, [ctypes.POINTER(vp), vp, i]),
+        "reduce_nvls_create_local": (i, [ctypes.POINTER(vp), i]),
+        "reduce_nvls_destroy": (i, [vp]),
+        "reduce_multi_nvls": (i, [i, i, vp, sz, vp, vp, vp, opts_p]),
     }
     for name, (res, args) in sigs.items():
         f = getattr(L, name)
@@ -474,6 +479,68 @@ def reduce_multi_team(x, op, team: Team, out=None, stream=None, **opt_kw):
                                _stream_handle(stream, x.device), team.handle,
                                ctypes.byref(opts) if opts is not None else None)
     _check(st, "reduce_multi_team")
+    return out
+
+
+class Nvls:
+    """The NVLink SHARP (multicast) combine of reduce_multi_nvls, built over an
+    NCCL communicator (a Comm) -- a collective: every rank constructs it.
+    mode 1: in-switch multimem.ld_reduce; mode 2: multicast store + rank-order
+    combine.  Raises ReduceError(REDUCE_ERR_UNSUPPORTED) on every rank when the
+    ranks have no NVLS multicast (e.g. one GPU)."""
+
+    UNSUPPORTED = 2
+
+    def __init__(self, comm: "Comm" = None, mode: int = 1, group=None, _local=None):
+        if _local is not None:
+            self.handle, self.rank, self.world, self.mode = _local, 0, 1, mode
+            return
+        import torch.distributed as dist
+        h = ctypes.c_void_p()
+        st = lib.reduce_nvls_create(ctypes.byref(h), ctypes.c_void_p(comm.handle), int(mode))
+        err = last_error() if st != OK else ""
+        world = comm.world
+        sts = [None] * world
+        if dist.is_initialized():
+            dist.all_gather_object(sts, (st, err), group=group)
+        else:
+            sts = [(st, err)]
+        if any(s != OK for s, _ in sts):
+            if st == OK and h.value:
+                lib.reduce_nvls_destroy(h)
+            bad = next(r for r, (s, _) in enumerate(sts) if s != OK)
+            raise ReduceError(sts[bad][0], f"Nvls (rank {bad}: {sts[bad][1]})")
+        self.handle, self.rank, self.world, self.mode = h.value, comm.rank, world, mode
+
+    @classmethod
+    def local(cls, mode: int = 1) -> "Nvls":
+        """One-member multicast team on the current GPU (driver multicast API,
+        no NCCL): the NVLS kernels at k = 1, for tests on a single GPU."""
+        h = ctypes.c_void_p()
+        _check(lib.reduce_nvls_create_local(ctypes.byref(h), int(mode)), "reduce_nvls_create_local")
+        return cls(_local=h.value, mode=mode)
+
+    def destroy(self) -> None:
+        if self.handle:
+            _check(lib.reduce_nvls_destroy(ctypes.c_void_p(self.handle)), "reduce_nvls_destroy")
+            self.handle = None
+
+
+def reduce_multi_nvls(x, op, nvls: Nvls, out=None, stream=None, **opt_kw):
+    """Every rank passes its local CUDA shard; every rank gets the global result
+    (cross-GPU combine through NVLS multicast inside the reduction kernel)."""
+    import torch
+    dt = _torch_dtype_code(x)
+    _check_cuda_in(x)
+    if out is None:
+        out = torch.empty(1, dtype=x.dtype, device=x.device)
+    else:
+        _check_out(out, x, 1)
+    opts = make_opts(**opt_kw) if opt_kw else None
+    st = lib.reduce_multi_nvls(dt, _op(op), x.data_ptr() or None, x.numel(), out.data_ptr(),
+                               _stream_handle(stream, x.device), nvls.handle,
+                               ctypes.byref(opts) if opts is not None else None)
+    _check(st, "reduce_multi_nvls")
     return out
 
 

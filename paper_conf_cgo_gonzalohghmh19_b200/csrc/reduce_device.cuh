@@ -177,6 +177,7 @@ __device__ __forceinline__ V warp_butterfly(V v, F f) {
 template <int DT, int OP> struct Tr;
 
 template <int OP> struct TrI32 {
+  static constexpr int kOp = OP;
   using Elem = int32_t;
   using Acc = typename std::conditional<OP == OP_SUM, uint32_t, int32_t>::type;
   using Grid = Acc;
@@ -213,6 +214,7 @@ template <int OP> struct TrI32 {
 };
 
 template <int OP> struct TrF32 {
+  static constexpr int kOp = OP;
   using Elem = float;
   using Acc = float;
   using Grid = typename std::conditional<OP == OP_SUM, double, uint32_t>::type;
@@ -268,6 +270,7 @@ template <int OP> struct TrF32 {
 };
 
 template <int OP> struct TrF64 {
+  static constexpr int kOp = OP;
   using Elem = double;
   using Acc = double;
   using Grid = typename std::conditional<OP == OP_SUM, double, unsigned long long>::type;
@@ -352,6 +355,7 @@ template <int OP> struct TrF64 {
 // s and c are converted to fp64 once per thread (exactly) and everything above
 // the thread runs in fp64.  The per-thread residual is O(n_t u_f^2) sum|x|.
 struct TrF32Acc {
+  static constexpr int kOp = OP_SUMACC;
   using Elem = float;
   using Acc = double;
   using Grid = double;
@@ -391,6 +395,7 @@ struct TrF32Acc {
 // result is hi + lo rounded once.  Non-finite inputs are carried by hi alone
 // (hi is the plain running sum), so inf / NaN follow reading R2.
 struct TrF64Acc {
+  static constexpr int kOp = OP_SUMACC;
   using Elem = double;
   using Acc = double2;  // x = hi, y = lo
   using Grid = double2;

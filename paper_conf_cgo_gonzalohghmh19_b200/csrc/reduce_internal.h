@@ -55,12 +55,29 @@ constexpr int max_block_threads(int dtype, int op, int unroll, int stage = STAGE
 struct TeamArgs {
   char* const* bufs;  // device array of k pointers (nullptr when not a team call)
   int k, rank;
-  int shared_gpu;     // another member runs on this GPU (no early PDL trigger)
+  short shared_gpu;   // another member runs on this GPU (no early PDL trigger)
+  // NVLS exchange (reduce_multi_nvls): bufs[j] is rank j's copy of an NCCL
+  // symmetric window (unicast, over NVLink); bufs[k] is the window's NVLink
+  // SHARP multicast address and bufs[k + 1] this member's call counters
+  // ([0] LL epoch, [1] barrier calls).  nvls: 0 = the peer-store team protocol
+  // above; 1 = arrive on every copy's counter with one multimem.red, then one
+  // multimem.ld_reduce (the reduction happens in the NVSwitch); 2 = one
+  // multimem.st of the value with the call's epoch into every copy
+  // (flag-in-data), then a rank-order combine of the local copy
+  // (deterministic).  (The struct keeps its 24 bytes: a larger kernel
+  // parameter block cost the headline kernel 18 registers.)
+  short nvls;
 };
 constexpr int kTeamMaxRanks = 256;
 constexpr size_t kTeamSlotBytes = 32;
 constexpr size_t kTeamEpochOff = 2 * kTeamMaxRanks * kTeamSlotBytes;
 constexpr size_t kTeamBufBytes = kTeamEpochOff + 16;
+// NVLS window layout (every rank's copy alike)
+constexpr size_t kNvlsCtrOff = 0;      // u32 barrier counter (+k per call, never reset)
+constexpr size_t kNvlsRedOff = 128;    // [parity] 16-byte value slots read by multimem.ld_reduce
+constexpr size_t kNvlsLLOff = 4096;    // [parity][rank] 32-byte {word, epoch} pair slots
+constexpr size_t kNvlsBytes = kNvlsLLOff + 2 * kTeamMaxRanks * kTeamSlotBytes;
+constexpr size_t kNvlsAllocBytes = (size_t)2 << 20;  // the multicast granularity
 
 // One launch of the main reduction kernel (steps S2-S5), fully resolved by the
 // host dispatcher (step S0).
@@ -190,7 +207,7 @@ cudaError_t launch_reduce(const LaunchDesc& d, cudaStream_t s);
 // Reduce `count` Grid-typed values in a fixed order with one block of
 // `block` threads and write the finalised (or raw) result to `out`.
 cudaError_t launch_combine(int dtype, int op, const void* vals, long long count, void* out,
-                           int raw_out, int block, cudaStream_t s, TeamArgs team = TeamArgs{nullptr, 0, 0, 0});
+                           int raw_out, int block, cudaStream_t s, TeamArgs team = TeamArgs{nullptr, 0, 0, 0, 0});
 
 // Write the identity into every accumulator slot of every (dtype, op) and zero
 // the tickets.  slots_base: 9 regions of kMaxSlots*kSlotBytes; tickets: 9 words

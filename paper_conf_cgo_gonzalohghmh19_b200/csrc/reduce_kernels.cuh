@@ -128,9 +128,152 @@ __device__ __noinline__ typename T::Grid team_exchange(typename T::Grid x, char*
   return acc;
 }
 
+// ---- cross-GPU combine through NVLink SHARP multicast -----
+// One thread of the block that owns this rank's raw result x.  bufs[j]: rank
+// j's copy of the NCCL symmetric window (unicast); mc: the window's multicast
+// address -- a store or reduction there reaches every rank's copy through the
+// NVSwitch, a multimem.ld_reduce returns the reduction of all copies.
+//  mode 1: x goes to the own copy's slot [parity]; one multimem.red.release
+//          adds 1 to every copy's barrier counter (the release orders the slot
+//          store before it); when the own counter reaches calls * k every rank
+//          has published, and ONE multimem.ld_reduce reduces the k slots in the
+//          switch.  double-double values (no switch op) are read from the k
+//          copies in rank order instead.
+//  mode 2: one multimem.st puts {word, epoch} pairs into slot [parity][rank]
+//          of every copy (flag-in-data, no fence, as team_exchange); the own
+//          copy is polled until all k slots carry the epoch and combined in
+//          rank order: deterministic for a fixed team.
+// Parity double-buffering as in team_exchange: a slot is rewritten two calls
+// later, after every rank passed the intervening call.
+template <class T>
+__device__ __forceinline__ bool mc_ld_reduce(const char* a, typename T::Grid& r) {
+  using G = typename T::Grid;
+  if constexpr (std::is_same<G, double>::value) {
+    double v;
+    asm volatile("multimem.ld_reduce.relaxed.sys.global.add.f64 %0, [%1];" : "=d"(v) : "l"(a) : "memory");
+    r = v;
+    return true;
+  } else if constexpr (std::is_same<G, uint32_t>::value) {
+    uint32_t v;
+    if constexpr (T::kOp == OP_SUM)
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.add.u32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+    else if constexpr (T::kOp == OP_MIN)
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.min.u32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+    else
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.max.u32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+    r = v;
+    return true;
+  } else if constexpr (std::is_same<G, int32_t>::value) {
+    int32_t v;
+    if constexpr (T::kOp == OP_MIN)
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.min.s32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+    else
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.max.s32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+    r = v;
+    return true;
+  } else if constexpr (std::is_same<G, unsigned long long>::value) {
+    unsigned long long v;
+    if constexpr (T::kOp == OP_MIN)
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.min.u64 %0, [%1];" : "=l"(v) : "l"(a) : "memory");
+    else
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.max.u64 %0, [%1];" : "=l"(v) : "l"(a) : "memory");
+    r = v;
+    return true;
+  } else {
+    return false;
+  }
+}
+
+template <class T>
+__device__ __noinline__ typename T::Grid nvls_exchange(typename T::Grid x, char* const* bufs, int k, int rank, int mode) {
+  using Grid = typename T::Grid;
+  static_assert(sizeof(Grid) <= 16 && sizeof(Grid) % 4 == 0, "nvls slot holds <= 4 words");
+  constexpr int NW = sizeof(Grid) / 4;
+  constexpr int NV = (NW + 1) / 2;
+  char* const mc = bufs[k];
+  volatile unsigned* c = (volatile unsigned*)bufs[k + 1];
+  char* own = bufs[rank];
+  unsigned w[4] = {0u, 0u, 0u, 0u};
+  memcpy(w, &x, sizeof(Grid));
+  if (mode == 1) {
+    const unsigned calls = c[1] + 1;
+    c[1] = calls;
+    const size_t slot = kNvlsRedOff + (size_t)(calls & 1) * 16;
+    asm volatile("st.relaxed.sys.global.v4.u32 [%0], {%1, %2, %3, %4};" :: "l"(own + slot), "r"(w[0]), "r"(w[1]),
+                 "r"(w[2]), "r"(w[3]) : "memory");
+    asm volatile("multimem.red.release.sys.global.add.u32 [%0], 1;" :: "l"(mc + kNvlsCtrOff) : "memory");
+    const unsigned target = calls * (unsigned)k;
+    unsigned got;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(got) : "l"(own + kNvlsCtrOff) : "memory");
+    if ((int)(got - target) < 0) {
+      const long long t0 = clock64();
+      do {
+        __nanosleep(32);
+        if (clock64() - t0 > (1ll << 35)) __trap();  // a member that never arrives: abort, not hang
+        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(got) : "l"(own + kNvlsCtrOff) : "memory");
+      } while ((int)(got - target) < 0);
+    }
+    Grid r;
+    if (mc_ld_reduce<T>(mc + slot, r)) return r;
+    Grid acc = T::gident();
+    for (int j = 0; j < k; ++j) {
+      unsigned v[4];
+      asm volatile("ld.relaxed.sys.global.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3])
+                   : "l"(bufs[j] + slot) : "memory");
+      Grid y;
+      memcpy(&y, v, sizeof(Grid));
+      acc = T::gcomb(acc, y);
+    }
+    return acc;
+  }
+  // mode 2: multicast flag-in-data
+  unsigned epoch = c[0] + 1;
+  if (epoch == 0) epoch = 2;  // 0 means "never written"; keep the parity alternating across the wrap
+  c[0] = epoch;
+  const int par = epoch & 1;
+  char* dst = mc + kNvlsLLOff + ((size_t)par * kTeamMaxRanks + rank) * kTeamSlotBytes;
+#pragma unroll
+  for (int v = 0; v < NV; ++v)
+    asm volatile("multimem.st.relaxed.sys.global.v4.f32 [%0], {%1, %2, %3, %4};" :: "l"(dst + 16 * v),
+                 "f"(__uint_as_float(w[2 * v])), "f"(__uint_as_float(epoch)), "f"(__uint_as_float(w[2 * v + 1])),
+                 "f"(__uint_as_float(epoch)) : "memory");
+  Grid acc = T::gident();
+  for (int j = 0; j < k; ++j) {
+    if (j == rank) {
+      acc = T::gcomb(acc, x);
+      continue;
+    }
+    const unsigned* src = (const unsigned*)(own + kNvlsLLOff + ((size_t)par * kTeamMaxRanks + j) * kTeamSlotBytes);
+    unsigned r[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+    for (int v = 0; v < NV; ++v) {
+      unsigned fa, fb;
+      ld_pairs_sys(src + 4 * v, r[2 * v], fa, r[2 * v + 1], fb);
+      if (fa != epoch || fb != epoch) {
+        const long long t0 = clock64();
+        do {
+          __nanosleep(32);
+          if (clock64() - t0 > (1ll << 35)) __trap();
+          ld_pairs_sys(src + 4 * v, r[2 * v], fa, r[2 * v + 1], fb);
+        } while (fa != epoch || fb != epoch);
+      }
+    }
+    Grid y;
+    memcpy(&y, r, sizeof(Grid));
+    acc = T::gcomb(acc, y);
+  }
+  return acc;
+}
+
+// The cross-rank step: scalars by value into the __noinline__ exchanges (a
+// reference to the parameter struct would copy it to the stack).
+#define RB_CROSS_RANK(T, g, t)                                                              \
+  ((t).nvls ? nvls_exchange<T>((g), (t).bufs, (t).k, (t).rank, (t).nvls)                     \
+            : team_exchange<T>((g), (t).bufs, (t).k, (t).rank))
+
 template <class T>
 __device__ __forceinline__ void store_out(typename T::Grid g, const KParams& p) {
-  if (p.team.k > 0) g = team_exchange<T>(g, p.team.bufs, p.team.k, p.team.rank);
+  if (p.team.k > 0) g = RB_CROSS_RANK(T, g, p.team);
   if (p.raw_out) *(typename T::Grid*)p.out = g;
   else T::finalize(g, p.out);
 }
@@ -373,7 +516,7 @@ __global__ void __launch_bounds__(1024) k_combine(const void* vals, long long co
   pdl_wait();
   typename T::Grid x = reduce_grid_values<T>((const typename T::Grid*)vals, count);
   if (threadIdx.x == 0) {
-    if (team.k > 0) x = team_exchange<T>(x, team.bufs, team.k, team.rank);
+    if (team.k > 0) x = RB_CROSS_RANK(T, x, team);
     if (raw_out) *(typename T::Grid*)out = x;
     else T::finalize(x, out);
   }

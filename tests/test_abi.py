@@ -179,3 +179,13 @@ def test_shard_range_partitions_exactly():
             assert ranges[0][0] == 0 and ranges[-1][1] == n
             assert all(a[1] == b[0] for a, b in zip(ranges, ranges[1:]))
             assert max(h - l for l, h in ranges) - min(h - l for l, h in ranges) <= 1
+
+
+def test_nvls_entry_points_reject_bad_arguments_without_cuda():
+    h = ctypes.c_void_p()
+    assert rb.lib.reduce_nvls_create_local(ctypes.byref(h), 3) == 1      # bad mode
+    assert rb.lib.reduce_nvls_create(ctypes.byref(h), None, 1) == 1      # no communicator
+    assert rb.lib.reduce_nvls_create(None, ctypes.c_void_p(8), 1) == 1   # no output
+    assert rb.lib.reduce_nvls_destroy(None) == 1
+    assert rb.lib.reduce_multi_nvls(1, 0, None, 0, None, None, None, None) == 1  # out NULL
+    assert "mode" in rb.last_error() or "NULL" in rb.last_error()

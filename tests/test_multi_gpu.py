@@ -1,6 +1,8 @@
 """Sharded mode on real GPUs: reduce_multi over NCCL (world = number of visible
 GPUs, capped at 8; the 1-GPU box runs world 1, which still exercises the
-NCCL all-reduce / all-gather + finalise path end to end)."""
+NCCL all-reduce / all-gather + finalise path end to end), and the NVLS
+combine (reduce_multi_nvls): parity where multicast exists, a clean
+REDUCE_ERR_UNSUPPORTED where it does not."""
 import json
 import os
 import subprocess
@@ -25,3 +27,11 @@ def test_reduce_multi_matches_oracle_of_concatenation():
     for l in lines:
         assert l["checked"] > 0 and not l["fails"], l
         assert l["deterministic_distinct"] == 1, l
+        assert l["comm_after_nvls"] == 1000.0 * world, l
+        for mode, r in l["nvls"].items():
+            if r["status"] == 0:   # NVLS multicast available: parity like reduce_multi
+                assert r["checked"] > 0 and not r["fails"], (mode, r)
+            else:                  # e.g. the 1-GPU box: a clean REDUCE_ERR_UNSUPPORTED
+                assert r["status"] == 2, (mode, r)
+    # every rank took the same branch
+    assert len({json.dumps({m: r["status"] for m, r in l["nvls"].items()}) for l in lines}) == 1
