@@ -65,9 +65,11 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--sharded", action="store_true",
                     help="use the sharded path even at one rank (exercises S7 on one GPU)")
-    ap.add_argument("--collective", default="team", choices=["team", "nccl"],
+    ap.add_argument("--collective", default="team", choices=["team", "nccl", "nvls"],
                     help="cross-GPU combine: 'team' = fused into the reduction kernel over peer memory "
-                         "(reduce_multi_team), 'nccl' = one ncclAllReduce of the per-rank scalar")
+                         "(reduce_multi_team), 'nccl' = one ncclAllReduce of the per-rank scalar, 'nvls' = "
+                         "fused into the kernel through NVLink SHARP multicast (reduce_multi_nvls: "
+                         "multimem.ld_reduce in the NVSwitch)")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="which series is the line's `value`: weak = --elements per GPU, strong = "
                          "--strong-total elements split over the N GPUs (both are always reported)")
@@ -310,8 +312,9 @@ def workload_config(args, world, plan, sharded=False):
     cfg = {"workload": f"fp32 sum of {args.n} (2^{args.n.bit_length() - 1}) elements per GPU"
                        + (" -- BASELINE configs[1] largest point" if world == 1 else
                           f" -- BASELINE configs[4] sharded sum, {world} GPUs, per-rank partials combined "
-                          + ("in the reduction kernel over peer memory (reduce_multi_team)" if args.collective == "team"
-                             else "by one NCCL all-reduce")),
+                          + {"team": "in the reduction kernel over peer memory (reduce_multi_team)",
+                             "nvls": "in the reduction kernel through NVLS multicast (reduce_multi_nvls)",
+                             "nccl": "by one NCCL all-reduce"}[args.collective]),
            "n_per_gpu": args.n, "total_bytes": args.n * 4 * world, "op": "sum", "mode": args.mode,
            "parallelism": f"shard{world}" if (world > 1 or sharded) else "single-gpu",
            "collective": args.collective if (world > 1 or sharded) else None,
@@ -402,13 +405,23 @@ def main():
                 raise
             combines["team"] = None
             collective_note = f"team combine unavailable ({e})"
+        nvls_note = None
         if args.share_gpu:
             combines["nccl"] = None  # NCCL refuses two ranks on one GPU
+            combines["nvls"] = None
+            nvls_note = "ranks share one GPU"
         else:
             combines["nccl"] = rb.Comm()
+            try:  # a collective: every rank gets the same outcome
+                combines["nvls"] = rb.Nvls(combines["nccl"], mode=1)
+            except rb.ReduceError as e:
+                combines["nvls"] = None
+                nvls_note = str(e)[-200:]
         if combines.get(args.collective) is None:
-            if args.collective == "team" and combines.get("nccl") is not None:
-                collective_note = (collective_note or "team combine unavailable") + "; fell back to the NCCL all-reduce"
+            if args.collective in ("team", "nvls") and combines.get("nccl") is not None:
+                collective_note = ((collective_note or f"{args.collective} combine unavailable")
+                                   + (f" ({nvls_note})" if args.collective == "nvls" else "")
+                                   + "; fell back to the NCCL all-reduce")
                 print(f"bench: {collective_note}", file=sys.stderr)
                 args.collective = "nccl"
             else:
@@ -417,6 +430,7 @@ def main():
         comm_info = {"world_size": world,
                      "team_members": None if combines.get("team") is None else combines["team"].world,
                      "nccl_comm_nranks": None if combines.get("nccl") is None else combines["nccl"].nranks(),
+                     "nvls": "available" if combines.get("nvls") is not None else f"unavailable: {nvls_note}",
                      "process_group_backend": dist.get_backend()}
         if comm_info["nccl_comm_nranks"] not in (None, world) or comm_info["team_members"] not in (None, world):
             raise SystemExit(f"bench: communicator size disagrees with WORLD_SIZE: {comm_info}")
@@ -426,6 +440,8 @@ def main():
     def sharded_call(name, xt, o):
         if name == "team":
             rb.reduce_multi_team(xt, "sum", combines["team"], out=o, stream=stream, mode=args.mode)
+        elif name == "nvls":
+            rb.reduce_multi_nvls(xt, "sum", combines["nvls"], out=o, stream=stream, mode=args.mode)
         else:
             rb.reduce_multi(xt, "sum", combines["nccl"], out=o, stream=stream, mode=args.mode)
 
@@ -474,9 +490,10 @@ def main():
     cross_check = None
     if comm is not None:
         cross_check = {}
-        for name in ("team", "nccl"):
+        for name in ("team", "nccl", "nvls"):
             cross_check[name] = (cross_rank_check(name, x) if combines.get(name) is not None
-                                 else "unavailable" + (" (ranks share one GPU)" if args.share_gpu and name == "nccl" else ""))
+                                 else "unavailable" + (" (ranks share one GPU)" if args.share_gpu and name != "team"
+                                                       else (f" ({nvls_note})" if name == "nvls" else "")))
         sync_all()
     # Single GPU: the K steps are captured once into a CUDA graph and replayed
     # (no host launch gaps between steps; the same kernels on the same
@@ -663,10 +680,7 @@ def main():
             with torch.cuda.stream(stream):
                 for _ in range(k_e2e):
                     xd.copy_(pinned, non_blocking=True)
-                    if args.collective == "team":
-                        rb.reduce_multi_team(xd, "sum", comm, out=out, stream=stream, mode=args.mode)
-                    else:
-                        rb.reduce_multi(xd, "sum", comm, out=out, stream=stream, mode=args.mode)
+                    sharded_call(args.collective, xd, out)
                     out.item()
             dt = allmax((time.perf_counter() - t0) / k_e2e)
         # the PCIe ceiling e2e runs against: a plain pinned H2D copy of the same bytes
@@ -1015,9 +1029,9 @@ def main():
         torch.cuda.synchronize(dev)
         if world > 1:
             dist.barrier()  # no member may unmap its team buffer while others still use it
-        for c in combines.values():
-            if c is not None:
-                c.destroy()
+        for name in ("nvls", "team", "nccl"):  # the NVLS window before the communicator it lives on
+            if combines.get(name) is not None:
+                combines[name].destroy()
         dist.destroy_process_group()
 
 
