@@ -73,7 +73,8 @@ struct Bal {
   static constexpr int kList = (int)C + 64;           // offsets entries kept in shared memory
   static constexpr size_t kPieceBytes = (size_t)EL * 32 * sizeof(Acc);
   static constexpr size_t kListBytes = ((size_t)kList * 2 + 15) / 16 * 16;
-  static constexpr size_t kWarpSmem = kPieceBytes + kListBytes;
+  static constexpr size_t kLaneBytes = 32 * 4 * 2;  // per lane: boundary mask word, list entries count
+  static constexpr size_t kWarpSmem = kPieceBytes + kListBytes + kLaneBytes;
 };
 
 // Element index (relative to `in`) of the 32-byte-aligned address at or below
@@ -146,7 +147,7 @@ struct BalRanges {
   }
 };
 
-template <int DT, int OP>
+template <int DT, int OP, int K>
 __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
   using T = Tr<DT, OP>;
   using B = Bal<T>;
@@ -155,10 +156,8 @@ __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
   const long long E0 = __ldg(p.offsets), E1 = __ldg(p.offsets + p.nseg);
   const long long P0 = bal_origin<B::s>(p.in, E0);
   const long long nchunks = E1 > E0 ? (E1 - P0 + B::C - 1) / B::C : 0;
-  const long long stride = (long long)gridDim.x * blockDim.x;
-#pragma unroll 1
-  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < p.nseg; i += stride) {
-    const long long lo = __ldg(p.offsets + i), hi = __ldg(p.offsets + i + 1);
+  const BalRanges R(nchunks > 0 ? nchunks : 1, p.b.nranges);
+  auto one = [&](long long i, long long lo, long long hi) {
     if (hi < lo) atomicOr(p.b.hdr, 1u);
     if (hi <= lo) {
       seg_store<T>(p, i, T::gident());
@@ -169,10 +168,22 @@ __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
       long long c1 = (hi - P0 + B::C - 1) / B::C;
       if (c1 > nchunks) c1 = nchunks;
       if (c0 < c1) {  // only segments holding a chunk start (the range arithmetic divides)
-        const BalRanges R(nchunks, p.b.nranges);
         for (long long w = R.first_at(c0); w < p.b.nranges && R.begin(w) < c1; ++w) p.b.start_seg[w] = (unsigned)i;
       }
     }
+  };
+  // K consecutive segments per thread per step (K from the host: the fewest
+  // steps for the grid), their K + 1 offsets loaded before any is used -- the
+  // loop is latency-bound, one round trip per step
+  const long long nthreads = (long long)gridDim.x * blockDim.x;
+#pragma unroll 1
+  for (long long i0 = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * K; i0 < p.nseg; i0 += nthreads * K) {
+    long long o[K + 1];
+#pragma unroll
+    for (int j = 0; j <= K; ++j) o[j] = i0 + j <= p.nseg ? __ldg(p.offsets + i0 + j) : LLONG_MAX;
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+      if (i0 + j < p.nseg) one(i0 + j, o[j], o[j + 1]);
   }
   pdl_trigger();
 }
@@ -295,6 +306,8 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   Acc* pieces = reinterpret_cast<Acc*>(bal_smem + wib * B::kWarpSmem);
   short* list = reinterpret_cast<short*>(bal_smem + wib * B::kWarpSmem + B::kPieceBytes);
+  unsigned* lmask = reinterpret_cast<unsigned*>(bal_smem + wib * B::kWarpSmem + B::kPieceBytes + B::kListBytes);
+  unsigned* lcnt = lmask + 32;
   pdl_wait();
   const long long nseg = p.nseg;
   const long long E0 = __ldg(p.offsets), E1 = __ldg(p.offsets + nseg);
@@ -363,6 +376,12 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
     int m = 0;
     bool ovf = false;
     long long v = vfirst;
+    // per lane: the bits of the boundaries in its elements and how many list
+    // entries fall there, set with shared atomics as the list is built (no
+    // per-lane search of the list afterwards)
+    lmask[lane] = 0u;
+    lcnt[lane] = 0u;
+    __syncwarp();
     // batches past the two prefetched ones are loaded four at a time (chunks
     // of very short segments need dozens: one round trip per four, not per one)
     long long q0 = 0, q1 = 0, q2 = 0, q3 = 0;
@@ -376,7 +395,13 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
         ovf = true;
         break;
       }
-      if (lane < cnt) list[m + lane] = (short)loc;
+      if (lane < cnt) {
+        list[m + lane] = (short)loc;
+        if (loc >= 0 && loc < (int)B::C) {
+          atomicOr(lmask + loc / B::EL, 1u << (loc % B::EL));
+          atomicAdd(lcnt + loc / B::EL, 1u);
+        }
+      }
       m += cnt;
       if (stop) break;
       base += 32;
@@ -407,17 +432,18 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
     unsigned fb = 0;
     Acc tv = T::ident();  // the lane's value (no boundary in the chunk) or its last piece
     if (!ovf) {
-      // the lane's boundaries as a bit mask (bit e: a segment starts at element e)
-      const int a0 = lane * B::EL;
-      {
-        int hi_i = m - 1;  // list[m - 1] == C > a0
-        while (i0 < hi_i) {
-          const int mid = (i0 + hi_i) >> 1;
-          if (list[mid] < a0) i0 = mid + 1; else hi_i = mid;
-        }
+      // the lane's boundaries as a bit mask (bit e: a segment starts at element e),
+      // and i0 = the list index of its first boundary: the entries before the
+      // chunk (list[0] == -1) plus those of the lanes below
+      mask = lmask[lane];
+      const int cnt = (int)lcnt[lane];
+      int incl = cnt;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const int y = __shfl_up_sync(0xffffffffu, incl, d);
+        if (lane >= d) incl += y;
       }
-#pragma unroll 1
-      for (int j = i0; list[j] < a0 + B::EL; ++j) mask |= 1ull << (list[j] - a0);
+      i0 = incl - cnt + (list[0] < 0 ? 1 : 0);
       fb = __ballot_sync(0xffffffffu, mask != 0ull);
       if (fb == 0u) {  // no boundary in the chunk: plain vector-tree fold
         Part<T> acc[T::NA];
@@ -595,9 +621,14 @@ cudaError_t launch_segbal_op(const SegParams& p0, int sms, cudaStream_t s) {
   long long grid = (long long)sms * per_sm;  // one wave: every warp owns one contiguous chunk range
   if (grid * kBalWarps > (long long)kBalRanges) grid = kBalRanges / kBalWarps;
   p.b.nranges = grid * kBalWarps;
-  long long sgrid = (p.nseg + 255) / 256;
+  // the scan: one step per thread where the grid allows (K segments each)
+  const long long full = (long long)sms * 8 * 256;
+  const int K = p.nseg <= full ? 1 : (p.nseg <= 4 * full ? 4 : 8);
+  long long sgrid = (p.nseg + 256ll * K - 1) / (256ll * K);
   if (sgrid > (long long)sms * 8) sgrid = (long long)sms * 8;
-  e = bal_launch(k_segbal_scan<DT, OP>, sgrid, 256, 0, p, s);
+  e = K == 1 ? bal_launch(k_segbal_scan<DT, OP, 1>, sgrid, 256, 0, p, s)
+             : (K == 4 ? bal_launch(k_segbal_scan<DT, OP, 4>, sgrid, 256, 0, p, s)
+                       : bal_launch(k_segbal_scan<DT, OP, 8>, sgrid, 256, 0, p, s));
   if (e != cudaSuccess) return e;
   e = bal_launch(k_segbal<DT, OP>, grid, kBalWarps * 32, smem, p, s);
   if (e != cudaSuccess) return e;
