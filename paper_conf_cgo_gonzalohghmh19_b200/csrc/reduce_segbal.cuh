@@ -428,6 +428,7 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
     if (ovf) k.s_next = bal_walk_next(p.offsets, nseg, s0 + m, chi, lane);
     if (c + 1 < ce) prefetch_list(k.s_next);  // the next chunk's offsets, while this one folds
     int i0 = 0, np = 0;
+    bool lane_dups = false;
     unsigned long long mask = 0;
     unsigned fb = 0;
     Acc tv = T::ident();  // the lane's value (no boundary in the chunk) or its last piece
@@ -444,6 +445,7 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
         if (lane >= d) incl += y;
       }
       i0 = incl - cnt + (list[0] < 0 ? 1 : 0);
+      lane_dups = cnt != __popcll(mask);  // repeated offsets (empty segments) in this lane's elements
       fb = __ballot_sync(0xffffffffu, mask != 0ull);
       if (fb == 0u) {  // no boundary in the chunk: plain vector-tree fold
         Part<T> acc[T::NA];
@@ -503,13 +505,21 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
           } else {                          // the chunk's first boundary: the incoming segment's piece
             firstv = T::to_grid(close);
           }
-          int j = i0;
+          // segments that start and end in this lane: the one opened by the
+          // lane's q-th boundary is s0 + (its list index); without repeated
+          // offsets in the lane that index is i0 + q - 1
+          if (!lane_dups) {
 #pragma unroll 1
-          for (int q = 1; q < np; ++q) {  // segments that start and end in this lane
-            const int o = list[j];
-            while (list[j + 1] == o) ++j;
-            bal_store<T>(p, (long long)s0 + j, T::to_grid(pieces[q * 32 + lane]));
-            ++j;
+            for (int q = 1; q < np; ++q) bal_store<T>(p, (long long)s0 + i0 + q - 1, T::to_grid(pieces[q * 32 + lane]));
+          } else {
+            int j = i0;
+#pragma unroll 1
+            for (int q = 1; q < np; ++q) {
+              const int o = list[j];
+              while (list[j + 1] == o) ++j;
+              bal_store<T>(p, (long long)s0 + j, T::to_grid(pieces[q * 32 + lane]));
+              ++j;
+            }
           }
         }
         k.first = shfl_idx_v(firstv, __ffs(fb) - 1);
