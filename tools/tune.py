@@ -98,23 +98,35 @@ def run(args):
                 # >= 20 calls per timed graph; regions repeat only when each is > 2x L2
                 R = max(20, min(100, (400 << 20) // nbytes)) if nbytes >= (256 << 20) else max(5, min(100, (400 << 20) // nbytes))
                 warm, timed = disjoint_regions(pool, R, n)
-                best = None
-                for c in candidates(dtype, op, mode, lb):
-                    opts = rb.make_opts(mode=mode, **c)
-                    k = [0]
+                # every candidate timed in `rounds` interleaved rounds (box-level
+                # drift hits all candidates alike), the median per candidate decides
+                cands = candidates(dtype, op, mode, lb)
+                times = [[] for _ in cands]
+                failed = set()
+                for rnd in range(args.rounds):
+                    for ci, c in enumerate(cands):
+                        if ci in failed:
+                            continue
+                        opts = rb.make_opts(mode=mode, **c)
+                        k = [0]
 
-                    def launch(t, opts=opts):
-                        i = k[0] = (k[0] + 1) % 4096
-                        rb.reduce_ptr(DT[dtype], op, t.data_ptr(), t.numel(), out[i:i + 1].data_ptr(),
-                                      stream.cuda_stream, opts)
-                    try:
-                        s = time_calls(launch, warm, timed, stream, repeats=2)
-                    except Exception as e:  # an invalid combination: record and skip
-                        results.append(dict(dtype=dtype, op=op, mode=mode, lb=lb, cfg=c, error=str(e)[:200]))
-                        torch.cuda.synchronize()
+                        def launch(t, opts=opts):
+                            i = k[0] = (k[0] + 1) % 4096
+                            rb.reduce_ptr(DT[dtype], op, t.data_ptr(), t.numel(), out[i:i + 1].data_ptr(),
+                                          stream.cuda_stream, opts)
+                        try:
+                            times[ci].append(time_calls(launch, warm, timed, stream, repeats=1))
+                        except Exception as e:  # an invalid combination: record and skip
+                            results.append(dict(dtype=dtype, op=op, mode=mode, lb=lb, cfg=c, error=str(e)[:200]))
+                            torch.cuda.synchronize()
+                            failed.add(ci)
+                best = None
+                for ci, c in enumerate(cands):
+                    if ci in failed or not times[ci]:
                         continue
+                    s = sorted(times[ci])[len(times[ci]) // 2]
                     results.append(dict(dtype=dtype, op=op, mode=mode, lb=lb, cfg=c, us=s * 1e6,
-                                        gbps=nbytes / s / 1e9))
+                                        gbps=nbytes / s / 1e9, rounds_us=[round(t * 1e6, 3) for t in times[ci]]))
                     if best is None or s < best[0]:
                         best = (s, c)
                 print(f"[{time.time() - t_start:7.1f}s] {dtype} {op} {mode} 2^{lb}B: best {best[0] * 1e6:8.2f} us "
@@ -189,6 +201,7 @@ def main():
     ap.add_argument("--min-lb", type=int, default=7)
     ap.add_argument("--max-lb", type=int, default=30)
     ap.add_argument("--out", default="gpurun_out/tune.json")
+    ap.add_argument("--rounds", type=int, default=3, help="interleaved timing rounds per candidate (median wins)")
     ap.add_argument("--emit", nargs="*")
     ap.add_argument("--dst", default=os.path.join(ROOT, "paper_conf_cgo_gonzalohghmh19_b200", "csrc",
                                                   "dispatch_table.inc"))
