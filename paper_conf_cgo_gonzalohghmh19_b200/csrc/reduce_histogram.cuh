@@ -28,6 +28,15 @@
 namespace rb {
 
 constexpr int kHistSharedMaxBins = 16384;  // 64 KB of u32 counters per block
+// A/B hooks (profiles/r02_hist_ab.txt, B200, 1 GiB): four vectors in flight
+// per thread on the replicated 32-bit path (+2-4 %), the next pair of vectors
+// loaded while the 16-bit path updates the current one (+1.6-3.4 %).
+#ifndef RB_HIST_V4
+#define RB_HIST_V4 1
+#endif
+#ifndef RB_HIST16_PIPE
+#define RB_HIST16_PIPE 1
+#endif
 
 // Bin of one element, or -1 if it is not counted.  Branch-free (selects and
 // predicated corrections), so the bins of a whole vector are computed with
@@ -115,6 +124,19 @@ __global__ void __launch_bounds__(256) k_histogram(const HistParams p, int parts
   }
   const unsigned long long stride = (unsigned long long)nblk * blockDim.x;
   unsigned long long v = (unsigned long long)blk * blockDim.x + threadIdx.x;
+#if RB_HIST_V4
+  for (; v + 3 * stride < p.body_vecs; v += 4 * stride) {
+    uint32_t r0[8], r1[8], r2[8], r3[8];
+    ld_v8(p.body + v * kVecBytes, r0);
+    ld_v8(p.body + (v + stride) * kVecBytes, r1);
+    ld_v8(p.body + (v + 2 * stride) * kVecBytes, r2);
+    ld_v8(p.body + (v + 3 * stride) * kVecBytes, r3);
+    hist_vec<DT, kShared>(r0, p, sbase, sdummy, rep_log2, b0, b1);
+    hist_vec<DT, kShared>(r1, p, sbase, sdummy, rep_log2, b0, b1);
+    hist_vec<DT, kShared>(r2, p, sbase, sdummy, rep_log2, b0, b1);
+    hist_vec<DT, kShared>(r3, p, sbase, sdummy, rep_log2, b0, b1);
+  }
+#endif
   for (; v + stride < p.body_vecs; v += 2 * stride) {
     uint32_t r0[8], r1[8];
     ld_v8(p.body + v * kVecBytes, r0);
@@ -199,6 +221,31 @@ __global__ void __launch_bounds__(1024) k_histogram16(const HistParams p) {
   };
   const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
   unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
+#if RB_HIST16_PIPE
+  // software pipeline: the next pair of vectors is in flight while this pair's
+  // counters are updated (the returning shared atomics of 16 elements take
+  // longer than a load round trip under bank conflicts)
+  if (v + stride < p.body_vecs) {
+    uint32_t r0[8], r1[8];
+    ld_v8(p.body + v * kVecBytes, r0);
+    ld_v8(p.body + (v + stride) * kVecBytes, r1);
+    v += 2 * stride;
+    for (; v + stride < p.body_vecs; v += 2 * stride) {
+      uint32_t n0[8], n1[8];
+      ld_v8(p.body + v * kVecBytes, n0);
+      ld_v8(p.body + (v + stride) * kVecBytes, n1);
+      count8(r0);
+      count8(r1);
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        r0[k] = n0[k];
+        r1[k] = n1[k];
+      }
+    }
+    count8(r0);
+    count8(r1);
+  }
+#else
   for (; v + stride < p.body_vecs; v += 2 * stride) {
     uint32_t r0[8], r1[8];
     ld_v8(p.body + v * kVecBytes, r0);
@@ -206,6 +253,7 @@ __global__ void __launch_bounds__(1024) k_histogram16(const HistParams p) {
     count8(r0);
     count8(r1);
   }
+#endif
   if (v < p.body_vecs) {
     uint32_t r[8];
     ld_v8(p.body + v * kVecBytes, r);
