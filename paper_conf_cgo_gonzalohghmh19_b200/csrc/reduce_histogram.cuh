@@ -37,6 +37,17 @@ constexpr int kHistSharedMaxBins = 16384;  // 64 KB of u32 counters per block
 #ifndef RB_HIST16_PIPE
 #define RB_HIST16_PIPE 1
 #endif
+// 16-bit path: non-returning shared atomics with block-synchronous flushes
+// (k_histogram16r, 65536 bins 3.21 -> 3.78 TB/s fp32, 3.34 -> 3.67 TB/s int32)
+// instead of a returning atomic and a carry check per update (k_histogram16);
+// RB_HIST16_VPI vectors per thread per flush (0: 4 for int32, whose bin
+// arithmetic needs more registers, 6 for fp32; profiles/r02_hist_ab.txt)
+#ifndef RB_HIST16_RED
+#define RB_HIST16_RED 1
+#endif
+#ifndef RB_HIST16_VPI
+#define RB_HIST16_VPI 0
+#endif
 
 // Bin of one element, or -1 if it is not counted.  Branch-free (selects and
 // predicated corrections), so the bins of a whole vector are computed with
@@ -277,6 +288,98 @@ __global__ void __launch_bounds__(1024) k_histogram16(const HistParams p) {
   }
 }
 
+// The same one-pass 16-bit histogram with NON-returning shared atomics
+// (red.shared) and block-synchronous flushes instead of a carry check per
+// update.  Every iteration each thread counts VPI vectors (8 VPI elements, 8 VPI
+// x 1024 per block); then, after a barrier, the block scans its counters and
+// moves every half that reached T (the multiple of T it holds) to `counts`.
+// After a flush every half is < T and an iteration adds at most 8 VPI x 1024,
+// with T + 8 VPI x 1024 <= 0xFFFF: a half never passes 0xFFFF and never
+// spills into its neighbour.
+// Uniform data never moves anything; the scan costs one 16-byte shared load per
+// four words per iteration.
+template <int DT>
+__global__ void __launch_bounds__(1024) k_histogram16r(const HistParams p) {
+  extern __shared__ unsigned sw[];
+  const int words = (p.nbins + 1) >> 1;
+  const int words4 = (words + 3) & ~3;  // the scan reads uint4
+  for (int i = threadIdx.x; i < words4 + 32; i += blockDim.x) sw[i] = 0u;
+  __syncthreads();
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sw);
+  const uint32_t sdummy = sbase + 4u * (uint32_t)(words4 + (threadIdx.x & 31));
+  auto count8 = [&](const uint32_t (&r)[8]) {
+    int bin[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) bin[k] = hist_bin<DT>(r[k], p);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {  // unconditional (uncounted elements add 0 to the lane's dummy word)
+      const bool ok = bin[k] >= 0;
+      const uint32_t a = ok ? sbase + 4u * (uint32_t)(bin[k] >> 1) : sdummy;
+      const uint32_t inc = ok ? 1u << ((bin[k] & 1) << 4) : 0u;
+      asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(inc) : "memory");
+    }
+  };
+  // VPI vectors per thread per iteration (8 VPI x 1024 elements per block); a
+  // half is moved once it reaches T, the largest power of two with
+  // T + 8 VPI x 1024 <= 0xFFFF
+  constexpr int VPI = RB_HIST16_VPI > 0 ? RB_HIST16_VPI : (DT == DT_I32 ? 4 : 6);
+  constexpr unsigned kE = 8u * VPI * 1024u;
+  constexpr unsigned kT = kE <= 32767u ? 16384u : (kE <= 49151u ? 16384u >> 1 : (kE <= 57343u ? 4096u : 2048u));
+  static_assert(kT + kE <= 0xFFFFu, "a half could wrap");
+  constexpr unsigned kHalfMask = (~(kT - 1u)) & 0xFFFFu;
+  constexpr unsigned kMask = kHalfMask | (kHalfMask << 16);
+  auto flush = [&]() {
+    __syncthreads();
+    for (int i = 4 * (int)threadIdx.x; i < words4; i += 4 * (int)blockDim.x) {
+      const uint4 w = *reinterpret_cast<const uint4*>(sw + i);
+      if (((w.x | w.y | w.z | w.w) & kMask) == 0u) continue;  // every half < T
+      const unsigned ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const unsigned lo = ws[j] & kHalfMask, hi = (ws[j] >> 16) & kHalfMask;
+        if (lo | hi) {
+          atomicSub(&sw[i + j], lo | (hi << 16));
+          if (lo) atomicAdd(p.counts + 2 * (i + j), lo);
+          if (hi) atomicAdd(p.counts + 2 * (i + j) + 1, hi);
+        }
+      }
+    }
+    __syncthreads();
+  };
+  const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
+  unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
+  // every thread of the block runs the same number of iterations (the barrier
+  // in flush): vectors past the body are skipped inside
+  const unsigned long long per_iter = VPI * stride;
+  const unsigned long long iters = (p.body_vecs + per_iter - 1) / per_iter;
+  for (unsigned long long it = 0; it < iters; ++it, v += per_iter) {
+    uint32_t r[VPI][8];
+#pragma unroll
+    for (int u = 0; u < VPI; ++u)
+      if (v + u * stride < p.body_vecs) ld_v8(p.body + (v + u * stride) * kVecBytes, r[u]);
+#pragma unroll
+    for (int u = 0; u < VPI; ++u)
+      if (v + u * stride < p.body_vecs) count8(r[u]);
+    flush();
+  }
+  if (blockIdx.x == 0 && threadIdx.x < 16) {  // head and tail elements (< 8 each)
+    const int t = threadIdx.x;
+    const bool mine = t < p.head || (t >= 8 && t - 8 < p.tail);
+    if (mine) {
+      const uint32_t w = t < p.head ? __ldg((const uint32_t*)p.in + t)
+                                    : __ldg((const uint32_t*)(p.body + p.body_vecs * kVecBytes) + (t - 8));
+      const int bn = hist_bin<DT>(w, p);
+      if (bn >= 0) atomicAdd(p.counts + bn, 1u);
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < words; i += blockDim.x) {
+    const unsigned w = sw[i];
+    if (w & 0xFFFFu) atomicAdd(p.counts + 2 * i, w & 0xFFFFu);
+    if (w >> 16) atomicAdd(p.counts + 2 * i + 1, w >> 16);
+  }
+}
+
 // Copies per bin: as many as keep a block's bins within 64 KB (<= 32).
 inline int hist_rep_log2(int bins_per_block) {
   int rl = 5;
@@ -294,11 +397,12 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
   if (p.nbins > kHistSharedMaxBins) {  // one pass with 16-bit shared counters if the histogram fits
     int optin = 0;
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-    const size_t smem16 = ((size_t)(p.nbins + 1) / 2 + 32) * sizeof(unsigned);
+    const size_t smem16 = (((size_t)(p.nbins + 1) / 2 + 3) / 4 * 4 + 32) * sizeof(unsigned);
     if (smem16 <= (size_t)optin) {
-      e = opt_in_smem((const void*)k_histogram16<DT>, (int)smem16);
+      auto k16 = RB_HIST16_RED ? k_histogram16r<DT> : k_histogram16<DT>;
+      e = opt_in_smem((const void*)k16, (int)smem16);
       if (e != cudaSuccess) return e;
-      const int per_sm = blocks_per_sm((const void*)k_histogram16<DT>, 1024, smem16);
+      const int per_sm = blocks_per_sm((const void*)k16, 1024, smem16);
       long long grid = (long long)sms * per_sm;
       const long long need = (long long)((p.body_vecs + 1023) / 1024);
       if (need < grid) grid = need < 1 ? 1 : need;
@@ -308,7 +412,7 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
       cfg.dynamicSmemBytes = smem16;
       cfg.stream = s;
       cfg.numAttrs = 0;
-      return cudaLaunchKernelEx(&cfg, k_histogram16<DT>, p);
+      return cudaLaunchKernelEx(&cfg, k16, p);
     }
   }
   const int parts = (p.nbins + kHistSharedMaxBins - 1) / kHistSharedMaxBins;
