@@ -17,7 +17,8 @@ for dt in (torch.int32, torch.float32, torch.float64):
         x = torch.arange(n + 3, device="cuda").to(dt)[3:]
         for op in ("sum", "min", "max"):
             for kw in (dict(), dict(mode="deterministic"), dict(grid_combine=3), dict(grid_combine=4, grid=8),
-                       dict(stage="smem", unroll=8, block=256), dict(block_combine=1), dict(block_combine=3, block=128)):
+                       dict(stage="smem", unroll=8, block=256), dict(block_combine=1), dict(block_combine=3, block=128),
+                       dict(input_ready=True), dict(grid_combine=1, block=32, unroll=1)):
                 rb.reduce(x, op, **kw)
         if dt != torch.int32:
             rb.reduce(x, "sum_accurate")
