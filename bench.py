@@ -75,6 +75,9 @@ def parse():
                          "--strong-total elements split over the N GPUs (both are always reported)")
     ap.add_argument("--strong-total", type=int, default=1 << 31,
                     help="total elements of the strong-scaling array (default 2^31 = 8 GiB fp32, configs[4])")
+    ap.add_argument("--nvls-check", action="store_true",
+                    help="also build the NVLS combine (reduce_multi_nvls) and cross-check it (it is built anyway "
+                         "with --collective nvls)")
     ap.add_argument("--share-gpu", action="store_true",
                     help="TEST MODE: every rank on cuda:0, gloo control plane, team combine over CUDA IPC "
                          "(validates the multi-rank path on a one-GPU box; timings are not scaling numbers)")
@@ -412,11 +415,15 @@ def main():
             nvls_note = "ranks share one GPU"
         else:
             combines["nccl"] = rb.Comm()
-            try:  # a collective: every rank gets the same outcome
-                combines["nvls"] = rb.Nvls(combines["nccl"], mode=1)
-            except rb.ReduceError as e:
+            if args.collective == "nvls" or args.nvls_check:
+                try:  # a collective: every rank gets the same outcome
+                    combines["nvls"] = rb.Nvls(combines["nccl"], mode=1)
+                except rb.ReduceError as e:
+                    combines["nvls"] = None
+                    nvls_note = str(e)[-200:]
+            else:
                 combines["nvls"] = None
-                nvls_note = str(e)[-200:]
+                nvls_note = "not requested (--collective nvls or --nvls-check)"
         if combines.get(args.collective) is None:
             if args.collective in ("team", "nvls") and combines.get("nccl") is not None:
                 collective_note = ((collective_note or f"{args.collective} combine unavailable")

@@ -349,6 +349,12 @@ int reduce_multi_team(int dtype, int op, const void* in_local, size_t n_local, v
  *   reduce_nvls_destroy: after every rank's last call completed (collective:
  *     window deregistration). */
 int reduce_nvls_create(void** nvls_out, void* comm, int mode);
+/* The local preconditions of reduce_nvls_create, no collective entered: NCCL
+ * with symmetric memory loadable, at least two ranks in `comm`, a multicast-
+ * capable device.  Ranks should agree on it (e.g. over their process group)
+ * before any of them calls reduce_nvls_create, so that no rank enters the
+ * collective registration alone. */
+int reduce_nvls_supported(void* comm);
 /* A one-member multicast team on the current GPU, built with the CUDA driver's
  * multicast API instead of NCCL (no second GPU needed): the same kernels and
  * protocol at k = 1 -- multimem.st / multimem.red / multimem.ld_reduce through

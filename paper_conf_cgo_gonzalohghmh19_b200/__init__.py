@@ -38,7 +38,8 @@ ABI_SYMBOLS = (
     "reduce_shutdown", "reduce_segmented", "reduce_batched", "reduce_histogram",
     "reduce_team_create", "reduce_team_ipc_handle_bytes", "reduce_team_buffer", "reduce_team_connect",
     "reduce_team_connect_local", "reduce_team_destroy", "reduce_multi_team",
-    "reduce_nvls_create", "reduce_nvls_create_local", "reduce_nvls_destroy", "reduce_multi_nvls",
+    "reduce_nvls_create", "reduce_nvls_create_local", "reduce_nvls_supported", "reduce_nvls_destroy",
+    "reduce_multi_nvls",
 )
 
 
@@ -105,6 +106,7 @@ def _load() -> ctypes.CDLL:
         "reduce_multi_team": (i, [i, i, vp, sz, vp, vp, vp, opts_p]),
         "reduce_nvls_create": (i, [ctypes.POINTER(vp), vp, i]),
         "reduce_nvls_create_local": (i, [ctypes.POINTER(vp), i]),
+        "reduce_nvls_supported": (i, [vp]),
         "reduce_nvls_destroy": (i, [vp]),
         "reduce_multi_nvls": (i, [i, i, vp, sz, vp, vp, vp, opts_p]),
     }
@@ -496,15 +498,23 @@ class Nvls:
             self.handle, self.rank, self.world, self.mode = _local, 0, 1, mode
             return
         import torch.distributed as dist
-        h = ctypes.c_void_p()
-        st = lib.reduce_nvls_create(ctypes.byref(h), ctypes.c_void_p(comm.handle), int(mode))
-        err = last_error() if st != OK else ""
         world = comm.world
-        sts = [None] * world
-        if dist.is_initialized():
-            dist.all_gather_object(sts, (st, err), group=group)
-        else:
-            sts = [(st, err)]
+
+        def agree(st, err):
+            sts = [None] * world
+            if dist.is_initialized():
+                dist.all_gather_object(sts, (st, err), group=group)
+            else:
+                sts = [(st, err)]
+            return sts
+        # the local preconditions first, agreed by every rank: nobody enters the
+        # collective registration alone
+        st = lib.reduce_nvls_supported(ctypes.c_void_p(comm.handle))
+        sts = agree(st, last_error() if st != OK else "")
+        h = ctypes.c_void_p()
+        if all(s == OK for s, _ in sts):
+            st = lib.reduce_nvls_create(ctypes.byref(h), ctypes.c_void_p(comm.handle), int(mode))
+            sts = agree(st, last_error() if st != OK else "")
         if any(s != OK for s, _ in sts):
             if st == OK and h.value:
                 lib.reduce_nvls_destroy(h)

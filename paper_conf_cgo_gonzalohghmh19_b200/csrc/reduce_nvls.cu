@@ -206,11 +206,30 @@ static int finish_setup(Nvls* v) {
 
 extern "C" {
 
+int reduce_nvls_supported(void* comm) {
+  if (!comm) return fail(REDUCE_ERR_INVALID_ARG, "comm is NULL");
+  if (!load_api()) return REDUCE_ERR_UNSUPPORTED;
+  int k = 0;
+  ncclResult_t r = g_api.CommCount((ncclComm_t)comm, &k);
+  if (r != ncclSuccess) return nccl_err(r, "ncclCommCount", REDUCE_ERR_NCCL);
+  if (k < 2) return fail(REDUCE_ERR_UNSUPPORTED, "NVLS needs at least two ranks");
+  if (k > kTeamMaxRanks) return fail(REDUCE_ERR_UNSUPPORTED, "more ranks than the exchange slots hold (256)");
+  if (!load_drv()) return REDUCE_ERR_UNSUPPORTED;
+  int dev = 0, mc = 0;
+  cudaGetDevice(&dev);
+  if (g_drv.DeviceGetAttribute(&mc, CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED, (CUdevice)dev) != CUDA_SUCCESS || !mc)
+    return fail(REDUCE_ERR_UNSUPPORTED, "this device has no multicast support");
+  return REDUCE_OK;
+}
+
 int reduce_nvls_create(void** nvls_out, void* comm, int mode) {
   if (!nvls_out || !comm) return fail(REDUCE_ERR_INVALID_ARG, "nvls_out / comm is NULL");
   if (mode != 1 && mode != 2) return fail(REDUCE_ERR_INVALID_ARG, "mode must be 1 (multimem.ld_reduce) or 2 (multicast store)");
   *nvls_out = nullptr;
-  if (!load_api()) return REDUCE_ERR_UNSUPPORTED;
+  {
+    const int st = reduce_nvls_supported(comm);  // local checks: no collective is entered without them
+    if (st != REDUCE_OK) return st;
+  }
   Nvls* v = new Nvls();
   v->comm = (ncclComm_t)comm;
   v->mode = mode;

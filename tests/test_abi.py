@@ -187,5 +187,6 @@ def test_nvls_entry_points_reject_bad_arguments_without_cuda():
     assert rb.lib.reduce_nvls_create(ctypes.byref(h), None, 1) == 1      # no communicator
     assert rb.lib.reduce_nvls_create(None, ctypes.c_void_p(8), 1) == 1   # no output
     assert rb.lib.reduce_nvls_destroy(None) == 1
+    assert rb.lib.reduce_nvls_supported(None) == 1
     assert rb.lib.reduce_multi_nvls(1, 0, None, 0, None, None, None, None) == 1  # out NULL
     assert "mode" in rb.last_error() or "NULL" in rb.last_error()
