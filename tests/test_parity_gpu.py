@@ -448,3 +448,39 @@ def test_per_thread_default_streams_get_their_own_workspace():
     assert not errors, errors
     for k in range(2):
         assert (outs[k].cpu().numpy() == (k + 1) * n).all(), k
+
+
+def test_prepare_covers_the_widest_partials_grid():
+    """reduce_prepare(stream, n) must size the partials for any plan of up to n
+    elements: fp64 accurate sums carry 16-byte
+    double-double partials, and fp64's smallest tile is 32 threads x 1 vector =
+    128 elements, so a forced TWO_PASS / LAST_BLOCK grid of 32-thread blocks is
+    the largest partials array.  Captured after prepare: no NOT_PREPARED."""
+    import torch
+    rb = _rb()
+    n = 65536 * 128  # exactly kMaxPartialBlocks tiles of 128 fp64 elements
+    x = synth.make("float64", n, "uniform_pm1", 12)
+    t = to_device(x)
+    s = torch.cuda.Stream()
+    rb.prepare(s, n)
+    outs = torch.empty(4, dtype=torch.float64, device="cuda")
+    g = torch.cuda.CUDAGraph()
+    variants = [dict(op="sum_accurate", grid_combine=2, block=32, unroll=1),
+                dict(op="sum_accurate", grid_combine=3, block=32, unroll=1),
+                dict(op="sum", grid_combine=2, block=32, unroll=1),
+                dict(op="max", grid_combine=3, block=32, unroll=1, mode="deterministic")]
+    with torch.cuda.graph(g, stream=s):
+        for i, v in enumerate(variants):
+            kw = {k: val for k, val in v.items() if k != "op"}
+            rb.reduce(t, v["op"], out=outs[i:i + 1], stream=s, **kw)
+    g.replay()
+    torch.cuda.synchronize()
+    for i, v in enumerate(variants):
+        kw = {k: val for k, val in v.items() if k != "op"}
+        p = rb.query_plan("float64", v["op"], n, in_ptr=t.data_ptr(), **kw)
+        assert p["grid"] == 65536, p
+        if v["op"] == "max":
+            check(x, "max", outs[i:i + 1].cpu().numpy(), p)
+        else:
+            ref = oracle.reduce(x, "sum")
+            assert abs(float(outs[i]) - ref.value) <= 2.0 ** -40 * ref.abs_sum, (v, float(outs[i]), ref.value)
