@@ -224,9 +224,26 @@ def reduce_ptr(dtype: int, op, in_ptr: int, n: int, out_ptr: int, stream: int = 
         raise ReduceError(st, "reduce_ex")
 
 
+_OPTS_CACHE: dict = {}
+
+
+def _opts_for(opt_kw):
+    """reduce_opts_t for keyword options, cached (the C side copies it per call)."""
+    if not opt_kw:
+        return None
+    key = tuple(sorted(opt_kw.items()))
+    o = _OPTS_CACHE.get(key)
+    if o is None:
+        o = make_opts(**opt_kw)
+        if len(_OPTS_CACHE) < 4096:
+            _OPTS_CACHE[key] = o
+    return o
+
+
 def reduce(x, op="sum", out=None, stream=None, **opt_kw):
     """Reduce a contiguous CUDA tensor to a 1-element device tensor (async)."""
-    if not x.is_cuda:
+    dev = x.get_device()  # -1 for host tensors
+    if dev < 0:
         raise ValueError("reduce() takes a CUDA tensor; use reduce_host() for host data")
     if not x.is_contiguous():
         raise ValueError("input must be contiguous")
@@ -234,12 +251,16 @@ def reduce(x, op="sum", out=None, stream=None, **opt_kw):
     if out is None:
         import torch
         out = torch.empty(1, dtype=x.dtype, device=x.device)
-    else:
-        _check_out(out, x, 1)
-    opts = make_opts(**opt_kw) if opt_kw else None
+    elif out.dtype is not x.dtype or out.get_device() != dev or not out.is_contiguous() or out.numel() < 1:
+        _check_out(out, x, 1)  # raises with the reason
+    opts = _opts_for(opt_kw)
     s = stream.cuda_stream if stream is not None and not isinstance(stream, int) else _stream_handle(stream, x.device)
-    with _on_device(x.device):
+    import torch
+    if torch.cuda.current_device() == dev:
         reduce_ptr(dt, op, x.data_ptr(), x.numel(), out.data_ptr(), s, opts)
+    else:
+        with torch.cuda.device(dev):
+            reduce_ptr(dt, op, x.data_ptr(), x.numel(), out.data_ptr(), s, opts)
     return out
 
 

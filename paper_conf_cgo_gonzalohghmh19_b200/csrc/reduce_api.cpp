@@ -131,22 +131,29 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
     return fail(REDUCE_ERR_INVALID_ARG, "fp64 accurate sums have no shared-atomic block combine");
 
   // ---- S0: table lookup by ceil(log2(bytes)); an op without tuned rows (the
-  // accurate sum, if the table predates it) falls back to the sum rows
+  // accurate sum, if the table predates it) falls back to the sum rows.  The
+  // first-match scan runs once per (dtype, op, mode, log2 bytes); its result
+  // is cached (a pointer store: benign if two threads fill the same entry).
   const unsigned long long bytes = (unsigned long long)n * (unsigned long long)s;
   const int lb = ilog2_ceil(bytes ? bytes : 1);
-  const DispatchEntry* e = nullptr;
-  for (int pass = 0; pass < 2 && (e == nullptr || e->dtype < 0); ++pass) {
-    const int op_row = pass == 0 ? op : REDUCE_SUM;
-    if (pass == 1 && op != REDUCE_SUM_ACCURATE) break;
-    for (const DispatchEntry& r : kDispatch) {
-      if ((r.dtype < 0 || r.dtype == dtype) && (r.op < 0 || r.op == op_row) && (r.mode < 0 || r.mode == mode) &&
-          lb <= r.max_log2_bytes) {
-        if (e == nullptr || r.dtype >= 0) e = &r;
-        break;
+  static std::atomic<const DispatchEntry*> cache[3][4][2][64];
+  std::atomic<const DispatchEntry*>& slot = cache[dtype][op][mode][lb & 63];
+  const DispatchEntry* e = slot.load(std::memory_order_relaxed);
+  if (e == nullptr) {
+    for (int pass = 0; pass < 2 && (e == nullptr || e->dtype < 0); ++pass) {
+      const int op_row = pass == 0 ? op : REDUCE_SUM;
+      if (pass == 1 && op != REDUCE_SUM_ACCURATE) break;
+      for (const DispatchEntry& r : kDispatch) {
+        if ((r.dtype < 0 || r.dtype == dtype) && (r.op < 0 || r.op == op_row) && (r.mode < 0 || r.mode == mode) &&
+            lb <= r.max_log2_bytes) {
+          if (e == nullptr || r.dtype >= 0) e = &r;
+          break;
+        }
       }
     }
+    if (!e) e = &kDispatch[sizeof(kDispatch) / sizeof(kDispatch[0]) - 1];
+    slot.store(e, std::memory_order_relaxed);
   }
-  if (!e) e = &kDispatch[sizeof(kDispatch) / sizeof(kDispatch[0]) - 1];
 
   int stage = o.stage ? o.stage : (e->stage == REDUCE_STAGE_SMEM ? REDUCE_STAGE_SMEM : REDUCE_STAGE_REG);
   int block = o.block ? o.block : e->block;

@@ -630,7 +630,11 @@ inline cudaError_t launch_kernel(void (*kern)(const KParams), const LaunchDesc& 
   q.pf_stride = 0;
   q.pf_tiles = 0;
   q.trig_window = kPdlBlocksPerSm * (unsigned)num_sms_cached();
-  if (p.early != 0 && d.tiles > 0) {
+  if (p.early != 0 && d.tiles > 0 && prefetch_budget_bytes() == 0) {
+    // the default: every block prefetches (or loads) its own first tile only
+    q.pf_stride = d.grid;
+    q.pf_tiles = 1;
+  } else if (p.early != 0 && d.tiles > 0) {
     // blocks resident at once (one wave): they issue the prefetches, striding
     // over the tiles, up to prefetch_budget_bytes() (L2 is 126 MB; the previous
     // grid's and this grid's streams share it)
