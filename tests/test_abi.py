@@ -190,3 +190,28 @@ def test_nvls_entry_points_reject_bad_arguments_without_cuda():
     assert rb.lib.reduce_nvls_supported(None) == 1
     assert rb.lib.reduce_multi_nvls(1, 0, None, 0, None, None, None, None) == 1  # out NULL
     assert "mode" in rb.last_error() or "NULL" in rb.last_error()
+
+
+def test_binding_rejects_host_tensors_and_bad_outputs_without_cuda():
+    """The Python binding validates before any CUDA call: host
+    inputs are refused, and caller-supplied outputs are checked (dtype, size,
+    device) so the C side never writes past a wrong buffer."""
+    import torch
+    with pytest.raises(ValueError):
+        rb.reduce(torch.ones(4), "sum")
+    with pytest.raises(ValueError):
+        rb.reduce_segmented(torch.ones(4), torch.zeros(2, dtype=torch.int64), "sum")
+    with pytest.raises(ValueError):
+        rb.reduce_batched(torch.ones(2, 2), "sum")
+    with pytest.raises(ValueError):
+        rb.histogram(torch.ones(4), 0.0, 1.0, 4)
+    # the output check itself (device-independent parts)
+    x = torch.ones(4)
+    with pytest.raises(ValueError, match="dtype"):
+        rb._check_out(torch.ones(1, dtype=torch.float64), x, 1)
+    with pytest.raises(ValueError):
+        rb._check_out(torch.ones(1), x, 1)        # not a CUDA tensor
+    assert rb._opts_for({}) is None
+    o1 = rb._opts_for({"mode": "deterministic", "grid": 8})
+    assert rb._opts_for({"grid": 8, "mode": "deterministic"}) is o1 and o1.mode == 1 and o1.grid == 8
+    assert rb.make_opts(input_ready=True).flags == rb.FLAG_INPUT_READY
