@@ -107,13 +107,20 @@ typedef enum {
  *                shared memory through distributed shared memory (DSMEM) and a
  *                cluster barrier -- no atomics, deterministic, one launch; the
  *                sm_90+/sm_100 form of the paper's two-stage per-SM partition
- *                 for medium arrays */
+ *                 for medium arrays
+ *   FLAGS      : every block but the last stores its partial with the call's
+ *                epoch beside each 4-byte word (flag-in-data records); the
+ *                last block polls them, reduces them in a fixed order and
+ *                publishes -- no atomics, no fences, deterministic, one launch
+ *                (a B200 design beside the paper's: one L2 round trip after the
+ *                loads instead of ATOMIC's three; grid <= 8192 blocks) */
 typedef enum {
   REDUCE_GC_DIRECT = 0,
   REDUCE_GC_ATOMIC = 1,
   REDUCE_GC_TWO_PASS = 2,
   REDUCE_GC_LAST_BLOCK = 3,
-  REDUCE_GC_CLUSTER = 4
+  REDUCE_GC_CLUSTER = 4,
+  REDUCE_GC_FLAGS = 5
 } reduce_grid_combine_t;
 
 /* Options for reduce_ex & co.  Zero-initialise, then set fields; every field

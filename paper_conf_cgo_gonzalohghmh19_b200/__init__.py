@@ -20,7 +20,7 @@ INT32, FLOAT32, FLOAT64 = 0, 1, 2
 SUM, MIN, MAX, SUM_ACCURATE = 0, 1, 2, 3
 MODE_FAST, MODE_DETERMINISTIC = 0, 1
 BC_SHFL, BC_SMEM_ATOMIC_WARP, BC_SMEM_ATOMIC_ALL, BC_SMEM_TREE = 0, 1, 2, 3
-GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER = 0, 1, 2, 3, 4
+GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER, GC_FLAGS = 0, 1, 2, 3, 4, 5
 STAGE_REG, STAGE_SMEM = 1, 2
 FLAG_INPUT_READY = 1
 OK = 0

@@ -5,6 +5,7 @@
 #include <atomic>
 #include <climits>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <mutex>
@@ -109,7 +110,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   int mode = o.mode < 0 ? g_mode.load() : o.mode;
   if (mode != REDUCE_MODE_FAST && mode != REDUCE_MODE_DETERMINISTIC)
     return fail(REDUCE_ERR_INVALID_ARG, "mode must be -1, REDUCE_MODE_FAST or REDUCE_MODE_DETERMINISTIC");
-  if (o.grid_combine < -1 || o.grid_combine > 4) return fail(REDUCE_ERR_INVALID_ARG, "bad grid_combine");
+  if (o.grid_combine < -1 || o.grid_combine > 5) return fail(REDUCE_ERR_INVALID_ARG, "bad grid_combine");
   if (o.block_combine < -1 || o.block_combine > 3) return fail(REDUCE_ERR_INVALID_ARG, "bad block_combine");
   if (o.unroll != 0 && o.unroll != 1 && o.unroll != 2 && o.unroll != 4 && o.unroll != 8 && o.unroll != 16)
     return fail(REDUCE_ERR_INVALID_ARG, "unroll must be 0, 1, 2, 4, 8 or 16");
@@ -215,6 +216,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
     grid = tiles > 0 ? tiles : 1;
     if (grid_cap > 0 && grid_cap < grid) grid = grid_cap;
     if ((gc == REDUCE_GC_TWO_PASS || gc == REDUCE_GC_LAST_BLOCK) && grid > kMaxPartialBlocks) grid = kMaxPartialBlocks;
+    if (gc == REDUCE_GC_FLAGS && grid > kMaxFlagBlocks) grid = kMaxFlagBlocks;
     if (grid > 0x7FFFFFFFll) grid = 0x7FFFFFFFll;
   }
   int nslots = 0;  // ATOMIC: a power of two <= min(grid, 32) (the kernel masks, no modulo)
@@ -246,6 +248,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
         case REDUCE_GC_ATOMIC: chain += (grid + nslots - 1) / nslots + 5; break;
         case REDUCE_GC_TWO_PASS: chain += (grid + 255) / 256 + 2 + 10; break;
         case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + 2 + 10; break;
+        case REDUCE_GC_FLAGS: chain += (grid + block - 1) / block + 10; break;  // per-thread run, 2 warp trees
         case REDUCE_GC_CLUSTER: chain += 5; break;
         default: break;
       }
@@ -258,6 +261,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
         case REDUCE_GC_ATOMIC: chain += (grid + nslots - 1) / nslots + 5; break;
         case REDUCE_GC_TWO_PASS: chain += (grid + 255) / 256 + 2 + 10; break;
         case REDUCE_GC_LAST_BLOCK: chain += (grid + block - 1) / block + 2 + 10; break;
+        case REDUCE_GC_FLAGS: chain += (grid + block - 1) / block + 10; break;  // per-thread run, 2 warp trees
         case REDUCE_GC_CLUSTER: chain += 5; break;
         default: break;
       }
@@ -290,6 +294,7 @@ static void free_workspace(Workspace* w) {
   cudaSetDevice(w->device);
   if (w->base) cudaFree(w->base);
   if (w->partials) cudaFree(w->partials);
+  if (w->flagrec) cudaFree(w->flagrec);
   if (w->segq) cudaFree(w->segq);
   if (w->segbal) cudaFree(w->segbal);
   if (w->staging) cudaFree(w->staging);
@@ -302,7 +307,17 @@ static void free_workspace(Workspace* w) {
   delete w;
 }
 
-int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
+// REDUCE_FLAGS_EPOCH0 (tests only): the epoch a new record area starts from,
+// so a test can cross the 32-bit wrap in a few calls
+static unsigned flags_epoch0() {
+  static const unsigned v = [] {
+    const char* e = std::getenv("REDUCE_FLAGS_EPOCH0");
+    return e ? (unsigned)std::strtoul(e, nullptr, 0) : 0u;
+  }();
+  return v;
+}
+
+int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out, size_t records_bytes) {
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
@@ -311,7 +326,8 @@ int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
   Workspace*& w = g_ws[key];
   const bool need_base = (w == nullptr);
   const bool need_partials = (w == nullptr || w->partials_bytes < partials_bytes);
-  if (need_base || need_partials) {
+  const bool need_records = records_bytes > 0 && (w == nullptr || w->flagrec_bytes < records_bytes);
+  if (need_base || need_partials || need_records) {
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     if (cudaStreamIsCapturing(stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
       if (need_base) g_ws.erase(key);
@@ -354,6 +370,27 @@ int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** out) {
     if (w->partials) cudaFreeAsync(w->partials, stream);
     w->partials = p;
     w->partials_bytes = want;
+  }
+  if (need_records) {
+    size_t want = records_bytes < (64u << 10) ? (64u << 10) : records_bytes;
+    char* p = nullptr;
+    e = cudaMallocAsync((void**)&p, kFlagHdrBytes + want, stream);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(REDUCE_ERR_NO_MEMORY, "cudaMallocAsync(flag records) failed");
+    }
+    // zero records never match an epoch (epochs are >= 1); the header holds
+    // the epoch and the record-area size (for the wrap, see flags_combine)
+    e = cudaMemsetAsync(p, 0, kFlagHdrBytes + want, stream);
+    struct { unsigned epoch, pad; unsigned long long bytes; } hdr = {flags_epoch0(), 0u, (unsigned long long)want};
+    if (e == cudaSuccess) e = cudaMemcpyAsync(p, &hdr, sizeof(hdr), cudaMemcpyHostToDevice, stream);
+    if (e != cudaSuccess) {
+      cudaFreeAsync(p, stream);
+      return cuda_fail(e, "flag records init");
+    }
+    if (w->flagrec) cudaFreeAsync(w->flagrec, stream);
+    w->flagrec = p;
+    w->flagrec_bytes = want;
   }
   *out = w;
   return REDUCE_OK;
@@ -422,6 +459,10 @@ int launch_plan(Plan* P, Workspace* ws, void* out, cudaStream_t stream, bool all
   d.slots = ws->slots + combo * kSlotRegionBytes;
   d.ticket = (unsigned*)(ws->tickets + combo * (size_t)kSlotBytes);
   d.partials = ws->partials;
+  if (d.gc == REDUCE_GC_FLAGS) {  // the epoch word and the records
+    d.ticket = (unsigned*)ws->flagrec;
+    d.partials = ws->flagrec + kFlagHdrBytes;
+  }
   d.early = 0;
   // Before the programmatic dependency resolves a kernel may touch its input:
   //  1 = register loads of the first tile, only on the caller's explicit
@@ -467,6 +508,17 @@ static size_t partials_needed(const Plan& P) {
   return 0;
 }
 
+// GC_FLAGS: one record of 16-byte {word, epoch, word, epoch} stores per two
+// words of the Grid value, per block
+static size_t record_bytes(int dtype, int op) { return (size_t)((grid_value_bytes(dtype, op) + 7) / 8) * 16; }
+static size_t records_needed(const Plan& P) {
+  return P.d.gc == REDUCE_GC_FLAGS ? (size_t)P.d.grid * record_bytes(P.dtype, P.op) : 0;
+}
+
+int get_workspace_for(cudaStream_t stream, const Plan& P, Workspace** ws) {
+  return get_workspace(stream, partials_needed(P), ws, records_needed(P));
+}
+
 }  // namespace rb
 
 using namespace rb;
@@ -482,7 +534,7 @@ int reduce_ex(int dtype, int op, const void* in, size_t n, void* out, reduce_str
   int st = make_plan(dtype, op, in, n, opts, 0, &P);
   if (st != REDUCE_OK) return st;
   Workspace* ws = nullptr;
-  st = get_workspace((cudaStream_t)stream, partials_needed(P), &ws);
+  st = get_workspace_for((cudaStream_t)stream, P, &ws);
   if (st != REDUCE_OK) return st;
   return launch_plan(&P, ws, out, (cudaStream_t)stream, /*allow_early=*/true);
 }
@@ -709,7 +761,8 @@ int reduce_prepare(reduce_stream_t stream, size_t max_n) {
   long long g = (long long)(tiles_min_tile < (unsigned long long)kMaxPartialBlocks ? tiles_min_tile : kMaxPartialBlocks);
   if (g < 1024) g = 1024;
   Workspace* ws = nullptr;
-  int st = get_workspace((cudaStream_t)stream, (size_t)g * 16, &ws);
+  const long long gf = g < kMaxFlagBlocks ? g : kMaxFlagBlocks;
+  int st = get_workspace((cudaStream_t)stream, (size_t)g * 16, &ws, (size_t)gf * 32);
   if (st != REDUCE_OK) return st;
   char* q = nullptr;
   st = get_seg_queue((cudaStream_t)stream, &q);  // so segmented calls can be captured too

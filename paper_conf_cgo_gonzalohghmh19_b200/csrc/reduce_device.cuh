@@ -22,7 +22,7 @@ namespace rb {
 constexpr int DT_I32 = 0, DT_F32 = 1, DT_F64 = 2;
 constexpr int OP_SUM = 0, OP_MIN = 1, OP_MAX = 2, OP_SUMACC = 3;
 constexpr int BC_SHFL = 0, BC_ATOMIC_WARP = 1, BC_ATOMIC_ALL = 2, BC_TREE = 3;
-constexpr int GC_DIRECT = 0, GC_ATOMIC = 1, GC_TWO_PASS = 2, GC_LAST_BLOCK = 3, GC_CLUSTER = 4;
+constexpr int GC_DIRECT = 0, GC_ATOMIC = 1, GC_TWO_PASS = 2, GC_LAST_BLOCK = 3, GC_CLUSTER = 4, GC_FLAGS = 5;
 constexpr int kVecBytes = 32;    // one 256-bit load per thread per vector
 
 // ------------------------------------------------------------------ loads ---
@@ -90,6 +90,27 @@ __device__ __forceinline__ unsigned ticket_acq_rel(unsigned* t) {
   unsigned old;
   asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(old) : "l"(t) : "memory");
   return old;
+}
+
+// Relaxed GPU-scope accesses of the flag-in-data partial records (GC_FLAGS):
+// served by L2, never by a stale L1 line.
+__device__ __forceinline__ unsigned ld_relaxed_u32(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed_u32(unsigned* p, unsigned v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_pairs_gpu(void* p, unsigned a, unsigned b, unsigned e) {
+  asm volatile("st.relaxed.gpu.global.v4.u32 [%0], {%1, %2, %3, %4};" :: "l"(p), "r"(a), "r"(e), "r"(b), "r"(e)
+               : "memory");
+}
+__device__ __forceinline__ uint4 ld_pairs_gpu(const void* p) {
+  uint4 v;
+  asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p) : "memory");
+  return v;
 }
 
 // Split cluster barrier (all threads of every CTA of the cluster take part).

@@ -43,10 +43,8 @@ extern "C" int reduce_host(int dtype, int op, const void* host_in, size_t n, voi
   Plan P;
   int st = make_plan(dtype, op, (const void*)(uintptr_t)256, n < chunk_elems ? n : chunk_elems, opts, 1, &P);
   if (st != REDUCE_OK) return st;
-  size_t pbytes = (P.d.gc == REDUCE_GC_TWO_PASS || P.d.gc == REDUCE_GC_LAST_BLOCK)
-                      ? (size_t)P.d.grid * (size_t)gbytes : 0;
   Workspace* ws = nullptr;
-  if ((st = get_workspace(cs, pbytes, &ws)) != REDUCE_OK) return st;
+  if ((st = get_workspace_for(cs, P, &ws)) != REDUCE_OK) return st;
 
   // staging: 2 x chunk_bytes, then the per-chunk raw values
   const size_t vals_bytes = (size_t)kMaxChunks * 16;  // up to 16-byte raw values (double-double)
@@ -88,6 +86,8 @@ extern "C" int reduce_host(int dtype, int op, const void* host_in, size_t n, voi
     if ((e = cudaStreamWaitEvent(cs, ws->ev_copied[b], 0)) != cudaSuccess) return cuda_fail(e, "wait");
     Plan C;
     if ((st = make_plan(dtype, op, buf, cnt, opts, 1, &C)) != REDUCE_OK) return st;
+    // the ragged last chunk may plan another grid combine than a full one
+    if ((st = get_workspace_for(cs, C, &ws)) != REDUCE_OK) return st;
     if ((st = launch_plan(&C, ws, vals + (size_t)c * gbytes, cs)) != REDUCE_OK) return st;
     if ((e = cudaEventRecord(ws->ev_done[b], cs)) != cudaSuccess) return cuda_fail(e, "record");
   }

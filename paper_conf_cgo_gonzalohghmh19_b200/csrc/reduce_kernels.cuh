@@ -278,10 +278,126 @@ __device__ __forceinline__ void store_out(typename T::Grid g, const KParams& p) 
   else T::finalize(g, p.out);
 }
 
+// GC_FLAGS: flag-in-data partial records polled by one fixed block -- no
+// atomic, no fence, no ticket.  Every block but the last stores its partial as
+// {word, epoch} pairs (one 16-byte relaxed store per two words: each aligned
+// 8-byte pair is written and read as one access, so a matching epoch implies
+// the word beside it -- the protocol of team_exchange, inside one GPU).  Block
+// G-1 (dispatched last, so it rarely waits) polls records 0..G-2 with loads in
+// flight, combines them in index order with its own value last and a fixed
+// tree (deterministic for a fixed launch shape), writes the result and
+// publishes the next epoch.  The epoch word (p.ticket) is read by every block
+// after the dependency resolves and advanced only by the poller, after every
+// record of the call was consumed; a record from an older call carries an
+// older epoch.  When the 32-bit epoch would wrap, the poller zeroes the whole
+// record area (its size in bytes is the 64-bit word at p.ticket + 2) first.
+// Replaces the ATOMIC chain red -> release -> ticket -> exchange (three L2
+// round trips after the loads) by one store and one poll (B200 probe,
+// tools/probes/probe_mid.cu "flags_fixed": -1.0 to -2.1 us per call at 1-64 MB).
+// (Scalars by value, as the exchanges below: a reference to the kernel's
+// parameter struct in a non-inlined function would copy it to the stack.)
 template <class T>
-__device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& p) {
+__device__ __noinline__ void flags_combine(typename T::Grid g, unsigned ep, char* const rec, unsigned* const ticket,
+                                           void* const out, const int raw_out, const TeamArgs team) {
+  using Grid = typename T::Grid;
+  static_assert(sizeof(Grid) <= 16 && sizeof(Grid) % 4 == 0, "a record holds <= 4 words");
+  constexpr int NW = sizeof(Grid) / 4;
+  constexpr int NV = (NW + 1) / 2;  // 16-byte stores {w, e, w, e} per record
+#ifndef RB_FLAGS_KB
+#define RB_FLAGS_KB 4
+#endif
+#ifndef RB_FLAGS_SLEEP
+#define RB_FLAGS_SLEEP 0
+#endif
+  constexpr int KB = NV == 1 ? RB_FLAGS_KB : 2;  // records in flight per thread
+  const unsigned G1 = gridDim.x - 1;
+  if (blockIdx.x != G1) {
+    if (threadIdx.x == 0) {
+      unsigned w[4] = {0u, 0u, 0u, 0u};
+      memcpy(w, &g, sizeof(Grid));
+#pragma unroll
+      for (int v = 0; v < NV; ++v) st_pairs_gpu(rec + ((size_t)blockIdx.x * NV + v) * 16, w[2 * v], w[2 * v + 1], ep);
+    }
+    return;
+  }
+  __shared__ unsigned s_ep;
+  __shared__ Grid s_own;
+  __shared__ Grid gpart[32];
+  if (threadIdx.x == 0) {
+    s_ep = ep;
+    s_own = g;
+  }
+  __syncthreads();
+  const unsigned e = s_ep;
+  const unsigned B = blockDim.x;
+  Grid x = T::gident();
+#pragma unroll 1
+  for (unsigned i0 = threadIdx.x; i0 < G1; i0 += KB * B) {
+    uint4 r[KB][NV];
+#pragma unroll
+    for (int j = 0; j < KB; ++j)
+      if (i0 + j * B < G1)
+#pragma unroll
+        for (int v = 0; v < NV; ++v) r[j][v] = ld_pairs_gpu(rec + ((size_t)(i0 + j * B) * NV + v) * 16);
+#pragma unroll
+    for (int j = 0; j < KB; ++j) {
+      if (i0 + j * B < G1) {
+        unsigned w[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+        for (int v = 0; v < NV; ++v) {
+          if (r[j][v].y != e || r[j][v].w != e) {
+            const long long t0 = clock64();
+            do {
+              if (RB_FLAGS_SLEEP > 0) __nanosleep(RB_FLAGS_SLEEP);
+              // a block that never publishes (a bug, not a race) must not hang the GPU
+              if (clock64() - t0 > (1ll << 35)) __trap();
+              r[j][v] = ld_pairs_gpu(rec + ((size_t)(i0 + j * B) * NV + v) * 16);
+            } while (r[j][v].y != e || r[j][v].w != e);
+          }
+          w[2 * v] = r[j][v].x;
+          w[2 * v + 1] = r[j][v].z;
+        }
+        Grid y;
+        memcpy(&y, w, sizeof(Grid));
+        x = T::gcomb(x, y);
+      }
+    }
+  }
+  if (threadIdx.x == G1 % B) x = T::gcomb(x, s_own);  // index G1 comes last in its thread's sequence
+  x = T::gwarp(x);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (B + 31) >> 5;
+  if (lane == 0) gpart[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    Grid y = lane < nw ? gpart[lane] : T::gident();
+    y = T::gwarp(y);
+    if (lane == 0) {
+      if (team.k > 0) y = RB_CROSS_RANK(T, y, team);
+      if (raw_out) *(Grid*)out = y;
+      else T::finalize(y, out);
+    }
+  }
+  if (e != 0xFFFFFFFFu) {
+    if (threadIdx.x == 0) st_relaxed_u32(ticket, e);
+    return;
+  }
+  // epoch wrap: no record may keep a value that a later epoch could match
+  const unsigned long long cap = *(const unsigned long long*)(ticket + 2);
+#pragma unroll 1
+  for (unsigned long long o = (unsigned long long)threadIdx.x * 16; o + 16 <= cap; o += (unsigned long long)B * 16)
+    *(uint4*)(rec + o) = make_uint4(0u, 0u, 0u, 0u);
+  __syncthreads();
+  if (threadIdx.x == 0) st_relaxed_u32(ticket, 0u);
+}
+
+template <class T>
+__device__ __forceinline__ void grid_combine(typename T::Grid g, const KParams& p, unsigned ep) {
   using Grid = typename T::Grid;
   __shared__ int s_last;
+  if (p.gc == GC_FLAGS) {
+    flags_combine<T>(g, ep, (char*)p.partials, p.ticket, p.out, p.raw_out, p.team);
+    return;
+  }
   if (p.gc == GC_DIRECT) {
     if (threadIdx.x == 0) store_out<T>(g, p);
     return;
@@ -431,6 +547,8 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
   const bool early_trigger = may_trigger && gridDim.x > win && blockIdx.x + win >= gridDim.x;
   if (early_trigger) pdl_trigger();
   if (p.gc == GC_CLUSTER) cluster_arrive_relaxed();  // phase 1: "this CTA has started"
+  // GC_FLAGS: this call's epoch, read now so the load's latency hides behind the tiles
+  const unsigned ep = (p.gc == GC_FLAGS && threadIdx.x == 0) ? ld_relaxed_u32(p.ticket) + 1u : 0u;
   Part<T> a[T::NA];
   init_parts<T>(a);
   uint32_t aux = 0;
@@ -505,7 +623,7 @@ __global__ void __launch_bounds__(max_block_threads(DT, OP, U, STAGE),
   }
   const Acc v = thread_result<T>(a, aux);
   const typename T::Grid g = block_combine<T, BC>(v);
-  grid_combine<T>(g, p);
+  grid_combine<T>(g, p, ep);
 }
 
 // Second pass of GC_TWO_PASS and the cross-chunk / cross-rank combine.

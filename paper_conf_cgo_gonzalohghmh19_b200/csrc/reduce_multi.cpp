@@ -141,10 +141,8 @@ int reduce_multi_ex(int dtype, int op, const void* in_local, size_t n_local, voi
   int st = make_plan(dtype, op, in_local, n_local, opts, direct ? 0 : 1, &P);
   if (st != REDUCE_OK) return st;
   if (!load_nccl()) return REDUCE_ERR_UNSUPPORTED;
-  const size_t pbytes = (P.d.gc == REDUCE_GC_TWO_PASS || P.d.gc == REDUCE_GC_LAST_BLOCK)
-                            ? (size_t)P.d.grid * (size_t)grid_value_bytes(dtype, op) : 0;
   Workspace* ws = nullptr;
-  st = get_workspace((cudaStream_t)stream, pbytes, &ws);
+  st = get_workspace_for((cudaStream_t)stream, P, &ws);
   if (st != REDUCE_OK) return st;
   cudaStream_t cs = (cudaStream_t)stream;
   ncclComm_t c = (ncclComm_t)comm;

@@ -393,10 +393,8 @@ int reduce_multi_nvls(int dtype, int op, const void* in_local, size_t n_local, v
   Plan P;
   int st = make_plan(dtype, op, in_local, n_local, opts, 0, &P);
   if (st != REDUCE_OK) return st;
-  const size_t pbytes = (P.d.gc == REDUCE_GC_TWO_PASS || P.d.gc == REDUCE_GC_LAST_BLOCK)
-                            ? (size_t)P.d.grid * (size_t)grid_value_bytes(dtype, op) : 0;
   Workspace* ws = nullptr;
-  if ((st = get_workspace((cudaStream_t)stream, pbytes, &ws)) != REDUCE_OK) return st;
+  if ((st = get_workspace_for((cudaStream_t)stream, P, &ws)) != REDUCE_OK) return st;
   P.d.team.bufs = v->d_peers;
   P.d.team.k = v->k;
   P.d.team.rank = v->rank;

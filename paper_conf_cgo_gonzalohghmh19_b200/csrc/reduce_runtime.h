@@ -23,6 +23,11 @@ struct Workspace {
   char* scalars = nullptr;     // 64 x 64-byte scratch scalars (raw results, gathers)
   char* partials = nullptr;    // per-block / per-chunk Grid values
   size_t partials_bytes = 0;
+  // GC_FLAGS: [0, kFlagHdrBytes) header (u32 epoch at 0, u64 record-area bytes
+  // at 8), then the flag-in-data records; never written by anything else, so a
+  // stale record can only carry an older epoch
+  char* flagrec = nullptr;
+  size_t flagrec_bytes = 0;    // record area (excluding the header)
   char* segq = nullptr;        // long-segment queue of reduce_segmented / reduce_batched (kSegQBytes)
   char* segbal = nullptr;      // chunk arrays of the element-balanced reduce_segmented (kBalBytes)
   // device bytes the last library call on this stream wrote for the caller
@@ -40,6 +45,8 @@ struct Workspace {
 constexpr size_t kScalarBytes = 64;
 constexpr int kNumScalars = 64;
 constexpr long long kMaxPartialBlocks = 1 << 16;  // grid cap for partials-based combines
+constexpr long long kMaxFlagBlocks = 1 << 13;     // grid cap for GC_FLAGS (one block polls them all)
+constexpr size_t kFlagHdrBytes = 256;
 
 // Resolved plan of one reduction call (step S0).
 struct Plan {
@@ -61,9 +68,12 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
               Plan* plan);
 
 // Find or create the workspace for (current device, stream) with at least
-// `partials_bytes` of partials.  Returns REDUCE_ERR_NOT_PREPARED when an
-// allocation would be needed during stream capture.
-int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** ws);
+// `partials_bytes` of partials and `records_bytes` of GC_FLAGS records.
+// Returns REDUCE_ERR_NOT_PREPARED when an allocation would be needed during
+// stream capture.
+int get_workspace(cudaStream_t stream, size_t partials_bytes, Workspace** ws, size_t records_bytes = 0);
+// The same, sized for one plan.
+int get_workspace_for(cudaStream_t stream, const Plan& plan, Workspace** ws);
 
 // Fill the workspace pointers of plan->d and launch it.  allow_early: a public
 // single-array call (reduce / reduce_ex), whose written bytes are exactly

@@ -36,7 +36,10 @@ the paper's Fig. 1(b) blocked / strided partition):
     thread (stride Bc), joined (2), butterflied (5), the warps' values
     butterflied again (5).  Bc is at least 256 (TWO_PASS) or `block`
     (LAST_BLOCK); a smaller Bc only lengthens the chain, so Bc = 256 /
-    block is an upper bound.
+    block is an upper bound.  FLAGS: the polling block (`block` threads)
+    folds the grid values into ONE accumulator per thread (stride block):
+    ceil(grid / block) additions, butterflied (5), the warps' values
+    butterflied again (5).
   * fp32 plain sums cross blocks in fp64: everything above the block adds
     < (grid + 64) 2^-53 sum|x|, which is < 2^-29 sum|x| = 1/32 u_f sum|x|
     for grid < 2^23, plus ONE fp32 rounding of the final value -> +1 (the
@@ -48,7 +51,7 @@ from __future__ import annotations
 import math
 
 VE = {"float32": 8, "float64": 4}   # elements per 32-byte vector
-GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER = 0, 1, 2, 3, 4
+GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER, GC_FLAGS = 0, 1, 2, 3, 4, 5
 BC_SHFL, BC_ATOMIC_WARP, BC_ATOMIC_ALL, BC_TREE = 0, 1, 2, 3
 
 
@@ -63,6 +66,8 @@ def _grid_terms(gc: int, grid: int, block: int, slots: int) -> int:
         return 5
     if gc == GC_ATOMIC:
         return _cdiv(grid, max(1, slots)) + 5
+    if gc == GC_FLAGS:
+        return _cdiv(grid, block) + 5 + 5
     bc = 256 if gc == GC_TWO_PASS else block
     return _cdiv(grid, 4 * bc) + 2 + 5 + 5
 

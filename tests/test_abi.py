@@ -63,7 +63,7 @@ def test_invalid_arguments_rejected_without_cuda(args, why):
 
 
 @pytest.mark.parametrize("kw", [
-    dict(mode=7), dict(grid_combine=9), dict(block_combine=5), dict(unroll=3),
+    dict(mode=7), dict(grid_combine=9), dict(grid_combine=6), dict(block_combine=5), dict(unroll=3),
     dict(block=48), dict(block=2048), dict(block=1024, unroll=8), dict(grid=-2), dict(grid=-5),
     dict(mode="deterministic", grid_combine=rb.GC_ATOMIC),
     dict(mode="deterministic", block_combine=rb.BC_SMEM_ATOMIC_ALL),

@@ -44,7 +44,8 @@ def _check(x, r, plan):
 
 VARIANTS = [dict(), dict(mode="deterministic"), dict(grid_combine=0, block=256), dict(grid_combine=2),
             dict(grid_combine=3), dict(grid_combine=4, grid=16), dict(stage="smem", unroll=8, block=256),
-            dict(block_combine=3, block=128), dict(grid=148, grid_combine=3)]
+            dict(block_combine=3, block=128), dict(grid=148, grid_combine=3), dict(grid_combine=5),
+            dict(grid_combine=5, block=32, unroll=1)]
 
 
 @pytest.mark.parametrize("dtype", ["float32", "float64"])

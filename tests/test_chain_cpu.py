@@ -14,7 +14,8 @@ VARIANTS = [dict(), dict(mode="deterministic"), dict(grid_combine=0, block=256),
             dict(stage="smem", unroll=8, block=256), dict(stage="smem", unroll=16, block=256),
             dict(block_combine=3, block=128), dict(block_combine=1), dict(block_combine=2, block=128),
             dict(grid=148, grid_combine=3), dict(grid=148, grid_combine=1, unroll=1),
-            dict(grid=7, grid_combine=2, block=64, unroll=2)]
+            dict(grid=7, grid_combine=2, block=64, unroll=2), dict(grid_combine=5), dict(grid_combine=5, block=32, unroll=1),
+            dict(grid=300, grid_combine=5, block=128)]
 
 
 @pytest.mark.parametrize("dtype,op", [("float32", "sum"), ("float64", "sum"), ("float32", "sum_accurate"),
@@ -71,5 +72,9 @@ def test_hand_counted_chains():
     # accurate fp32, 3 tiles per block of U = 8: 24 lane additions + 1 + 3 (8 accumulators)
     p = _plan(grid=10, block=256, unroll=8, tiles=30, grid_combine=4)
     assert chain_bound("float32", "sum_accurate", p) == 24 + 1 + 3 + 10 + 5
+    # fp64 FLAGS, 2000 blocks of 256: the polling thread folds ceil(2000/256) = 8
+    # records, then two 5-level butterflies
+    p = _plan(grid=2000, block=256, unroll=4, tiles=2000, grid_combine=5)
+    assert chain_bound("float64", "sum", p) == (2 + 2 + 2) + 10 + 8 + 10
     # empty input: only the fixed levels remain
     assert chain_bound("float32", "sum", _plan(tiles=0)) == 0 + 3 + 2 + 10

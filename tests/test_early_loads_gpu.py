@@ -80,7 +80,8 @@ def test_early_triggering_user_kernel_every_variant():
     """The same producer before every grid combine and both stagings."""
     from tests import pdl_producer
     for v in (dict(grid_combine=0, block=1024), dict(grid_combine=1), dict(grid_combine=2), dict(grid_combine=3),
-              dict(grid_combine=4, grid=16), dict(stage="smem", unroll=8, block=256), dict(mode="deterministic")):
+              dict(grid_combine=4, grid=16), dict(stage="smem", unroll=8, block=256), dict(mode="deterministic"),
+              dict(grid_combine=5)):
         got = _run(lambda k, x, s: pdl_producer.produce(x.data_ptr(), N, k + 1, 5000, s.cuda_stream), iters=300, **v)
         want = _want(np.arange(1, 301))
         assert (got == want).all(), (v, np.flatnonzero(got != want)[:10])

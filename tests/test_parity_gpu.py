@@ -112,7 +112,7 @@ def test_size_sweep(dtype):
 # ------------------------------------------------------------- every variant on the same inputs
 VARIANTS = []
 for bc in range(4):
-    for gc in range(5):
+    for gc in range(6):
         for blk, u, st in ((32, 1, 1), (128, 2, 1), (256, 4, 1), (512, 8, 1), (1024, 1, 1),
                            (32, 16, 2), (128, 16, 2), (256, 8, 2), (1024, 4, 2)):
             VARIANTS.append(dict(block_combine=bc, grid_combine=gc, block=blk, unroll=u, stage=st))

@@ -38,7 +38,8 @@ __device__ __forceinline__ void ldv8(const void* p, uint32_t (&r)[8]) {
 // EARLY: 0 none, 1 first tile into registers before the wait, 2 bulk L2
 // prefetch of every tile this CTA will read before the wait.  The grid may be
 // smaller than the tile count (persistent: CTA b reads tiles b, b+G, ...).
-template <int MODE, int EARLY, bool TRIG0>  // MODE 0 store, 1 atomic, 2 relaxed ticket, 3 packed, 4 flags
+template <int MODE, int EARLY, bool TRIG0>  // MODE 0 store, 1 atomic, 2 relaxed ticket, 3 packed, 4 flags,
+                                            // 5 flags polled by the fixed block G-1 (no ticket)
 __global__ void __launch_bounds__(256) k(P p) {
   const long long tiles = p.tiles;
   uint32_t r[4][8];
@@ -103,6 +104,14 @@ __global__ void __launch_bounds__(256) k(P p) {
           *p.out = __uint_as_float((unsigned)(old + add));
           atomicExch((unsigned long long*)p.slots, 0ull);
         }
+      } else if (MODE == 5) {
+        if (blockIdx.x != gridDim.x - 1) {
+          const unsigned long long b = (unsigned long long)__double_as_longlong((double)v);
+          asm volatile("st.relaxed.gpu.global.v4.u32 [%0], {%1, %2, %3, %4};" :: "l"(p.partials + 2 * blockIdx.x),
+                       "r"((unsigned)b), "r"(p.epoch), "r"((unsigned)(b >> 32)), "r"(p.epoch) : "memory");
+        }
+        last = blockIdx.x == gridDim.x - 1;
+        part[0] = v;
       } else {
         // flag-in-data partial {value bits, epoch} then a relaxed ticket
         const unsigned epoch = p.epoch;
@@ -124,6 +133,42 @@ __global__ void __launch_bounds__(256) k(P p) {
       if (threadIdx.x == 0) {
         *p.out = (float)x;
         atomicExch(p.ticket, 0u);
+      }
+    }
+  }
+  if (MODE == 5) {
+    __syncthreads();
+    if (last) {
+      double x = threadIdx.x == 0 ? (double)part[0] : 0.0;
+      const int G1 = (int)gridDim.x - 1;
+      for (int i0 = threadIdx.x; i0 < G1; i0 += 256 * 8) {
+        unsigned a[8], fa[8], b2[8], fb[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          fa[j] = fb[j] = p.epoch; a[j] = b2[j] = 0u;
+          if (i0 + 256 * j < G1)
+            asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(a[j]), "=r"(fa[j]), "=r"(b2[j]), "=r"(fb[j])
+                         : "l"(p.partials + 2 * (i0 + 256 * j)) : "memory");
+        }
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          while (fa[j] != p.epoch || fb[j] != p.epoch) {
+            __nanosleep(20);
+            asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(a[j]), "=r"(fa[j]), "=r"(b2[j]), "=r"(fb[j])
+                         : "l"(p.partials + 2 * (i0 + 256 * j)) : "memory");
+          }
+          x += __longlong_as_double((long long)(((unsigned long long)b2[j] << 32) | a[j]));
+        }
+      }
+      for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+      __shared__ double dp[8];
+      __syncthreads();
+      if ((threadIdx.x & 31) == 0) dp[threadIdx.x >> 5] = x;
+      __syncthreads();
+      if (threadIdx.x < 32) {
+        double y = threadIdx.x < 8 ? dp[threadIdx.x] : 0.0;
+        for (int o = 4; o; o >>= 1) y += __shfl_xor_sync(0xffffffffu, y, o);
+        if (threadIdx.x == 0) *p.out = (float)y;
       }
     }
   }
@@ -182,12 +227,16 @@ int main() {
   cudaStream_t s;
   CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
   struct V { const char* name; KF f; int per_sm; };  // per_sm 0: one tile per CTA
-  V vs[] = {{"store", k<0, 0, false>, 0}, {"atomic", k<1, 0, false>, 0}, {"atomic_relaxed_WRONG", k<2, 0, false>, 0},
+  V vs[] = {{"store_pf", k<0, 2, false>, 0}, {"atomic_pf", k<1, 2, false>, 0}, {"packed_int_pf", k<3, 2, false>, 0},
+            {"flags_fixed_pf", k<5, 2, false>, 0}, {"flags_fixed", k<5, 0, false>, 0}, {"flags_fixed_early", k<5, 1, false>, 0},
+            {"atomic_early", k<1, 1, false>, 0}};
+  V vs_old[] = {{"store", k<0, 0, false>, 0}, {"atomic", k<1, 0, false>, 0}, {"atomic_relaxed_WRONG", k<2, 0, false>, 0},
             {"packed_int", k<3, 0, false>, 0}, {"flags_relaxed", k<4, 0, false>, 0},
             {"store_pf", k<0, 2, false>, 0}, {"atomic_pf", k<1, 2, false>, 0}, {"packed_int_pf", k<3, 2, false>, 0},
             {"flags_pf", k<4, 2, false>, 0}, {"atomic_early", k<1, 1, false>, 0}, {"packed_early", k<3, 1, false>, 0},
             {"flags_early", k<4, 1, false>, 0}};
-  for (int lb = 20; lb <= 26; lb += 2) {
+  for (int lb = 20; lb <= 28; lb += 2) {
+    (void)vs_old;
     const size_t bytes = 1ull << lb;
     const long long tiles = (long long)(bytes / (256 * 4 * 32));
     const int R = 100;

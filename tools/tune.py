@@ -35,7 +35,7 @@ MAXBLK = lambda dt, op, u: 512 if (u >= 8 or (dt == "float64" and op != "sum" an
 
 
 def candidates(dtype, op, mode, lb):
-    gcs = [1, 2, 3] if mode == "fast" else [2, 3]
+    gcs = [1, 2, 3, 5] if mode == "fast" else [2, 3, 5]
     if op == "sum_accurate" and dtype == "float64":
         gcs = [g for g in gcs if g != 1]  # double-double: no value atomics
     out = []
@@ -59,8 +59,8 @@ def candidates(dtype, op, mode, lb):
             if blk * u * 32 <= 128 * 1024:
                 out.append(dict(block=blk, unroll=u, grid_combine=4, block_combine=0, grid=c, stage=2))
     if lb >= 24:
-        for blk, g in itertools.product((256, 512), (148 * 2, 148 * 4, 148 * 8)):
-            out.append(dict(block=blk, unroll=4, grid_combine=gcs[0], block_combine=0, grid=g))
+        for blk, g, gc in itertools.product((256, 512), (148 * 2, 148 * 4, 148 * 8), (gcs[0], 5)):
+            out.append(dict(block=blk, unroll=4, grid_combine=gc, block_combine=0, grid=g))
     for c in out:
         c.setdefault("stage", 1)
     ok = lambda c: (c["block"] <= (512 if op == "sum_accurate" else 1024) if c["stage"] == 2
