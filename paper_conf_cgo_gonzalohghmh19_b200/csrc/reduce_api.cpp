@@ -730,6 +730,7 @@ int reduce_histogram(int dtype, const void* in, size_t n, double lo, double hi, 
   }
   p.nbins = nbins;
   p.counts = counts;
+  p.merge64 = ((uintptr_t)counts % 8u) == 0 && (unsigned long long)n < (1ull << 32);
   note_unknown_output((cudaStream_t)stream);
   cudaError_t e = launch_histogram(dtype, p, 256, (cudaStream_t)stream);
   if (e != cudaSuccess) return cuda_fail(e, "histogram launch");

@@ -196,6 +196,8 @@ struct HistParams {
   float lo_f, hi_f, scale_f;    // fp32 input: (float)lo, (float)hi, (float)(nbins / (hi - lo))
   int nbins;
   unsigned* counts;             // device, nbins
+  int merge64;                  // counts 8-byte aligned and n < 2^32: a bin pair is merged with ONE
+                                //   64-bit global add (no count can carry into its neighbour)
 };
 cudaError_t launch_histogram(int dtype, const HistParams& p, int block, cudaStream_t s);
 

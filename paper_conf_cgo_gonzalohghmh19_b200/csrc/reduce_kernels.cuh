@@ -50,6 +50,11 @@ struct KParams {
   unsigned trig_window;  // blocks of the last ~wave (kPdlBlocksPerSm x SMs), set by launch_kernel
 };
 
+// Polling loops spin without sleeping for this many cycles (~10 us), then
+// back off with nanosleep: a sleep per miss added 0.3-1 us per call to the
+// FLAGS combine (profiles/r02_flags_ab.jsonl); long waits still yield.
+constexpr long long kSpinCycles = 20000;
+
 // ---- one-shot cross-GPU combine through peer memory ------
 // Executed by ONE thread of the block that owns this rank's raw result x.
 // Flag-in-data protocol (as NCCL's "LL"): every 4-byte word of x travels with
@@ -113,7 +118,7 @@ __device__ __noinline__ typename T::Grid team_exchange(typename T::Grid x, char*
       if (fa != epoch || fb != epoch) {
         const long long t0 = clock64();
         do {
-          __nanosleep(32);
+          if (clock64() - t0 > kSpinCycles) __nanosleep(64);  // spin first: a sleep costs ~0.5 us of latency
           // a member that never arrives must not hang the GPU: after ~2^35
           // cycles (> 15 s) abort the kernel -- the error surfaces at the sync
           if (clock64() - t0 > (1ll << 35)) __trap();
@@ -208,7 +213,7 @@ __device__ __noinline__ typename T::Grid nvls_exchange(typename T::Grid x, char*
     if ((int)(got - target) < 0) {
       const long long t0 = clock64();
       do {
-        __nanosleep(32);
+        if (clock64() - t0 > kSpinCycles) __nanosleep(64);  // spin first: a sleep costs ~0.5 us of latency
         if (clock64() - t0 > (1ll << 35)) __trap();  // a member that never arrives: abort, not hang
         asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(got) : "l"(own + kNvlsCtrOff) : "memory");
       } while ((int)(got - target) < 0);
@@ -252,7 +257,7 @@ __device__ __noinline__ typename T::Grid nvls_exchange(typename T::Grid x, char*
       if (fa != epoch || fb != epoch) {
         const long long t0 = clock64();
         do {
-          __nanosleep(32);
+          if (clock64() - t0 > kSpinCycles) __nanosleep(64);  // spin first: a sleep costs ~0.5 us of latency
           if (clock64() - t0 > (1ll << 35)) __trap();
           ld_pairs_sys(src + 4 * v, r[2 * v], fa, r[2 * v + 1], fb);
         } while (fa != epoch || fb != epoch);
@@ -307,7 +312,7 @@ __device__ __noinline__ void flags_combine(typename T::Grid g, unsigned ep, char
 #define RB_FLAGS_KB 4
 #endif
 #ifndef RB_FLAGS_SLEEP
-#define RB_FLAGS_SLEEP 0
+#define RB_FLAGS_SLEEP 64
 #endif
   constexpr int KB = NV == 1 ? RB_FLAGS_KB : 2;  // records in flight per thread
   const unsigned G1 = gridDim.x - 1;
@@ -348,7 +353,7 @@ __device__ __noinline__ void flags_combine(typename T::Grid g, unsigned ep, char
           if (r[j][v].y != e || r[j][v].w != e) {
             const long long t0 = clock64();
             do {
-              if (RB_FLAGS_SLEEP > 0) __nanosleep(RB_FLAGS_SLEEP);
+              if (RB_FLAGS_SLEEP > 0 && clock64() - t0 > kSpinCycles) __nanosleep(RB_FLAGS_SLEEP);
               // a block that never publishes (a bug, not a race) must not hang the GPU
               if (clock64() - t0 > (1ll << 35)) __trap();
               r[j][v] = ld_pairs_gpu(rec + ((size_t)(i0 + j * B) * NV + v) * 16);

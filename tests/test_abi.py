@@ -93,8 +93,10 @@ def test_query_plan_modes():
     fast = rb.query_plan("float32", "sum", n, mode="fast")
     det = rb.query_plan("float32", "sum", n, mode="deterministic")
     assert fast["grid_combine"] == rb.GC_ATOMIC and fast["launches"] == 1
-    assert det["grid_combine"] == rb.GC_TWO_PASS and det["launches"] == 2
-    assert det["grid"] <= 1 << 16
+    # deterministic: a fixed-order combine (the tuner's pick), never value atomics
+    assert det["grid_combine"] in (rb.GC_TWO_PASS, rb.GC_LAST_BLOCK, rb.GC_FLAGS)
+    assert det["launches"] == (2 if det["grid_combine"] == rb.GC_TWO_PASS else 1)
+    assert det["grid"] <= (1 << 13 if det["grid_combine"] == rb.GC_FLAGS else 1 << 16)
     # one block per 32 KiB tile at the headline size
     tile = fast["block"] * fast["unroll"] * 32
     assert fast["tiles"] == (n * 4) // tile and fast["grid"] == fast["tiles"]

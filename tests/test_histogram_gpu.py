@@ -120,3 +120,26 @@ def test_histogram_16bit_counters_carry(dtype, nbins):
     want = oracle.histogram(x, lo, hi, nbins)
     assert (got == want).all(), np.nonzero(got != want)[0][:5]
     assert int(got.sum()) == int(want.sum())
+
+
+@pytest.mark.parametrize("nbins", [16385, 65535, 65536])
+def test_histogram_16bit_merge_aligned_and_misaligned_counts(nbins):
+    """The 16-bit path merges a shared word's two halves with one 64-bit global
+    add when `counts` is 8-byte aligned (and n < 2^32), else with two 32-bit
+    adds; an odd nbins leaves the last word's high half without a bin (the
+    64-bit add must not touch counts[nbins]).  Both layouts, a sentinel past
+    the end, and counts that are not zero on entry (the call overwrites them)."""
+    import torch
+    rb = _rb()
+    n = (1 << 22) + 5
+    x = synth.make("float32", n, "uniform01", 61)
+    x[:1000] = np.float32(1.0 - 1e-7)  # the last bin gets a heavy count
+    t = to_device(x, 3)
+    want = oracle.histogram(x, 0.0, 1.0, nbins)
+    for off in (0, 1):  # counts 8-byte aligned, then 4 bytes past alignment
+        buf = torch.full((nbins + 4,), 12345, dtype=torch.int32, device="cuda")
+        counts = buf[off:off + nbins]
+        rb.histogram(t, 0.0, 1.0, nbins, counts=counts)
+        got = counts.cpu().numpy().view(np.uint32)
+        assert (got == want).all(), (nbins, off, np.nonzero(got != want)[0][:5])
+        assert int(buf[off + nbins].item()) == 12345  # nothing written past the end
