@@ -877,7 +877,7 @@ def main():
                     sec = time_calls(launch_3, regs_w, regs_t, stream, repeats=2)
                     pp = rb.query_plan(dt_name, op, m, in_ptr=regs_t[0].data_ptr(), **kw)
                     row[arm] = {"us": round(sec * 1e6, 2), "GBps": round(m * es / sec / 1e9, 1),
-                                "grid_combine": ["direct", "atomic", "two_pass", "last_block", "cluster"][pp["grid_combine"]],
+                                "grid_combine": rb.GC_NAMES[pp["grid_combine"]],
                                 "grid": pp["grid"], "block": pp["block"], "unroll": pp["unroll"]}
                 if dt_name == "float64" and op == "sum":
                     # distinct results over 20 runs on the same input

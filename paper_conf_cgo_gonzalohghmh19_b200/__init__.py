@@ -21,6 +21,7 @@ SUM, MIN, MAX, SUM_ACCURATE = 0, 1, 2, 3
 MODE_FAST, MODE_DETERMINISTIC = 0, 1
 BC_SHFL, BC_SMEM_ATOMIC_WARP, BC_SMEM_ATOMIC_ALL, BC_SMEM_TREE = 0, 1, 2, 3
 GC_DIRECT, GC_ATOMIC, GC_TWO_PASS, GC_LAST_BLOCK, GC_CLUSTER, GC_FLAGS = 0, 1, 2, 3, 4, 5
+GC_NAMES = ("direct", "atomic", "two_pass", "last_block", "cluster", "flags")  # indexed by reduce_grid_combine_t
 STAGE_REG, STAGE_SMEM = 1, 2
 FLAG_INPUT_READY = 1
 OK = 0

@@ -217,3 +217,13 @@ def test_binding_rejects_host_tensors_and_bad_outputs_without_cuda():
     o1 = rb._opts_for({"mode": "deterministic", "grid": 8})
     assert rb._opts_for({"grid": 8, "mode": "deterministic"}) is o1 and o1.mode == 1 and o1.grid == 8
     assert rb.make_opts(input_ready=True).flags == rb.FLAG_INPUT_READY
+
+
+def test_grid_combine_names_cover_every_combine():
+    """bench.py labels plans with GC_NAMES: every value the C side accepts has one."""
+    assert len(rb.GC_NAMES) == rb.GC_FLAGS + 1 and rb.GC_NAMES[rb.GC_FLAGS] == "flags"
+    for gc in range(len(rb.GC_NAMES)):
+        p = rb.query_plan("float32", "sum", 1 << 20, grid_combine=gc, **({"grid": 16} if gc == rb.GC_CLUSTER else {}))
+        assert p["grid_combine"] == gc
+    with pytest.raises(rb.ReduceError):
+        rb.query_plan("float32", "sum", 1 << 20, grid_combine=len(rb.GC_NAMES))
