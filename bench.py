@@ -738,7 +738,10 @@ def main():
         for dist_name, pool in (("U[0,1)", x), ("U[-1,1)", x_pm1)):
             for k in range(10, 29):
                 m = 1 << k
-                R = max(3, min(100, (256 << 20) // (4 * m))) if 4 * m < (256 << 20) else 20
+                # >= 20 calls per graph (the graph's own launch latency, ~1-3 us, is
+                # spread over R calls); regions cycle only when each is far beyond
+                # what L2 can keep between revisits (disjoint_regions)
+                R = max(20, min(100, (256 << 20) // (4 * m)))
                 warm, timed = disjoint_regions(pool, R, m)
                 p = rb.query_plan("float32", "sum", m, in_ptr=timed[0].data_ptr(), mode=args.mode)
                 ctr = [0]

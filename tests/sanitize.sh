@@ -1,7 +1,7 @@
 #!/usr/bin/env bash
 # compute-sanitizer pass over every kernel family (SURVEY section 4 "Sanitizers"):
 # memcheck, racecheck, synccheck and initcheck on small ragged sizes, every grid
-# combine (DIRECT, ATOMIC, TWO_PASS, LAST_BLOCK, CLUSTER), both staging modes,
+# combine (DIRECT, ATOMIC, TWO_PASS, LAST_BLOCK, CLUSTER, FLAGS), both staging modes,
 # every segmented group with and without the long-segment queue, the histogram
 # bin-replication and quotient paths, and the team combine.
 # Usage (GPU box): bash tests/sanitize.sh  -> exit 0 iff every tool reports 0 errors.
@@ -18,7 +18,8 @@ for dt in (torch.int32, torch.float32, torch.float64):
         for op in ("sum", "min", "max"):
             for kw in (dict(), dict(mode="deterministic"), dict(grid_combine=3), dict(grid_combine=4, grid=8),
                        dict(stage="smem", unroll=8, block=256), dict(block_combine=1), dict(block_combine=3, block=128),
-                       dict(input_ready=True), dict(grid_combine=1, block=32, unroll=1)):
+                       dict(input_ready=True), dict(grid_combine=1, block=32, unroll=1), dict(grid_combine=5),
+                       dict(grid_combine=5, block=32, unroll=1), dict(grid_combine=5, mode="deterministic", grid=3)):
                 rb.reduce(x, op, **kw)
         if dt != torch.int32:
             rb.reduce(x, "sum_accurate")
@@ -65,7 +66,7 @@ for dt in (torch.int32, torch.float32, torch.float64):
         if dt != torch.int32:
             rb.reduce_segmented(lbase, loffs, "sum_accurate", seg_group=g)
     if dt != torch.float64:
-        for nb in (7, 256, 4096, 20000, 1 << 20):
+        for nb in (7, 256, 4096, 20000, 20001, 1 << 20):
             rb.histogram(base, 0, 4000, nb)
         if dt == torch.int32:  # both int32 quotient paths and clamped bounds
             rb.histogram(base, -2.0 ** 31, 2.0 ** 31, 1000)
@@ -80,7 +81,7 @@ for dt in (torch.int32, torch.float32, torch.float64):
     for n in (0, 33, (1 << 20) + 3):
         x = torch.arange(n + 1, device="cuda").to(dt)[1:]
         for op in ("sum", "min", "max"):
-            for kw in (dict(), dict(mode="deterministic"), dict(grid_combine=4, grid=8)):
+            for kw in (dict(), dict(mode="deterministic"), dict(grid_combine=4, grid=8), dict(grid_combine=5)):
                 rb.reduce_multi_team(x, op, team, **kw)
 torch.cuda.synchronize()
 team.destroy()

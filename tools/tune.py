@@ -96,7 +96,7 @@ def run(args):
                 nbytes = 1 << lb
                 n = nbytes // ELEM[dtype]
                 # >= 20 calls per timed graph; regions repeat only when each is > 2x L2
-                R = max(20, min(100, (400 << 20) // nbytes)) if nbytes >= (256 << 20) else max(5, min(100, (400 << 20) // nbytes))
+                R = max(20, min(100, (400 << 20) // nbytes))
                 warm, timed = disjoint_regions(pool, R, n)
                 # every candidate timed in `rounds` interleaved rounds (box-level
                 # drift hits all candidates alike), the median per candidate decides
