@@ -135,16 +135,22 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
   // accurate sum, if the table predates it) falls back to the sum rows.  The
   // first-match scan runs once per (dtype, op, mode, log2 bytes); its result
   // is cached (a pointer store: benign if two threads fill the same entry).
+  // Calls with REDUCE_FLAG_INPUT_READY use their own tuned table (early
+  // register loads make other launch shapes win), when one was generated.
   const unsigned long long bytes = (unsigned long long)n * (unsigned long long)s;
   const int lb = ilog2_ceil(bytes ? bytes : 1);
-  static std::atomic<const DispatchEntry*> cache[3][4][2][64];
-  std::atomic<const DispatchEntry*>& slot = cache[dtype][op][mode][lb & 63];
+  const int ready = (kHaveReadyTable && (o.flags & REDUCE_FLAG_INPUT_READY)) ? 1 : 0;
+  static std::atomic<const DispatchEntry*> cache[2][3][4][2][64];
+  std::atomic<const DispatchEntry*>& slot = cache[ready][dtype][op][mode][lb & 63];
   const DispatchEntry* e = slot.load(std::memory_order_relaxed);
   if (e == nullptr) {
+    const DispatchEntry* tab = ready ? kDispatchReady : kDispatch;
+    const size_t rows = ready ? sizeof(kDispatchReady) / sizeof(kDispatchReady[0]) : sizeof(kDispatch) / sizeof(kDispatch[0]);
     for (int pass = 0; pass < 2 && (e == nullptr || e->dtype < 0); ++pass) {
       const int op_row = pass == 0 ? op : REDUCE_SUM;
       if (pass == 1 && op != REDUCE_SUM_ACCURATE) break;
-      for (const DispatchEntry& r : kDispatch) {
+      for (size_t i = 0; i < rows; ++i) {
+        const DispatchEntry& r = tab[i];
         if ((r.dtype < 0 || r.dtype == dtype) && (r.op < 0 || r.op == op_row) && (r.mode < 0 || r.mode == mode) &&
             lb <= r.max_log2_bytes) {
           if (e == nullptr || r.dtype >= 0) e = &r;
@@ -152,7 +158,7 @@ int make_plan(int dtype, int op, const void* in, size_t n, const reduce_opts_t* 
         }
       }
     }
-    if (!e) e = &kDispatch[sizeof(kDispatch) / sizeof(kDispatch[0]) - 1];
+    if (!e) e = &tab[rows - 1];
     slot.store(e, std::memory_order_relaxed);
   }
 

@@ -15,7 +15,7 @@ VARIANTS = [dict(), dict(mode="deterministic"), dict(grid_combine=0, block=256),
             dict(block_combine=3, block=128), dict(block_combine=1), dict(block_combine=2, block=128),
             dict(grid=148, grid_combine=3), dict(grid=148, grid_combine=1, unroll=1),
             dict(grid=7, grid_combine=2, block=64, unroll=2), dict(grid_combine=5), dict(grid_combine=5, block=32, unroll=1),
-            dict(grid=300, grid_combine=5, block=128)]
+            dict(grid=300, grid_combine=5, block=128), dict(input_ready=True), dict(input_ready=True, mode="deterministic")]
 
 
 @pytest.mark.parametrize("dtype,op", [("float32", "sum"), ("float64", "sum"), ("float32", "sum_accurate"),

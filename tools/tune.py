@@ -107,7 +107,7 @@ def run(args):
                     for ci, c in enumerate(cands):
                         if ci in failed:
                             continue
-                        opts = rb.make_opts(mode=mode, **c)
+                        opts = rb.make_opts(mode=mode, input_ready=args.input_ready, **c)
                         k = [0]
 
                         def launch(t, opts=opts):
@@ -117,7 +117,8 @@ def run(args):
                         try:
                             times[ci].append(time_calls(launch, warm, timed, stream, repeats=1))
                         except Exception as e:  # an invalid combination: record and skip
-                            results.append(dict(dtype=dtype, op=op, mode=mode, lb=lb, cfg=c, error=str(e)[:200]))
+                            results.append(dict(dtype=dtype, op=op, mode=mode, lb=lb, cfg=c, error=str(e)[:200],
+                                                ready=int(args.input_ready)))
                             torch.cuda.synchronize()
                             failed.add(ci)
                 best = None
@@ -126,28 +127,22 @@ def run(args):
                         continue
                     s = sorted(times[ci])[len(times[ci]) // 2]
                     results.append(dict(dtype=dtype, op=op, mode=mode, lb=lb, cfg=c, us=s * 1e6,
-                                        gbps=nbytes / s / 1e9, rounds_us=[round(t * 1e6, 3) for t in times[ci]]))
+                                        gbps=nbytes / s / 1e9, rounds_us=[round(t * 1e6, 3) for t in times[ci]],
+                                        ready=int(args.input_ready)))
                     if best is None or s < best[0]:
                         best = (s, c)
-                print(f"[{time.time() - t_start:7.1f}s] {dtype} {op} {mode} 2^{lb}B: best {best[0] * 1e6:8.2f} us "
+                print(f"[{time.time() - t_start:7.1f}s] {dtype} {op} {mode}{' ready' if args.input_ready else ''} 2^{lb}B: best {best[0] * 1e6:8.2f} us "
                       f"{nbytes / best[0] / 1e9:8.1f} GB/s {best[1]}", flush=True)
                 with open(args.out, "w") as f:
                     json.dump(results, f)
     return results
 
 
-def emit(paths, dst, tol=0.01):
+def table_rows(by, tol):
     """Pick, per (dtype, op, mode, log2 bytes), the fastest candidate -- but among
     candidates within `tol` of the fastest (timer noise) keep the previous size
     bucket's choice when it qualifies, so the table only changes where the
     measurements say it must."""
-    by = {}
-    for p in paths:  # a later file replaces earlier measurements of the same bucket
-        cur = {}
-        for r in json.load(open(p)):
-            if "us" in r:
-                cur.setdefault((r["dtype"], r["op"], r["mode"], r["lb"]), []).append(r)
-        by.update(cur)
     sig = lambda c: (c["block"], c["unroll"], c["grid_combine"], c["block_combine"], c["grid"], c.get("stage", 1))
     rows = []
     groups = sorted(set(k[:3] for k in by))
@@ -174,23 +169,45 @@ def emit(paths, dst, tol=0.01):
         if op == "max" and (dtype, "min", mode) not in groups:
             for r in [r for r in rows if r[:3] == (DT[dtype], OPC["max"], MODE[mode])]:
                 rows.append((r[0], OPC["min"]) + r[2:])
+    return rows
+
+
+def emit(paths, dst, tol=0.01):
+    """Write dispatch_table.inc: kDispatch from the default-path measurements and
+    kDispatchReady from the REDUCE_FLAG_INPUT_READY ones (tune.py --input-ready)."""
+    by = {0: {}, 1: {}}
+    for p in paths:  # a later file replaces earlier measurements of the same bucket
+        cur = {0: {}, 1: {}}
+        for r in json.load(open(p)):
+            if "us" in r:
+                cur[r.get("ready", 0)].setdefault((r["dtype"], r["op"], r["mode"], r["lb"]), []).append(r)
+        for k in (0, 1):
+            by[k].update(cur[k])
     lines = [
         "// dispatch_table.inc -- variant / launch choice per (dtype, op, mode, size).",
         "// Step S0 of DESIGN.md: the paper picks a code version per size and",
         "// architecture by tuning (P:L483); the winners change with size",
         "// (P:L681-L687, P:L691-L735, P:L739-L781).  GENERATED by tools/tune.py from",
         "// B200 measurements (device time per call, cold inputs); first match wins.",
+        "// kDispatch: the default (safe) stream ordering; kDispatchReady: calls with",
+        "// REDUCE_FLAG_INPUT_READY, whose first tile may be loaded before the",
+        "// programmatic dependency resolves (so other launch shapes win).",
         "//",
         "// fields: dtype, op, mode, max_log2_bytes, block, unroll, grid_combine, block_combine, grid_cap, stage",
         "//   (grid_cap 0 = one block per tile; stage 1 = registers, 2 = shared memory via cp.async)",
         "//   trailing comment: measured GB/s at the bucket that ended the row",
-        "static const DispatchEntry kDispatch[] = {",
     ]
-    for r in rows:
-        lines.append("    {%d, %d, %d, %d, %d, %d, %d, %d, %d, %d},  // %.1f GB/s" % r)
-    lines += ["    {-1, -1, -1, 63, 256, 4, -1, 0, 0, 1},  // fallback", "};", ""]
+    total = 0
+    for k, name in ((0, "kDispatch"), (1, "kDispatchReady")):
+        rows = table_rows(by[k], tol)
+        total += len(rows)
+        lines.append(f"static const DispatchEntry {name}[] = {{")
+        for r in rows:
+            lines.append("    {%d, %d, %d, %d, %d, %d, %d, %d, %d, %d},  // %.1f GB/s" % r)
+        lines += ["    {-1, -1, -1, 63, 256, 4, -1, 0, 0, 1},  // fallback", "};"]
+    lines += [f"static constexpr bool kHaveReadyTable = {'true' if by[1] else 'false'};", ""]
     open(dst, "w").write("\n".join(lines))
-    print(f"wrote {len(rows)} rows to {dst}")
+    print(f"wrote {total} rows to {dst}")
 
 
 def main():
@@ -203,6 +220,8 @@ def main():
     ap.add_argument("--out", default="gpurun_out/tune.json")
     ap.add_argument("--rounds", type=int, default=3, help="interleaved timing rounds per candidate (median wins)")
     ap.add_argument("--emit", nargs="*")
+    ap.add_argument("--input-ready", action="store_true",
+                    help="time every candidate with REDUCE_FLAG_INPUT_READY (rows for kDispatchReady)")
     ap.add_argument("--dst", default=os.path.join(ROOT, "paper_conf_cgo_gonzalohghmh19_b200", "csrc",
                                                   "dispatch_table.inc"))
     args = ap.parse_args()
