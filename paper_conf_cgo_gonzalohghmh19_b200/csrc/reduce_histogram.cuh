@@ -40,13 +40,21 @@ constexpr int kHistSharedMaxBins = 16384;  // 64 KB of u32 counters per block
 // 16-bit path: non-returning shared atomics with block-synchronous flushes
 // (k_histogram16r, 65536 bins 3.21 -> 3.78 TB/s fp32, 3.34 -> 3.67 TB/s int32)
 // instead of a returning atomic and a carry check per update (k_histogram16);
-// RB_HIST16_VPI vectors per thread per flush (0: 4 for int32, whose bin
-// arithmetic needs more registers, 6 for fp32; profiles/r02_hist_ab.txt)
+// RB_HIST16_VPI_{F32,I32} vectors per thread per flush, with the next
+// iteration's loads rolled across the flush (RB_HIST16_ROLL; 65536 bins fp32
+// 276.6 -> 253.6 us, int32 at 5 vectors 292.9 -> 274.0 us,
+// profiles/r02_hist_roll_ab.txt)
 #ifndef RB_HIST16_RED
 #define RB_HIST16_RED 1
 #endif
-#ifndef RB_HIST16_VPI
-#define RB_HIST16_VPI 0
+#ifndef RB_HIST16_ROLL
+#define RB_HIST16_ROLL 1
+#endif
+#ifndef RB_HIST16_VPI_F32
+#define RB_HIST16_VPI_F32 6
+#endif
+#ifndef RB_HIST16_VPI_I32
+#define RB_HIST16_VPI_I32 5
 #endif
 
 // Bin of one element, or -1 if it is not counted.  Branch-free (selects and
@@ -322,13 +330,16 @@ __global__ void __launch_bounds__(1024) k_histogram16r(const HistParams p) {
   // VPI vectors per thread per iteration (8 VPI x 1024 elements per block); a
   // half is moved once it reaches T, the largest power of two with
   // T + 8 VPI x 1024 <= 0xFFFF
-  constexpr int VPI = RB_HIST16_VPI > 0 ? RB_HIST16_VPI : (DT == DT_I32 ? 4 : 6);
+  constexpr int VPI = DT == DT_I32 ? RB_HIST16_VPI_I32 : RB_HIST16_VPI_F32;
   constexpr unsigned kE = 8u * VPI * 1024u;
   constexpr unsigned kT = kE <= 32767u ? 16384u : (kE <= 49151u ? 16384u >> 1 : (kE <= 57343u ? 4096u : 2048u));
   static_assert(kT + kE <= 0xFFFFu, "a half could wrap");
   constexpr unsigned kHalfMask = (~(kT - 1u)) & 0xFFFFu;
   constexpr unsigned kMask = kHalfMask | (kHalfMask << 16);
   auto flush = [&]() {
+#ifdef RB_HIST16_PROBE_NOFLUSH
+    return;
+#endif
     __syncthreads();
     for (int i = 4 * (int)threadIdx.x; i < words4; i += 4 * (int)blockDim.x) {
       const uint4 w = *reinterpret_cast<const uint4*>(sw + i);
@@ -352,6 +363,25 @@ __global__ void __launch_bounds__(1024) k_histogram16r(const HistParams p) {
   // in flush): vectors past the body are skipped inside
   const unsigned long long per_iter = VPI * stride;
   const unsigned long long iters = (p.body_vecs + per_iter - 1) / per_iter;
+#if RB_HIST16_ROLL
+  // rolling loads: vector u of the next iteration is loaded into r[u] as soon
+  // as this iteration's vector u is counted, so the next iteration's loads are
+  // in flight across the flush and its barriers (1 block per SM: no other
+  // block hides the latency there; A/B profiles/r02_hist_roll_ab.txt)
+  uint32_t r[VPI][8];
+#pragma unroll
+  for (int u = 0; u < VPI; ++u)
+    if (v + u * stride < p.body_vecs) ld_v8(p.body + (v + u * stride) * kVecBytes, r[u]);
+  for (unsigned long long it = 0; it < iters; ++it, v += per_iter) {
+    const unsigned long long vn = v + per_iter;
+#pragma unroll
+    for (int u = 0; u < VPI; ++u) {
+      if (v + u * stride < p.body_vecs) count8(r[u]);
+      if (vn + u * stride < p.body_vecs) ld_v8(p.body + (vn + u * stride) * kVecBytes, r[u]);
+    }
+    flush();
+  }
+#else
   for (unsigned long long it = 0; it < iters; ++it, v += per_iter) {
     uint32_t r[VPI][8];
 #pragma unroll
@@ -362,6 +392,7 @@ __global__ void __launch_bounds__(1024) k_histogram16r(const HistParams p) {
       if (v + u * stride < p.body_vecs) count8(r[u]);
     flush();
   }
+#endif
   if (blockIdx.x == 0 && threadIdx.x < 16) {  // head and tail elements (< 8 each)
     const int t = threadIdx.x;
     const bool mine = t < p.head || (t >= 8 && t - 8 < p.tail);
@@ -373,6 +404,9 @@ __global__ void __launch_bounds__(1024) k_histogram16r(const HistParams p) {
     }
   }
   __syncthreads();
+#ifdef RB_HIST16_PROBE_NOMERGE
+  return;
+#endif
   // final merge: a word's two halves into counts[2i], counts[2i + 1] with ONE
   // 64-bit global add when both bins exist and no count can carry into its
   // neighbour (p.merge64), else two 32-bit adds -- the 148 x 32768 merge adds
@@ -401,8 +435,12 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+#ifdef RB_HIST_PROBE_NOMEMSET
+  cudaError_t e = cudaSuccess;  // measurement only: counts are not zeroed
+#else
   cudaError_t e = cudaMemsetAsync(p.counts, 0, (size_t)p.nbins * sizeof(unsigned), s);
   if (e != cudaSuccess) return e;
+#endif
   if (p.nbins > kHistSharedMaxBins) {  // one pass with 16-bit shared counters if the histogram fits
     int optin = 0;
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);

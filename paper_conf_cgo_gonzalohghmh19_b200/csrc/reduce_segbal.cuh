@@ -25,11 +25,14 @@
 //                   prefetched) is copied into shared memory as chunk-local
 //                   positions; each lane turns the boundaries in its range
 //                   into a bit mask, folds its elements in order, closing a
-//                   piece at every set bit (pieces go to shared memory).  A
-//                   segmented scan over the 32 lanes (5 shuffle steps, fixed
-//                   order) joins the pieces of segments that cross lanes.
-//                   Segments that start and end in the chunk are written
-//                   directly.  A chunk without boundaries folds with the plain
+//                   piece at every set bit (the piece a boundary at chunk
+//                   position e closes goes to shared slot e).  A segmented
+//                   scan over the 32 lanes (5 shuffle steps, fixed order)
+//                   joins the pieces of segments that cross lanes.  Segments
+//                   that start and end in the chunk are then written in list
+//                   order, 32 consecutive outputs per store instruction (the
+//                   value of [list[j], list[j+1]) is slot list[j+1]).  A
+//                   chunk without boundaries folds with the plain
 //                   vector tree.  The range leaves its first piece (the
 //                   segment open at its start) and its last (the segment
 //                   open at its end) for the fix-up.
@@ -58,6 +61,9 @@ namespace rb {
 #ifndef RB_SEGBAL_MINB
 #define RB_SEGBAL_MINB 5
 #endif
+#ifndef RB_SEGBAL_L1PF
+#define RB_SEGBAL_L1PF 0
+#endif
 constexpr int kBalWarps = 4;                    // warps per block of k_segbal
 // resident blocks asked of ptxas: 5 (96 registers, 20 warps per SM) for the
 // 4-byte plain ops; fp64 and accurate sums need more registers (4 blocks)
@@ -73,7 +79,7 @@ struct Bal {
   static constexpr int kList = (int)C + 64;           // offsets entries kept in shared memory
   static constexpr size_t kPieceBytes = (size_t)EL * 32 * sizeof(Acc);
   static constexpr size_t kListBytes = ((size_t)kList * 2 + 15) / 16 * 16;
-  static constexpr size_t kLaneBytes = 32 * 4 * 2;  // per lane: boundary mask word, list entries count
+  static constexpr size_t kLaneBytes = 32 * 4;  // per lane: boundary mask word
   static constexpr size_t kWarpSmem = kPieceBytes + kListBytes + kLaneBytes;
 };
 
@@ -307,7 +313,6 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
   Acc* pieces = reinterpret_cast<Acc*>(bal_smem + wib * B::kWarpSmem);
   short* list = reinterpret_cast<short*>(bal_smem + wib * B::kWarpSmem + B::kPieceBytes);
   unsigned* lmask = reinterpret_cast<unsigned*>(bal_smem + wib * B::kWarpSmem + B::kPieceBytes + B::kListBytes);
-  unsigned* lcnt = lmask + 32;
   pdl_wait();
   const long long nseg = p.nseg;
   const long long E0 = __ldg(p.offsets), E1 = __ldg(p.offsets + nseg);
@@ -358,6 +363,11 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
   auto prefetch_list = [&](long long s) {
     vfirst = s + lane <= nseg ? __ldg(p.offsets + s + lane) : LLONG_MAX;
     vsecond = s + 32 + lane <= nseg ? __ldg(p.offsets + s + 32 + lane) : LLONG_MAX;
+#if RB_SEGBAL_L1PF
+    // the entries past those two batches into L1 (one 128-byte line per lane:
+    // 512 offsets), so a chunk of short segments finds its further batches there
+    if (s + 64 + 16 * lane <= nseg) asm volatile("prefetch.global.L1 [%0];" ::"l"(p.offsets + s + 64 + 16 * lane));
+#endif
   };
   // the chunk's data: loaded into `cur` as soon as the previous chunk's fold
   // has consumed it, so the loads fly during that chunk's scan / emission and
@@ -380,7 +390,6 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
     // entries fall there, set with shared atomics as the list is built (no
     // per-lane search of the list afterwards)
     lmask[lane] = 0u;
-    lcnt[lane] = 0u;
     __syncwarp();
     // batches past the two prefetched ones are loaded four at a time (chunks
     // of very short segments need dozens: one round trip per four, not per one)
@@ -397,10 +406,7 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
       }
       if (lane < cnt) {
         list[m + lane] = (short)loc;
-        if (loc >= 0 && loc < (int)B::C) {
-          atomicOr(lmask + loc / B::EL, 1u << (loc % B::EL));
-          atomicAdd(lcnt + loc / B::EL, 1u);
-        }
+        if (loc >= 0 && loc < (int)B::C) atomicOr(lmask + loc / B::EL, 1u << (loc % B::EL));
       }
       m += cnt;
       if (stop) break;
@@ -427,25 +433,12 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
     k.s_next = s0 + m - 2;
     if (ovf) k.s_next = bal_walk_next(p.offsets, nseg, s0 + m, chi, lane);
     if (c + 1 < ce) prefetch_list(k.s_next);  // the next chunk's offsets, while this one folds
-    int i0 = 0, np = 0;
-    bool lane_dups = false;
     unsigned long long mask = 0;
     unsigned fb = 0;
     Acc tv = T::ident();  // the lane's value (no boundary in the chunk) or its last piece
     if (!ovf) {
-      // the lane's boundaries as a bit mask (bit e: a segment starts at element e),
-      // and i0 = the list index of its first boundary: the entries before the
-      // chunk (list[0] == -1) plus those of the lanes below
+      // the lane's boundaries as a bit mask (bit e: a segment starts at element e)
       mask = lmask[lane];
-      const int cnt = (int)lcnt[lane];
-      int incl = cnt;
-#pragma unroll
-      for (int d = 1; d < 32; d <<= 1) {
-        const int y = __shfl_up_sync(0xffffffffu, incl, d);
-        if (lane >= d) incl += y;
-      }
-      i0 = incl - cnt + (list[0] < 0 ? 1 : 0);
-      lane_dups = cnt != __popcll(mask);  // repeated offsets (empty segments) in this lane's elements
       fb = __ballot_sync(0xffffffffu, mask != 0ull);
       if (fb == 0u) {  // no boundary in the chunk: plain vector-tree fold
         Part<T> acc[T::NA];
@@ -455,14 +448,15 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
         for (int j = 0; j < kBalVecsPerLane; ++j) fold_vec<T>(acc, aux, cur[j], j);
         tv = thread_result<T>(acc, aux);
       } else {
-        // fold element by element, closing a piece at every boundary
+        // fold element by element; the piece that a boundary at element e
+        // closes goes to slot e of the lane (pieces[e * 32 + lane]: a constant
+        // address per element, bank = lane)
         Part<T> a = PartOf<T>::ident();
         uint32_t aux = 0;
 #pragma unroll
         for (int e = 0; e < B::EL; ++e) {  // fully unrolled: constant register indices and shifts
           if ((mask >> e) & 1ull) {
-            pieces[np * 32 + lane] = T::finish(PartOf<T>::to_acc(a), aux);
-            ++np;
+            pieces[e * 32 + lane] = T::finish(PartOf<T>::to_acc(a), aux);
             a = PartOf<T>::ident();
             aux = 0;
           }
@@ -498,29 +492,23 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
         const Acc carry_in = shfl_up_v(x, 1);
         Grid firstv = T::gident();
         if (f) {
-          const Acc head = pieces[lane];
+          // the lane's first piece closes the segment open at its start
+          const int e1 = __ffsll((long long)mask) - 1;
+          const Acc head = pieces[e1 * 32 + lane];
           const Acc close = lane > 0 ? T::comb(carry_in, head) : head;
-          if (fb & ((1u << lane) - 1u)) {  // the segment holding element a0 - 1 closes here
-            bal_store<T>(p, (long long)s0 + i0 - 1, T::to_grid(close));
-          } else {                          // the chunk's first boundary: the incoming segment's piece
-            firstv = T::to_grid(close);
-          }
-          // segments that start and end in this lane: the one opened by the
-          // lane's q-th boundary is s0 + (its list index); without repeated
-          // offsets in the lane that index is i0 + q - 1
-          if (!lane_dups) {
+          if (fb & ((1u << lane) - 1u)) pieces[e1 * 32 + lane] = close;  // opened in this chunk
+          else firstv = T::to_grid(close);  // the chunk's first boundary: the incoming segment
+        }
+        __syncwarp();
+        // every segment that starts and ends in the chunk, in list order (one
+        // coalesced store per 32): segment s0 + j is [list[j], list[j + 1]);
+        // its value is the piece closed at list[j + 1] (empty segments keep
+        // the identity the scan kernel wrote)
+        const int jA = list[0] < 0 ? 1 : 0;
 #pragma unroll 1
-            for (int q = 1; q < np; ++q) bal_store<T>(p, (long long)s0 + i0 + q - 1, T::to_grid(pieces[q * 32 + lane]));
-          } else {
-            int j = i0;
-#pragma unroll 1
-            for (int q = 1; q < np; ++q) {
-              const int o = list[j];
-              while (list[j + 1] == o) ++j;
-              bal_store<T>(p, (long long)s0 + j, T::to_grid(pieces[q * 32 + lane]));
-              ++j;
-            }
-          }
+        for (int j = jA + lane; j < m - 2; j += 32) {
+          const int lo = list[j], hi = list[j + 1];
+          if (lo != hi) bal_store<T>(p, (long long)s0 + j, T::to_grid(pieces[(hi % B::EL) * 32 + hi / B::EL]));
         }
         k.first = shfl_idx_v(firstv, __ffs(fb) - 1);
         k.last = shfl_idx_v(T::to_grid(x), 31);
