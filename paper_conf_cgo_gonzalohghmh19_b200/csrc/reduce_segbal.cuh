@@ -50,6 +50,7 @@
 // modulo 32 and offsets[0].
 #pragma once
 #include <climits>
+#include <cstdlib>
 #include "reduce_segmented.cuh"
 
 namespace rb {
@@ -60,9 +61,6 @@ namespace rb {
 #endif
 #ifndef RB_SEGBAL_MINB
 #define RB_SEGBAL_MINB 5
-#endif
-#ifndef RB_SEGBAL_L1PF
-#define RB_SEGBAL_L1PF 0
 #endif
 constexpr int kBalWarps = 4;                    // warps per block of k_segbal
 // resident blocks asked of ptxas: 5 (96 registers, 20 warps per SM) for the
@@ -363,11 +361,6 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
   auto prefetch_list = [&](long long s) {
     vfirst = s + lane <= nseg ? __ldg(p.offsets + s + lane) : LLONG_MAX;
     vsecond = s + 32 + lane <= nseg ? __ldg(p.offsets + s + 32 + lane) : LLONG_MAX;
-#if RB_SEGBAL_L1PF
-    // the entries past those two batches into L1 (one 128-byte line per lane:
-    // 512 offsets), so a chunk of short segments finds its further batches there
-    if (s + 64 + 16 * lane <= nseg) asm volatile("prefetch.global.L1 [%0];" ::"l"(p.offsets + s + 64 + 16 * lane));
-#endif
   };
   // the chunk's data: loaded into `cur` as soon as the previous chunk's fold
   // has consumed it, so the loads fly during that chunk's scan / emission and
@@ -608,6 +601,17 @@ cudaError_t bal_launch(K kernel, long long grid, int block, size_t smem, const S
   return cudaLaunchKernelEx(&cfg, kernel, p);
 }
 
+// Measurement only (tools/probes/segbal_split.py): REDUCE_SEGBAL_ONLY=scan|main|fix
+// launches just that kernel of the three, reusing what the previous full call
+// left in the workspace (same inputs: same values), to time each in a graph.
+// (read on every call once it was set at the first call: the probe switches it)
+inline int segbal_only() {
+  static const bool probing = std::getenv("REDUCE_SEGBAL_ONLY") != nullptr;
+  if (!probing) return 0;
+  const char* e = std::getenv("REDUCE_SEGBAL_ONLY");
+  return !e ? 0 : (e[0] == 's' ? 1 : (e[0] == 'm' ? 2 : (e[0] == 'f' ? 3 : 0)));
+}
+
 template <int DT, int OP>
 cudaError_t launch_segbal_op(const SegParams& p0, int sms, cudaStream_t s) {
   using B = Bal<Tr<DT, OP>>;
@@ -624,13 +628,19 @@ cudaError_t launch_segbal_op(const SegParams& p0, int sms, cudaStream_t s) {
   const int K = p.nseg <= full ? 1 : (p.nseg <= 4 * full ? 4 : 8);
   long long sgrid = (p.nseg + 256ll * K - 1) / (256ll * K);
   if (sgrid > (long long)sms * 8) sgrid = (long long)sms * 8;
-  e = K == 1 ? bal_launch(k_segbal_scan<DT, OP, 1>, sgrid, 256, 0, p, s)
-             : (K == 4 ? bal_launch(k_segbal_scan<DT, OP, 4>, sgrid, 256, 0, p, s)
-                       : bal_launch(k_segbal_scan<DT, OP, 8>, sgrid, 256, 0, p, s));
-  if (e != cudaSuccess) return e;
-  e = bal_launch(k_segbal<DT, OP>, grid, kBalWarps * 32, smem, p, s);
-  if (e != cudaSuccess) return e;
-  return bal_launch(k_segbal_fix<DT, OP>, (p.b.nranges + 7) / 8, 256, 0, p, s);
+  const int only = segbal_only();
+  if (only == 0 || only == 1) {
+    e = K == 1 ? bal_launch(k_segbal_scan<DT, OP, 1>, sgrid, 256, 0, p, s)
+               : (K == 4 ? bal_launch(k_segbal_scan<DT, OP, 4>, sgrid, 256, 0, p, s)
+                         : bal_launch(k_segbal_scan<DT, OP, 8>, sgrid, 256, 0, p, s));
+    if (e != cudaSuccess) return e;
+  }
+  if (only == 0 || only == 2) {
+    e = bal_launch(k_segbal<DT, OP>, grid, kBalWarps * 32, smem, p, s);
+    if (e != cudaSuccess) return e;
+  }
+  if (only == 0 || only == 3) return bal_launch(k_segbal_fix<DT, OP>, (p.b.nranges + 7) / 8, 256, 0, p, s);
+  return cudaSuccess;
 }
 
 template <int DT>
