@@ -143,3 +143,50 @@ def test_histogram_16bit_merge_aligned_and_misaligned_counts(nbins):
         got = counts.cpu().numpy().view(np.uint32)
         assert (got == want).all(), (nbins, off, np.nonzero(got != want)[0][:5])
         assert int(buf[off + nbins].item()) == 12345  # nothing written past the end
+
+
+def test_histogram_back_to_back_and_graphs():
+    """Every call overwrites `counts` whatever they held: back-to-back calls on
+    one stream with different bin counts and grid sizes (the replicated 32-bit,
+    bin-range and 16-bit paths), garbage in `counts` on entry, inputs rewritten
+    by torch kernels right before each call, reduce() calls interleaved, and a
+    captured graph replayed with fresh inputs."""
+    import torch
+    rb = _rb()
+    s = torch.cuda.Stream()
+    cases = [(256, 0), (1000, 1), (65536, 4097), (40000, 1 << 20), (7, 13), (16384, (1 << 21) + 3), (256, 1 << 22)]
+    with torch.cuda.stream(s):
+        rb.prepare(s, 1 << 22)
+        xs = [torch.empty(n, dtype=torch.float32, device="cuda") for _, n in cases]
+        outs = [torch.full((nb,), -7, dtype=torch.int32, device="cuda") for nb, _ in cases]
+        for it in range(3):
+            hosts = []
+            for k, ((nb, n), xt) in enumerate(zip(cases, xs)):
+                x = synth.make("float32", n, "uniform_pm1", 700 + 10 * it + k)
+                xt.copy_(torch.from_numpy(x).to("cuda", non_blocking=False))
+                xt.mul_(1.0)  # a torch kernel writes the input right before the histogram
+                outs[k].fill_(12345)
+                rb.histogram(xt, -0.9, 0.95, nb, counts=outs[k], stream=s)
+                rb.reduce(xt, "max", stream=s) if n else None
+                hosts.append(x)
+            s.synchronize()
+            for (nb, n), x, o in zip(cases, hosts, outs):
+                want = oracle.histogram(x, -0.9, 0.95, nb)
+                got = o.cpu().numpy().view(np.uint32)
+                assert (got == want).all(), (it, nb, n, np.nonzero(got != want)[0][:5])
+        # graph: two histograms captured, replayed with new inputs
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            rb.histogram(xs[2], -0.9, 0.95, 65536, counts=outs[2], stream=s)
+            rb.histogram(xs[6], -0.9, 0.95, 256, counts=outs[6], stream=s)
+        for rep in range(3):
+            x2 = synth.make("float32", xs[2].numel(), "uniform_pm1", 900 + rep)
+            x6 = synth.make("float32", xs[6].numel(), "uniform_pm1", 950 + rep)
+            xs[2].copy_(torch.from_numpy(x2))
+            xs[6].copy_(torch.from_numpy(x6))
+            outs[2].fill_(-1)
+            outs[6].fill_(-1)
+            g.replay()
+            s.synchronize()
+            assert (outs[2].cpu().numpy().view(np.uint32) == oracle.histogram(x2, -0.9, 0.95, 65536)).all(), rep
+            assert (outs[6].cpu().numpy().view(np.uint32) == oracle.histogram(x6, -0.9, 0.95, 256)).all(), rep
