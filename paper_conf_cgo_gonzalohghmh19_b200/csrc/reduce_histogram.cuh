@@ -92,27 +92,67 @@ __device__ __forceinline__ int hist_bin(uint32_t w, const HistParams& p) {
   }
 }
 
+// The same rule in fewer instructions for the shared-memory kernels (nbins <=
+// 2^22): the bin as an unsigned value, >= nbins when the element is not
+// counted.  fp32: floor(t) for t = fl(fl(x - lo) * scale) in [0, 2^23) is the
+// bit pattern of fl_rz(t + 2^23) minus that of 2^23 (the round-toward-zero
+// add lands on the integer grid), so no float-to-int conversion; t < 0
+// (x < lo) wraps to a huge value, NaN and x >= hi are forced out by the one
+// compare left.  The kernels were issue-bound on this arithmetic (ncu,
+// profiles/r02_ncu_hist_pairs_vs_16r.json).
+#ifndef RB_HIST_UBIN
+#define RB_HIST_UBIN 1
+#endif
+template <int DT>
+__device__ __forceinline__ unsigned hist_ubin(uint32_t w, const HistParams& p) {
+  if constexpr (DT == DT_I32) {
+    if (p.narrow) {
+      const bool in = w - p.lo_c32 <= p.lim32;
+      const unsigned num = (w - p.lo32) * (unsigned)p.nbins;
+      const unsigned t = __umulhi(num, p.magic32);
+      const unsigned q = (t + ((num - t) >> 1)) >> p.shift32;
+      return in ? q : 0xFFFFFFFFu;
+    }
+    const int b = hist_bin<DT>(w, p);
+    return b < 0 ? 0xFFFFFFFFu : (unsigned)b;
+  } else {
+#if RB_HIST_UBIN
+    const float x = __uint_as_float(w);
+    const float t = __fmul_rn(__fsub_rn(x, p.lo_f), p.scale_f);
+    const unsigned u = __float_as_uint(__fadd_rz(t, 8388608.0f)) - 0x4B000000u;
+    return x < p.hi_f ? u : 0xFFFFFFFFu;
+#else
+    const int b = hist_bin<DT>(w, p);
+    return b < 0 ? 0xFFFFFFFFu : (unsigned)b;
+#endif
+  }
+}
+
 // Count the 8 elements of one vector: bins [b0, b1) in shared memory at byte
 // address sbase (this lane's copy; a bin's R copies are adjacent words), or
 // straight into global `counts`.
 template <int DT, bool kShared>
 __device__ __forceinline__ void hist_vec(const uint32_t (&r)[8], const HistParams& p, uint32_t sbase,
                                          uint32_t sdummy, int rshift, int b0, int b1) {
-  int bin[8];
+  if constexpr (kShared) {
+    unsigned ub[8];
 #pragma unroll
-  for (int k = 0; k < 8; ++k) bin[k] = hist_bin<DT>(r[k], p);
+    for (int k = 0; k < 8; ++k) ub[k] = hist_ubin<DT>(r[k], p) - (unsigned)b0;  // >= b1 - b0: not counted here
 #pragma unroll
-  for (int k = 0; k < 8; ++k) {
-    if constexpr (kShared) {
-      // unconditional: an element that is not counted adds 0 to this lane's
-      // own dummy word (ptxas turns any predicated shared atomic into a
-      // branch-wrapped one -- a reconvergence region per element)
-      const uint32_t ok = bin[k] >= b0 && bin[k] < b1;
-      const uint32_t a = ok ? sbase + ((uint32_t)(bin[k] - b0) << (rshift + 2)) : sdummy;
-      asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(ok) : "memory");
-    } else {
-      if (bin[k] >= 0) atomicAdd(p.counts + bin[k], 1u);
+    for (int k = 0; k < 8; ++k) {
+      // unconditional: an element that is not counted adds to this lane's own
+      // dummy word, never merged (ptxas turns any predicated shared atomic
+      // into a branch-wrapped one -- a reconvergence region per element)
+      const uint32_t a = ub[k] < (unsigned)(b1 - b0) ? sbase + (ub[k] << (rshift + 2)) : sdummy;
+      asm volatile("red.shared.add.u32 [%0], 1;" ::"r"(a) : "memory");
     }
+  } else {
+    int bin[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) bin[k] = hist_bin<DT>(r[k], p);
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (bin[k] >= 0) atomicAdd(p.counts + bin[k], 1u);
   }
 }
 
@@ -316,15 +356,13 @@ __global__ void __launch_bounds__(1024) k_histogram16r(const HistParams p) {
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(sw);
   const uint32_t sdummy = sbase + 4u * (uint32_t)(words4 + (threadIdx.x & 31));
   auto count8 = [&](const uint32_t (&r)[8]) {
-    int bin[8];
+    unsigned u[8];
 #pragma unroll
-    for (int k = 0; k < 8; ++k) bin[k] = hist_bin<DT>(r[k], p);
+    for (int k = 0; k < 8; ++k) u[k] = hist_ubin<DT>(r[k], p);  // >= nbins: not counted
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {  // unconditional (uncounted elements add 0 to the lane's dummy word)
-      const bool ok = bin[k] >= 0;
-      const uint32_t a = ok ? sbase + 4u * (uint32_t)(bin[k] >> 1) : sdummy;
-      const uint32_t inc = ok ? 1u << ((bin[k] & 1) << 4) : 0u;
-      asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(inc) : "memory");
+    for (int k = 0; k < 8; ++k) {  // unconditional (uncounted elements go to the lane's dummy word, never read)
+      const uint32_t a = u[k] < (unsigned)p.nbins ? sbase + 4u * (u[k] >> 1) : sdummy;
+      asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(1u << ((u[k] & 1u) << 4)) : "memory");
     }
   };
   // VPI vectors per thread per iteration (8 VPI x 1024 elements per block); a
