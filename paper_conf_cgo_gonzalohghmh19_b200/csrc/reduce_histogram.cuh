@@ -461,9 +461,24 @@ __global__ void __launch_bounds__(1024) k_histogram16r(const HistParams p) {
   }
 }
 
-// Copies per bin: as many as keep a block's bins within 64 KB (<= 32).
+#ifndef RB_HIST_REP_MAX
+#define RB_HIST_REP_MAX 5
+#endif
+// Resident blocks per SM of the shared-bin kernel (256 threads each): 4
+// (1024 threads) beat the occupancy maximum of 7-8 for fp32 (256 bins 167.9 ->
+// 154.0 us; 2 per SM: 181 us; profiles/r02_hist_heur_bps_ab.txt); int32's
+// registers allow 3 anyway.
+#ifndef RB_HIST_BLOCKS_PER_SM
+#define RB_HIST_BLOCKS_PER_SM 4
+#endif
+// Copies per bin (round 2): only as many as give >= 256 distinct words (few
+// bins: one copy per lane group, so a warp's updates do not pile onto a
+// handful of addresses); from 256 bins up one copy -- the 32-copy layout
+// (lane l -> copy l, conflict-free banks) measured 12-19 % slower there
+// (fp32 256 bins 195.0 -> 171.2 us, profiles/r02_hist_rep_bps_ab.txt).
 inline int hist_rep_log2(int bins_per_block) {
-  int rl = 5;
+  int rl = 0;
+  while (rl < RB_HIST_REP_MAX && (long long)bins_per_block << rl < 256) ++rl;
   while (rl > 0 && (long long)bins_per_block * (1 << rl) * 4 > 64 * 1024) --rl;
   return rl;
 }
@@ -511,7 +526,8 @@ cudaError_t launch_histogram_dt(const HistParams& p, int block, cudaStream_t s) 
     if (e != cudaSuccess) return e;
   }
   // one wave per part group: as many blocks as fit (the shared bins limit residency)
-  const int per_sm = blocks_per_sm((const void*)kernel, block, smem);
+  int per_sm = blocks_per_sm((const void*)kernel, block, smem);
+  if (shared && RB_HIST_BLOCKS_PER_SM > 0 && per_sm > RB_HIST_BLOCKS_PER_SM) per_sm = RB_HIST_BLOCKS_PER_SM;
   long long per_part = (long long)sms * per_sm / (shared ? parts : 1);
   const long long need = (long long)((p.body_vecs + block - 1) / block);
   if (need < per_part) per_part = need;

@@ -190,3 +190,32 @@ def test_histogram_back_to_back_and_graphs():
             s.synchronize()
             assert (outs[2].cpu().numpy().view(np.uint32) == oracle.histogram(x2, -0.9, 0.95, 65536)).all(), rep
             assert (outs[6].cpu().numpy().view(np.uint32) == oracle.histogram(x6, -0.9, 0.95, 256)).all(), rep
+
+
+
+@pytest.mark.parametrize("nbins", [1, 3, 256, 1000, 16384, 16385, 65536, 100000, 131072])
+def test_histogram_f32_bin_edges(nbins):
+    """The shared-memory kernels compute an fp32 bin as the bits of
+    fl_rz(t + 2^23) minus those of 2^23 (t = fl(fl(x - lo) * scale)) instead of a
+    float-to-int conversion; x < lo must wrap out of range and x >= hi / NaN be
+    forced out.  Elements at and one ulp around lo, hi and every sampled bin
+    edge, -0.0 with lo = 0, subnormals, +-inf, NaN, on two ranges (bit-exact
+    against the oracle's rule, DESIGN R13)."""
+    rb = _rb()
+    rng = np.random.Generator(np.random.PCG64(77 + nbins))
+    for lo, hi in ((0.0, 1.0), (-3.25, 11.5)):
+        lo32, hi32 = np.float32(lo), np.float32(hi)
+        k = np.unique(np.concatenate([np.arange(min(nbins, 64)), rng.integers(0, nbins + 1, 2000)]))
+        edges = (lo32 + (k.astype(np.float64) * (hi - lo) / nbins)).astype(np.float32)
+        vals = [edges, np.nextafter(edges, np.float32(-np.inf)), np.nextafter(edges, np.float32(np.inf)),
+                np.array([lo32, hi32, np.nextafter(lo32, np.float32(-1e30)), np.nextafter(hi32, np.float32(-1e30)),
+                          np.nextafter(hi32, np.float32(1e30)), np.float32(-0.0), np.float32(1e-45),
+                          np.float32(-1e-45), np.float32(np.inf), np.float32(-np.inf), np.float32(np.nan)],
+                         dtype=np.float32)]
+        x = np.concatenate(vals).astype(np.float32)
+        x = np.concatenate([x, rng.uniform(lo - 1, hi + 1, 300_000).astype(np.float32)])
+        rng.shuffle(x)
+        t = to_device(x, 5)
+        got = rb.histogram(t, lo, hi, nbins).cpu().numpy().view(np.uint32)
+        want = oracle.histogram(x, lo, hi, nbins)
+        assert (got == want).all(), (nbins, lo, hi, np.nonzero(got != want)[0][:5])

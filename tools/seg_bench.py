@@ -86,7 +86,7 @@ def main():
     for dtype, t, lo, hi in (("float32", xh, 0.0, 1.0), ("int32", xi, -1000.0, 1001.0)):
         if args.only and args.only != "histogram":
             break
-        for nbins in (16, 256, 512, 1024, 4096, 16384, 65536):
+        for nbins in (1, 4, 16, 64, 256, 512, 1024, 4096, 16384, 65536):
             if args.quick and nbins not in (256, 65536):
                 continue
             hc = torch.empty(nbins, dtype=torch.int32, device=dev)
