@@ -66,7 +66,7 @@ for dt in (torch.int32, torch.float32, torch.float64):
         if dt != torch.int32:
             rb.reduce_segmented(lbase, loffs, "sum_accurate", seg_group=g)
     if dt != torch.float64:
-        for nb in (7, 256, 4096, 20000, 20001, 1 << 20):
+        for nb in (1, 7, 16, 256, 4096, 20000, 20001, 65536, 1 << 20):
             rb.histogram(base, 0, 4000, nb)
         if dt == torch.int32:  # both int32 quotient paths and clamped bounds
             rb.histogram(base, -2.0 ** 31, 2.0 ** 31, 1000)
