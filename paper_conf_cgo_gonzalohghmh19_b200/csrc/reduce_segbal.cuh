@@ -62,6 +62,9 @@ namespace rb {
 #ifndef RB_SEGBAL_MINB
 #define RB_SEGBAL_MINB 5
 #endif
+#ifndef RB_SEGBAL_SPLIT
+#define RB_SEGBAL_SPLIT 1
+#endif
 constexpr int kBalWarps = 4;                    // warps per block of k_segbal
 // resident blocks asked of ptxas: 5 (96 registers, 20 warps per SM) for the
 // 4-byte plain ops; fp64 and accurate sums need more registers (4 blocks)
@@ -429,6 +432,16 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
     unsigned long long mask = 0;
     unsigned fb = 0;
     Acc tv = T::ident();  // the lane's value (no boundary in the chunk) or its last piece
+    // an interior next chunk is loaded in two halves, the first as soon as the
+    // fold has consumed the first half of `cur` (RB_SEGBAL_SPLIT; power-law
+    // 60.4 -> 57.6 us; each vector as soon as it is consumed: slower,
+    // profiles/r02_segbal_split_ab.txt, profiles/r02_segbal_split2_ab.txt)
+    const bool split = RB_SEGBAL_SPLIT && !ovf && c + 1 < ce && interior(c + 1);
+    const char* lpn = p.in + ((P0 + (c + 1) * B::C) + (long long)lane * B::EL) * B::s;
+    auto load_half = [&](int h) {
+#pragma unroll
+      for (int j = h * kBalVecsPerLane / 2; j < (h + 1) * kBalVecsPerLane / 2; ++j) ld_v8(lpn + j * kVecBytes, cur[j]);
+    };
     if (!ovf) {
       // the lane's boundaries as a bit mask (bit e: a segment starts at element e)
       mask = lmask[lane];
@@ -438,7 +451,10 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
         init_parts<T>(acc);
         uint32_t aux = 0;
 #pragma unroll
-        for (int j = 0; j < kBalVecsPerLane; ++j) fold_vec<T>(acc, aux, cur[j], j);
+        for (int j = 0; j < kBalVecsPerLane; ++j) {
+          fold_vec<T>(acc, aux, cur[j], j);
+          if (j == kBalVecsPerLane / 2 - 1 && split) load_half(0);
+        }
         tv = thread_result<T>(acc, aux);
       } else {
         // fold element by element; the piece that a boundary at element e
@@ -448,6 +464,7 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
         uint32_t aux = 0;
 #pragma unroll
         for (int e = 0; e < B::EL; ++e) {  // fully unrolled: constant register indices and shifts
+          if (e == B::EL / 2 && split) load_half(0);  // the first half of `cur` is consumed
           if ((mask >> e) & 1ull) {
             pieces[e * 32 + lane] = T::finish(PartOf<T>::to_acc(a), aux);
             a = PartOf<T>::ident();
@@ -458,7 +475,8 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
         tv = T::finish(PartOf<T>::to_acc(a), aux);
       }
     }
-    load_data(c + 1);  // `cur` is consumed: the next chunk's loads fly from here
+    if (split) load_half(1);
+    else load_data(c + 1);  // `cur` is consumed: the next chunk's loads fly from here  // `cur` is consumed: the next chunk's loads fly from here
     if (ovf) {
       const long long sn = k.s_next;
       k = bal_chunk_walk<T>(p, clo, chi, E0, E1, s0, lane);
