@@ -154,6 +154,20 @@ struct BalRanges {
   }
 };
 
+// BalRanges in 32-bit arithmetic for the scan (chunk counts below 2^31: inline
+// 32-bit divisions instead of the 64-bit division routine; the per-segment form
+// of round 1 diverged on that arithmetic, 4.3 of the scan's 7.4 us)
+struct BalRanges32 {
+  unsigned per, rem, t;
+  __device__ BalRanges32(unsigned nchunks, unsigned nranges)
+      : per(nchunks / nranges), rem(nchunks % nranges), t(rem * (per + 1u)) {}
+  __device__ unsigned begin(unsigned w) const { return w * per + (w < rem ? w : rem); }
+  __device__ unsigned first_at(unsigned c) const {
+    if (per == 0) return c;
+    return c <= t ? (c + per) / (per + 1u) : rem + (c - t + per - 1u) / per;
+  }
+};
+
 template <int DT, int OP, int K>
 __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
   using T = Tr<DT, OP>;
@@ -163,22 +177,7 @@ __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
   const long long E0 = __ldg(p.offsets), E1 = __ldg(p.offsets + p.nseg);
   const long long P0 = bal_origin<B::s>(p.in, E0);
   const long long nchunks = E1 > E0 ? (E1 - P0 + B::C - 1) / B::C : 0;
-  const BalRanges R(nchunks > 0 ? nchunks : 1, p.b.nranges);
-  auto one = [&](long long i, long long lo, long long hi) {
-    if (hi < lo) atomicOr(p.b.hdr, 1u);
-    if (hi <= lo) {
-      seg_store<T>(p, i, T::gident());
-    } else if (nchunks > 0) {
-      // start_seg[w] = i for the ranges whose first chunk starts in [lo, hi)
-      // (chunk 0 starts at E0, chunk c > 0 at P0 + c*C)
-      const long long c0 = lo <= E0 ? 0 : (lo - P0 + B::C - 1) / B::C;
-      long long c1 = (hi - P0 + B::C - 1) / B::C;
-      if (c1 > nchunks) c1 = nchunks;
-      if (c0 < c1) {  // only segments holding a chunk start (the range arithmetic divides)
-        for (long long w = R.first_at(c0); w < p.b.nranges && R.begin(w) < c1; ++w) p.b.start_seg[w] = (unsigned)i;
-      }
-    }
-  };
+  const bool narrow = nchunks < (1ll << 31) && p.b.nranges < (1ll << 31);
   // K consecutive segments per thread per step (K from the host: the fewest
   // steps for the grid), their K + 1 offsets loaded before any is used -- the
   // loop is latency-bound, one round trip per step
@@ -188,9 +187,48 @@ __global__ void __launch_bounds__(256) k_segbal_scan(const SegParams p) {
     long long o[K + 1];
 #pragma unroll
     for (int j = 0; j <= K; ++j) o[j] = i0 + j <= p.nseg ? __ldg(p.offsets + i0 + j) : LLONG_MAX;
+    // the identity for empty segments, the flag for decreasing offsets
 #pragma unroll
-    for (int j = 0; j < K; ++j)
-      if (i0 + j < p.nseg) one(i0 + j, o[j], o[j + 1]);
+    for (int j = 0; j < K; ++j) {
+      if (i0 + j < p.nseg) {
+        if (o[j + 1] < o[j]) atomicOr(p.b.hdr, 1u);
+        if (o[j + 1] <= o[j]) seg_store<T>(p, i0 + j, T::gident());
+      }
+    }
+    // start_seg[w] for the ranges whose first chunk starts in this thread's
+    // elements [o[0], o[K'])  (chunk 0 starts at E0, chunk c > 0 at P0 + c*C;
+    // once per thread, not per segment: the per-segment form diverged on the
+    // range arithmetic, 4.3 of the scan's 7.4 us)
+    if (nchunks > 0) {
+      const long long kv = p.nseg - i0 < K ? p.nseg - i0 : K;  // segments this thread holds
+      long long hi = o[0];
+#pragma unroll
+      for (int j = 1; j <= K; ++j)
+        if (j <= kv) hi = o[j];
+      const long long lo = o[0];
+      const long long c0 = lo <= E0 ? 0 : (long long)((unsigned long long)(lo - P0 + B::C - 1) / B::C);
+      long long c1 = hi <= E0 ? 0 : (long long)((unsigned long long)(hi - P0 + B::C - 1) / B::C);
+      if (c1 > nchunks) c1 = nchunks;
+      if (c0 < c1) {
+        auto claim = [&](long long w, long long cs) {
+          const long long pos = cs == 0 ? E0 : P0 + cs * B::C;
+          // the non-empty segment holding pos: the last j with o[j] <= pos
+          int js = 0;
+#pragma unroll
+          for (int j = 1; j < K; ++j)
+            if (j < kv && o[j] <= pos) js = j;
+          p.b.start_seg[w] = (unsigned)(i0 + js);
+        };
+        if (narrow) {
+          const BalRanges32 R((unsigned)nchunks, (unsigned)p.b.nranges);
+          for (unsigned w = R.first_at((unsigned)c0); w < (unsigned)p.b.nranges && R.begin(w) < (unsigned)c1; ++w)
+            claim(w, R.begin(w));
+        } else {
+          const BalRanges R(nchunks, p.b.nranges);
+          for (long long w = R.first_at(c0); w < p.b.nranges && R.begin(w) < c1; ++w) claim(w, R.begin(w));
+        }
+      }
+    }
   }
   pdl_trigger();
 }
