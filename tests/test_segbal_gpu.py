@@ -292,3 +292,36 @@ def test_concurrent_streams_independent_workspaces():
         want = _reduceat(x, offs, "sum")
         want = ((want + 2 ** 31) % 2 ** 32 - 2 ** 31).astype(np.int32)
         assert (o.cpu().numpy() == want).all()
+
+
+@pytest.mark.parametrize("lead", [0, 1, 5, 37])
+def test_many_segments_scan_instances(lead):
+    """Segment counts that select the scan kernel's K = 1 / 4 / 8 segments per
+    thread (nseg up to ~1.6 M), with `lead` empty segments first, runs of 3-11
+    empty segments that straddle the scan threads' K-segment groups, a segment
+    spanning many warp ranges and single-element segments: every range start
+    the scan claims (once per thread, round 2) must be the non-empty segment
+    holding the range's first element.  int32 sum (mod 2^32) / max bit-exact
+    against numpy reduceat, misaligned input."""
+    import torch
+    import paper_conf_cgo_gonzalohghmh19_b200 as rb
+    rng = np.random.Generator(np.random.PCG64(500 + lead))
+    for nseg in (200_000, 700_000, 1_600_000):
+        lens = rng.integers(1, 40, nseg)
+        lens[:lead] = 0
+        for start in rng.integers(lead, nseg - 20, 300):  # empty runs of 3..11
+            lens[start:start + rng.integers(3, 12)] = 0
+        lens[nseg // 2] = 3_000_000  # one segment across many ranges
+        lens[nseg // 3: nseg // 3 + 5000] = 1
+        offs = np.concatenate([[7], 7 + np.cumsum(lens)])
+        n = int(offs[-1]) + 5
+        x = synth.make("int32", n, "int_full", 70 + lead)
+        xt = torch.empty(n + 1, dtype=torch.int32, device="cuda")[1:]
+        xt.copy_(torch.from_numpy(x))
+        ot = torch.from_numpy(offs).cuda()
+        for op in ("sum", "max"):
+            got = rb.reduce_segmented(xt, ot, op).cpu().numpy()
+            want = _reduceat(x, offs, op)
+            if op == "sum":
+                want = ((want + 2 ** 31) % 2 ** 32 - 2 ** 31).astype(np.int32)
+            assert (got == want.astype(np.int32)).all(), (nseg, op, np.nonzero(got != want)[0][:5])
