@@ -161,8 +161,12 @@ __device__ __forceinline__ void hist_vec(const uint32_t (&r)[8], const HistParam
 // copies per bin, reading the whole input -- `parts` passes over the data
 // instead of one global atomic per element.  !kShared: every element is one
 // global atomic (very many bins).
+#ifndef RB_HIST_MINB_I32
+#define RB_HIST_MINB_I32 4  // int32 shared bins at 64 registers: 4 blocks per SM (256 bins 198.7 -> 173.3 us, profiles/r02_hist_i32_minb_ab.txt)
+#endif
 template <int DT, bool kShared>
-__global__ void __launch_bounds__(256) k_histogram(const HistParams p, int parts, int rep_log2) {
+__global__ void __launch_bounds__(256, (DT == DT_I32 && kShared) ? RB_HIST_MINB_I32 : 1)
+    k_histogram(const HistParams p, int parts, int rep_log2) {
   extern __shared__ unsigned sbins[];
   int b0 = 0, b1 = p.nbins;
   unsigned blk = blockIdx.x, nblk = gridDim.x;
