@@ -133,7 +133,7 @@ constexpr size_t kBalHdrBytes = 256;
 constexpr size_t kBalBytes = kBalHdrBytes + (size_t)kBalRanges * (4 /* start_seg */ + 16 /* first */ +
                                                                    16 /* last */ + 4 /* last_seg */ + 4 /* flags */);
 struct SegBal {
-  unsigned* hdr;         // [0] non-monotone offsets seen, [1] fix-up ticket (both self-resetting)
+  unsigned* hdr;         // [0] non-monotone offsets seen (set by the scan, cleared by the fix-up kernel)
   unsigned* start_seg;   // [w]: the segment holding range w's first element
   void* first_val;       // Grid[w]: range w's piece of the segment open at its start
   void* last_val;        // Grid[w]: range w's piece of the segment still open at its end

@@ -368,6 +368,10 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
       const Acc w = bal_warp_range<T>(p, lo, hi, lane);
       if (lane == 0) seg_store<T>(p, seg, T::to_grid(w));
     }
+    if (lane == 0) {  // no range pieces: the fix-up joins nothing
+      p.b.flags[gw] = 0u;
+      p.b.last_seg[gw] = 0xFFFFFFFFu;
+    }
     pdl_trigger();
     return;
   }
@@ -588,16 +592,20 @@ __global__ void __launch_bounds__(kBalWarps * 32, bal_min_blocks(DT, OP)) k_segb
 
 // One warp per range whose last piece opens a segment: joins it with the
 // first pieces of the following ranges up to the one where the segment closes
-// (32 ranges per step, fixed order).  The last block resets the call's flags.
+// (32 ranges per step, fixed order).  Block 0 clears the call's non-monotone
+// flag: every reader (the chunk kernel) has completed, and the chunk kernel's
+// fallback leaves no open range pieces, so this kernel never needs the flag
+// (round 2: no end-of-call ticket, fix 3.7 -> 2.7 us,
+// profiles/r02_segbal_fix_noticket_ab.txt).
 template <int DT, int OP>
 __global__ void __launch_bounds__(256) k_segbal_fix(const SegParams p) {
   using T = Tr<DT, OP>;
   using Grid = typename T::Grid;
   pdl_wait();
-  const unsigned nonmono = *(volatile unsigned*)p.b.hdr;
+  if (blockIdx.x == 0 && threadIdx.x == 0) p.b.hdr[0] = 0u;
   const long long nr = p.b.nranges;
   const int lane = threadIdx.x & 31;
-  if (!nonmono) {
+  {
     const long long nw = (long long)gridDim.x * (blockDim.x >> 5);
     const Grid* fv = (const Grid*)p.b.first_val;
 #pragma unroll 1
@@ -633,11 +641,6 @@ __global__ void __launch_bounds__(256) k_segbal_fix(const SegParams p) {
       }
       if (lane == 0) seg_store<T>(p, ls, x);
     }
-  }
-  __syncthreads();
-  if (threadIdx.x == 0 && ticket_acq_rel(p.b.hdr + 1) == gridDim.x - 1) {
-    p.b.hdr[0] = 0u;
-    p.b.hdr[1] = 0u;
   }
   pdl_trigger();
 }
