@@ -47,6 +47,9 @@ constexpr int kHistSharedMaxBins = 16384;  // 64 KB of u32 counters per block
 #ifndef RB_HIST16_RED
 #define RB_HIST16_RED 1
 #endif
+#ifndef RB_HIST16_ONE_BARRIER
+#define RB_HIST16_ONE_BARRIER 1
+#endif
 #ifndef RB_HIST16_ROLL
 #define RB_HIST16_ROLL 1
 #endif
@@ -397,7 +400,14 @@ __global__ void __launch_bounds__(1024) k_histogram16r(const HistParams p) {
         }
       }
     }
+#if !RB_HIST16_ONE_BARRIER
     __syncthreads();
+#endif
+    // (round 2: no barrier after the scan.  Between two scans of a word only
+    // one iteration's updates land -- the first barrier orders every update of
+    // iteration i before the scan of flush i, and a thread starts iteration i+1
+    // only after its own part of that scan -- and the scan's subtraction only
+    // removes what it read, so a half stays < T + E <= 0xFFFF as before.)
   };
   const unsigned long long stride = (unsigned long long)gridDim.x * blockDim.x;
   unsigned long long v = (unsigned long long)blockIdx.x * blockDim.x + threadIdx.x;
