@@ -50,8 +50,24 @@ def _deps() -> list[str]:
             + glob.glob(os.path.join(CSRC, "*.inc")) + [os.path.join(ROOT, "include", "reduce.h"), __file__])
 
 
+STAMP = os.path.join(BUILD, "flags.stamp")  # the experiment flags the in-tree library was built with
+
+
+def _extra_flags() -> str:
+    return " ".join(os.environ.get("REDUCE_B200_NVCC_FLAGS", "").split())
+
+
 def up_to_date() -> bool:
+    """The in-tree library is newer than every source AND was built with the
+    current experiment flags (an A/B build with -D... flags is never reused by a
+    default build, and the reverse)."""
     if not os.path.exists(LIB):
+        return False
+    try:
+        with open(STAMP) as fh:
+            if fh.read().strip() != _extra_flags():
+                return False
+    except OSError:
         return False
     t = os.path.getmtime(LIB)
     return all(os.path.getmtime(d) <= t for d in _deps())
@@ -85,6 +101,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
     os.replace(tmp, LIB)
+    with open(STAMP, "w") as fh:
+        fh.write(_extra_flags() + "\n")
     return LIB
 
 
