@@ -65,7 +65,10 @@ namespace rb {
 #ifndef RB_SEGBAL_SPLIT
 #define RB_SEGBAL_SPLIT 1
 #endif
-constexpr int kBalWarps = 4;                    // warps per block of k_segbal
+#ifndef RB_SEGBAL_WARPS
+#define RB_SEGBAL_WARPS 4
+#endif
+constexpr int kBalWarps = RB_SEGBAL_WARPS;      // warps per block of k_segbal
 // resident blocks asked of ptxas: 5 (96 registers, 20 warps per SM) for the
 // 4-byte plain ops; fp64 and accurate sums need more registers (4 blocks)
 constexpr int bal_min_blocks(int dt, int op) { return (dt != 2 && op != 3) ? RB_SEGBAL_MINB : 4; }
